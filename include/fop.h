@@ -1,0 +1,236 @@
+/*
+ * fop.h — C ABI of the B200-native fused-operator library (libfop.so).
+ *
+ * A fused AI/DL operator is given the way the paper states its problem
+ * (§II-§III): an ordered list of STATEMENTS over
+ * TENSORS.  Each statement runs over a box iteration domain
+ * D_S(p) = { i | 0 <= i_l < E_l } (eqs for D_X, D_Y), has one write
+ * access and several read accesses, and an expression DAG (the abstract
+ * f, g of Fig. 2).  Access functions are "either a constant or an
+ * affine form where only one loop iterator is present with coefficient 1"
+ * — that is exactly fop_access below.
+ *
+ * Reading (reading D1): loops are declared once for the whole fused
+ * operator (fop_desc.extent[]) and each statement lists the loops it iterates,
+ * outermost first.  Two statements that list the same loop id share that
+ * iterator (the i/k of Fig. 2's X and Y).  This is how the dependence relation
+ * delta_{X->Y} of P:149 (i_X = i_Y, k_X = k_Y) is expressed without isl.
+ *
+ * Semantics (what every result must equal, checked against oracle/):
+ * statements execute in textual order; each iterates its loops in
+ * lexicographic order (the schedule theta of P:119-121); ASSIGN stores the DAG
+ * value converted (RNE) to the write tensor's dtype; REDUCE overwrites each
+ * output element with op-reduce over the statement's reduction loops (loops on
+ * which the write access does not depend) of the DAG value, then applies the
+ * finalize DAG (e.g. /768 for a mean); a later statement reads the STORED
+ * (rounded) values.  Arithmetic nodes are fp32; add/sub/mul/div/sqrt are IEEE
+ * correctly rounded and never contracted.
+ *
+ * Ownership: the caller owns every buffer (host descriptors, device tensors,
+ * workspace).  fop_plan copies the descriptor; a plan is immutable after
+ * fop_plan returns and may be run concurrently on several streams (only the
+ * lazy per-context module load takes an internal lock).  No function throws or
+ * aborts across the ABI: every failure is a fop_status plus a thread-local
+ * message (fop_last_error).
+ */
+#ifndef FOP_H
+#define FOP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FOP_ABI_VERSION 1
+
+#define FOP_MAX_RANK     8   /* tensor rank */
+#define FOP_MAX_LOOPS    8   /* loops of the fused operator */
+#define FOP_MAX_TENSORS 16
+#define FOP_MAX_STMTS    8
+#define FOP_MAX_ACC      8   /* accesses per statement; acc[0] is the write */
+#define FOP_MAX_NODES   48   /* DAG nodes per statement */
+#define FOP_MAX_FIN      8   /* finalize nodes per REDUCE statement */
+#define FOP_MAX_LAUNCH   8   /* kernel launches per plan */
+#define FOP_MAX_SCEN     8   /* scenarios kept per statement ("set to 8") */
+
+typedef enum {
+  FOP_OK = 0,
+  FOP_E_INVALID = 1,     /* malformed descriptor / arguments */
+  FOP_E_UNSUPPORTED = 2, /* valid, but outside what the kernels implement */
+  FOP_E_ALIGN = 3,       /* pointer alignment violates the tensor dtype itself */
+  FOP_E_CUDA = 4,        /* CUDA driver failure (no driver, launch error, ...) */
+  FOP_E_NOMEM = 5,
+  FOP_E_JIT = 6          /* NVRTC compilation of a generated kernel failed */
+} fop_status;
+
+typedef enum { FOP_F32 = 0, FOP_F16 = 1, FOP_BF16 = 2, FOP_I32 = 3 } fop_dtype;
+
+/* IN: read only.  OUT: written.  INOUT: read and written.  TEMP: an
+ * intermediate of the fused operator (graph-kernel fusion removes
+ * intermediate allocations); its pointer may be NULL — the plan either
+ * keeps it in registers or places it in the workspace. */
+typedef enum { FOP_IN = 1, FOP_OUT = 2, FOP_INOUT = 3, FOP_TEMP = 4 } fop_role;
+
+typedef enum { FOP_ASSIGN = 0, FOP_REDUCE = 1 } fop_kind;
+typedef enum { FOP_RED_SUM = 0, FOP_RED_MAX = 1 } fop_reduce_op;
+
+typedef enum {
+  FOP_OP_LOAD = 0,      /* a = read access index (1..nacc-1) */
+  FOP_OP_CONST = 1,     /* imm (fp32) */
+  FOP_OP_ACC = 2,       /* finalize DAG only: the reduced value */
+  FOP_OP_ADD = 3, FOP_OP_SUB = 4, FOP_OP_MUL = 5, FOP_OP_DIV = 6,
+  FOP_OP_MAX = 7, FOP_OP_MIN = 8,          /* fmaxf/fminf semantics */
+  FOP_OP_NEG = 9, FOP_OP_ABS = 10, FOP_OP_SQRT = 11,
+  FOP_OP_RELU = 12,     /* v > 0 ? v : +0 (reading R15) */
+  FOP_OP_EXP = 13, FOP_OP_LOG = 14, FOP_OP_TANH = 15, FOP_OP_SIGMOID = 16,
+  FOP_OP_GELU_TANH = 17, /* 0.5 v (1 + tanh(sqrt(2/pi)(v + 0.044715 v^3))) */
+  FOP_OP_GELU_ERF = 18,  /* 0.5 v (1 + erf(v / sqrt 2)) */
+  FOP_OP_CAST = 19,      /* round a to dtype `cvt`, value continues as fp32 */
+  FOP_OP__COUNT = 20
+} fop_opcode;
+
+typedef struct {
+  int32_t rank;
+  int32_t dtype;                 /* fop_dtype */
+  int32_t role;                  /* fop_role */
+  int32_t _pad;
+  int64_t shape[FOP_MAX_RANK];
+  int64_t stride[FOP_MAX_RANK];  /* in ELEMENTS; 0 allowed (expand-style broadcast) */
+} fop_tensor;
+
+/* index_r = (loop[r] >= 0 ? i_{loop[r]} : 0) + offset[r]     (P:355 access form) */
+typedef struct {
+  int32_t tensor;
+  int32_t loop[FOP_MAX_RANK];    /* global loop id per tensor dim, -1 = constant */
+  int64_t offset[FOP_MAX_RANK];
+} fop_access;
+
+typedef struct {
+  int32_t op;                    /* fop_opcode */
+  int32_t a, b;                  /* operand node indices (earlier nodes) or access index */
+  int32_t cvt;                   /* fop_dtype for FOP_OP_CAST */
+  float imm;                     /* FOP_OP_CONST */
+  int32_t _pad;
+} fop_node;
+
+typedef struct {
+  int32_t kind;                  /* fop_kind */
+  int32_t reduce_op;             /* fop_reduce_op (REDUCE only) */
+  int32_t nloops;
+  int32_t loop[FOP_MAX_LOOPS];   /* loop ids, outermost first (original nest order) */
+  int32_t nacc;
+  fop_access acc[FOP_MAX_ACC];   /* acc[0] = write access */
+  int32_t nnodes;
+  fop_node node[FOP_MAX_NODES];  /* topological; the statement value is the last node */
+  int32_t nfin;
+  fop_node fin[FOP_MAX_FIN];     /* REDUCE finalize DAG over FOP_OP_ACC/CONST; empty = identity */
+} fop_stmt;
+
+typedef struct {
+  int32_t nloops;
+  int64_t extent[FOP_MAX_LOOPS]; /* E_l >= 1 (box domain) */
+  int32_t ntensors;
+  fop_tensor t[FOP_MAX_TENSORS];
+  int32_t nstmts;
+  fop_stmt s[FOP_MAX_STMTS];
+} fop_desc;
+
+/* Planner options.  fop_plan_opts_default() fills the paper's values:
+ * W = (5,3,1,1,1), L = 1024 (reading R5), 8 scenarios,
+ * 16-byte vectors (128-bit), readings R1 + R6 on. */
+enum {
+  FOP_READING_R1_THREAD_TERM = 1,  /* w5*F*N/L instead of the printed w5*F*L/N (P:338 vs P:347) */
+  FOP_READING_R6_STRIDE1_C   = 2   /* |C| counts only stride-1 accesses */
+};
+enum { FOP_ORDER_PAPER = 0, FOP_ORDER_MEMORY = 1 };
+
+typedef struct {
+  double w[5];
+  int32_t thread_limit;          /* L of Algorithm 2 */
+  int32_t max_scenarios;
+  int32_t max_vec_bytes;         /* 16 (LDG/STG.128) or 32 (LDG/STG.256, sm_100a) */
+  int32_t readings;              /* FOP_READING_* bit set */
+  int32_t force_width;           /* 0 = planner decides; k = cap vector width at k elements (1 = "novec") */
+  int32_t coalesce_order;        /* FOP_ORDER_PAPER: threads follow the scenario order; MEMORY: write-memory order */
+  int32_t sm_count;              /* 0 = 148 (B200); used for grid sizing */
+  int32_t jit;                   /* 1 = compile kernels at fop_plan (NVRTC, sm_100a); 0 = analysis only */
+} fop_plan_opts;
+
+typedef enum {
+  FOP_CLASS_EW = 0,          /* elementwise / broadcast */
+  FOP_CLASS_TRANSPOSE = 1,   /* store-contiguous loop != load-contiguous loop */
+  FOP_CLASS_ROW_REDUCE = 2,  /* vector loop is a reduction loop */
+  FOP_CLASS_COL_REDUCE = 3   /* vector loop is parallel, reduction elsewhere */
+} fop_kernel_class;
+
+typedef struct {
+  int32_t kernel_class;      /* fop_kernel_class */
+  int32_t main_stmt;
+  uint32_t stmt_mask;        /* statements fused into this launch (bit s) */
+  int32_t vec_loop;          /* loop id carrying the explicit vector type */
+  int32_t width;             /* elements per vector access on the write side */
+  int32_t read_loop;         /* TRANSPOSE: loop contiguous for the transposed read, else -1 */
+  int32_t read_width;        /* TRANSPOSE: elements per read vector */
+  int32_t coal_loop;         /* next loop mapped to threads (scenario goal (ii)), -1 if none */
+  int64_t grid;
+  int32_t block;
+  int32_t _pad;
+} fop_launch_info;
+
+typedef struct {
+  int32_t nstmts;
+  int32_t nscen[FOP_MAX_STMTS];                        /* scenarios kept per statement */
+  int32_t scen_len[FOP_MAX_STMTS][FOP_MAX_SCEN];
+  int32_t scenario[FOP_MAX_STMTS][FOP_MAX_SCEN][3];    /* loop ids, outermost -> innermost */
+  double  inner_score[FOP_MAX_STMTS][FOP_MAX_LOOPS];   /* cost at the innermost position, by stmt loop position */
+  int32_t nlaunch;
+  fop_launch_info launch[FOP_MAX_LAUNCH];
+  size_t  workspace_bytes;
+} fop_plan_info;
+
+typedef struct fop_plan fop_plan_t;   /* opaque, immutable after fop_plan */
+
+int         fop_abi_version(void);
+void        fop_plan_opts_default(fop_plan_opts* opts);
+
+/* Validate the descriptor (row a1), analyse strides (a2), rank scenarios with
+ * Algorithm 2 + cost() (a3), choose widths (a4), kernel classes and
+ * launches (a5), generate and (opts->jit) compile the kernels for sm_100a.
+ * Host only: needs neither a GPU nor a CUDA context.  opts may be NULL
+ * (= fop_plan_opts_default).  On failure *out is NULL. */
+fop_status  fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t** out);
+fop_status  fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* out);
+size_t      fop_plan_workspace_bytes(const fop_plan_t* plan);
+/* Generated CUDA source / compiled cubin of launch i (inspection, tests).
+ * Pointers stay owned by the plan. */
+fop_status  fop_plan_source(const fop_plan_t* plan, int32_t launch, const char** src);
+fop_status  fop_plan_cubin(const fop_plan_t* plan, int32_t launch, const void** data, size_t* size);
+
+/* Run the fused operator.  dev_ptrs[i] = device base address of desc.t[i]
+ * (NULL allowed for TEMP tensors), nptrs = desc.ntensors.  workspace: device
+ * buffer of fop_plan_workspace_bytes() bytes, ZERO-FILLED before its first use
+ * with this plan (kernels leave it zeroed again), NULL if 0 bytes.
+ * stream: a CUstream / cudaStream_t (NULL = legacy default stream) of the
+ * CURRENT CUDA context.  Asynchronous and stream-ordered.  A base pointer that
+ * is not aligned for the planned vector width silently selects a narrower
+ * variant (same bits).  Returns FOP_E_CUDA if the driver or launch fails. */
+fop_status  fop_run(const fop_plan_t* plan, void* const* dev_ptrs, int32_t nptrs,
+                    void* workspace, void* stream);
+
+/* End-to-end variant: host_ptrs[i] are PINNED host buffers (dense, same
+ * layout as desc.t[i]); IN/INOUT tensors are copied host->device, the
+ * operator runs, OUT/INOUT tensors are copied device->host, all enqueued on
+ * `stream`.  The caller synchronises the stream before reading host_ptrs. */
+fop_status  fop_run_host(const fop_plan_t* plan, void* const* host_ptrs,
+                         void* const* dev_ptrs, int32_t nptrs, void* workspace, void* stream);
+
+void        fop_plan_destroy(fop_plan_t* plan);
+const char* fop_status_str(fop_status s);
+const char* fop_last_error(void);      /* thread-local detail of the last failure */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FOP_H */
