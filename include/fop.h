@@ -43,6 +43,12 @@
 extern "C" {
 #endif
 
+#if defined(__GNUC__)
+#define FOP_API __attribute__((visibility("default")))
+#else
+#define FOP_API
+#endif
+
 #define FOP_ABI_VERSION 1
 
 #define FOP_MAX_RANK     8   /* tensor rank */
@@ -192,21 +198,21 @@ typedef struct {
 
 typedef struct fop_plan fop_plan_t;   /* opaque, immutable after fop_plan */
 
-int         fop_abi_version(void);
-void        fop_plan_opts_default(fop_plan_opts* opts);
+FOP_API int         fop_abi_version(void);
+FOP_API void        fop_plan_opts_default(fop_plan_opts* opts);
 
 /* Validate the descriptor (row a1), analyse strides (a2), rank scenarios with
  * Algorithm 2 + cost() (a3), choose widths (a4), kernel classes and
  * launches (a5), generate and (opts->jit) compile the kernels for sm_100a.
  * Host only: needs neither a GPU nor a CUDA context.  opts may be NULL
  * (= fop_plan_opts_default).  On failure *out is NULL. */
-fop_status  fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t** out);
-fop_status  fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* out);
-size_t      fop_plan_workspace_bytes(const fop_plan_t* plan);
+FOP_API fop_status  fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t** out);
+FOP_API fop_status  fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* out);
+FOP_API size_t      fop_plan_workspace_bytes(const fop_plan_t* plan);
 /* Generated CUDA source / compiled cubin of launch i (inspection, tests).
  * Pointers stay owned by the plan. */
-fop_status  fop_plan_source(const fop_plan_t* plan, int32_t launch, const char** src);
-fop_status  fop_plan_cubin(const fop_plan_t* plan, int32_t launch, const void** data, size_t* size);
+FOP_API fop_status  fop_plan_source(const fop_plan_t* plan, int32_t launch, const char** src);
+FOP_API fop_status  fop_plan_cubin(const fop_plan_t* plan, int32_t launch, const void** data, size_t* size);
 
 /* Run the fused operator.  dev_ptrs[i] = device base address of desc.t[i]
  * (NULL allowed for TEMP tensors), nptrs = desc.ntensors.  workspace: device
@@ -216,19 +222,19 @@ fop_status  fop_plan_cubin(const fop_plan_t* plan, int32_t launch, const void** 
  * CURRENT CUDA context.  Asynchronous and stream-ordered.  A base pointer that
  * is not aligned for the planned vector width silently selects a narrower
  * variant (same bits).  Returns FOP_E_CUDA if the driver or launch fails. */
-fop_status  fop_run(const fop_plan_t* plan, void* const* dev_ptrs, int32_t nptrs,
+FOP_API fop_status  fop_run(const fop_plan_t* plan, void* const* dev_ptrs, int32_t nptrs,
                     void* workspace, void* stream);
 
 /* End-to-end variant: host_ptrs[i] are PINNED host buffers (dense, same
  * layout as desc.t[i]); IN/INOUT tensors are copied host->device, the
  * operator runs, OUT/INOUT tensors are copied device->host, all enqueued on
  * `stream`.  The caller synchronises the stream before reading host_ptrs. */
-fop_status  fop_run_host(const fop_plan_t* plan, void* const* host_ptrs,
+FOP_API fop_status  fop_run_host(const fop_plan_t* plan, void* const* host_ptrs,
                          void* const* dev_ptrs, int32_t nptrs, void* workspace, void* stream);
 
-void        fop_plan_destroy(fop_plan_t* plan);
-const char* fop_status_str(fop_status s);
-const char* fop_last_error(void);      /* thread-local detail of the last failure */
+FOP_API void        fop_plan_destroy(fop_plan_t* plan);
+FOP_API const char* fop_status_str(fop_status s);
+FOP_API const char* fop_last_error(void);      /* thread-local detail of the last failure */
 
 #ifdef __cplusplus
 }

@@ -1,0 +1,194 @@
+// abi.cpp — the extern "C" entry points declared in include/fop.h.
+// Every entry point converts internal failures into a fop_status plus a
+// thread-local message; nothing throws or aborts across the ABI.
+#include <cstring>
+#include <exception>
+#include <new>
+#include <string>
+
+#include "fop_internal.h"
+
+struct fop_plan {
+  fop::Plan p;
+};
+
+namespace fop {
+static thread_local std::string g_err;
+void set_error(const std::string& msg) { g_err = msg; }
+void fail(fop_status s, const std::string& msg) { throw Error{s, msg}; }
+}  // namespace fop
+
+template <class F>
+static fop_status guarded(F&& f) {
+  try {
+    return f();
+  } catch (const fop::Error& e) {
+    fop::set_error(e.msg);
+    return e.status;
+  } catch (const std::bad_alloc&) {
+    fop::set_error("out of host memory");
+    return FOP_E_NOMEM;
+  } catch (const std::exception& e) {
+    fop::set_error(e.what());
+    return FOP_E_INVALID;
+  } catch (...) {
+    fop::set_error("unknown internal error");
+    return FOP_E_INVALID;
+  }
+}
+
+extern "C" {
+
+int fop_abi_version(void) { return FOP_ABI_VERSION; }
+
+void fop_plan_opts_default(fop_plan_opts* o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof *o);
+  o->w[0] = 5;  // w1: store vectorisation
+  o->w[1] = 3;  // w2: load vectorisation
+  o->w[2] = 1;  // w3: 1/M, short jumps
+  o->w[3] = 1;  // w4: |C|, many stride-1 accesses
+  o->w[4] = 1;  // w5: thread term
+  o->thread_limit = 1024;  // R5
+  o->max_scenarios = 8;
+  o->max_vec_bytes = 16;   // 128-bit vector types
+  o->readings = FOP_READING_R1_THREAD_TERM | FOP_READING_R6_STRIDE1_C;
+  o->force_width = 0;
+  o->coalesce_order = FOP_ORDER_PAPER;
+  o->sm_count = 148;
+  o->jit = 1;
+}
+
+fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t** out) {
+  if (out) *out = nullptr;
+  return guarded([&] {
+    if (!desc || !out) fop::fail(FOP_E_INVALID, "NULL descriptor or output pointer");
+    auto* h = new struct fop_plan();
+    try {
+      fop::Plan& p = h->p;
+      std::memcpy(&p.desc, desc, sizeof *desc);
+      if (opts) std::memcpy(&p.opts, opts, sizeof *opts);
+      else fop_plan_opts_default(&p.opts);
+      if (p.opts.thread_limit <= 0) fop::fail(FOP_E_INVALID, "thread_limit must be > 0");
+      if (p.opts.max_vec_bytes != 4 && p.opts.max_vec_bytes != 8 && p.opts.max_vec_bytes != 16 &&
+          p.opts.max_vec_bytes != 32)
+        fop::fail(FOP_E_INVALID, "max_vec_bytes must be 4, 8, 16 or 32");
+      fop::validate(p.desc);
+      fop::plan_launches(p);
+      // narrow (scalar) variants for misaligned base pointers: geometry now,
+      // compiled on first use; workspace sized for the larger of the two
+      p.narrow.clear();
+      for (size_t i = 0; i < p.launches.size(); i++) {
+        fop::Launch N = p.launches[i];
+        N.scalar_variant = true;
+        N.cubin.clear();
+        N.src.clear();
+        fop::finalize_launch_geometry(p, N);
+        N.ws_off = p.launches[i].ws_off;
+        if (N.ws_bytes > p.launches[i].ws_bytes) {
+          N.ws_off = (p.ws_bytes + 255) & ~size_t(255);
+          p.ws_bytes = N.ws_off + N.ws_bytes;
+        }
+        p.narrow.push_back(N);
+      }
+      for (size_t i = 0; i < p.launches.size(); i++) {
+        fop::generate(p, p.launches[i], (int)i);
+        if (p.opts.jit) fop::jit_compile(p.launches[i]);
+      }
+    } catch (...) {
+      delete h;
+      throw;
+    }
+    *out = h;
+    return FOP_OK;
+  });
+}
+
+fop_status fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* o) {
+  return guarded([&] {
+    if (!plan || !o) fop::fail(FOP_E_INVALID, "NULL argument");
+    const fop::Plan& p = plan->p;
+    std::memset(o, 0, sizeof *o);
+    o->nstmts = p.desc.nstmts;
+    for (int s = 0; s < p.desc.nstmts; s++) {
+      const fop::Scenarios& sc = p.scen[s];
+      o->nscen[s] = sc.nscen;
+      for (int k = 0; k < sc.nscen; k++) {
+        o->scen_len[s][k] = sc.len[k];
+        for (int q = 0; q < 3; q++) o->scenario[s][k][q] = q < sc.len[k] ? sc.loops[k][q] : -1;
+      }
+      for (int k = 0; k < p.desc.s[s].nloops; k++) o->inner_score[s][k] = sc.inner_score[k];
+    }
+    o->nlaunch = (int)p.launches.size();
+    for (size_t i = 0; i < p.launches.size() && i < FOP_MAX_LAUNCH; i++) {
+      const fop::Launch& L = p.launches[i];
+      fop_launch_info& li = o->launch[i];
+      li.kernel_class = L.kclass;
+      li.main_stmt = L.main_stmt;
+      li.stmt_mask = L.mask;
+      li.vec_loop = L.vec_loop;
+      li.width = L.width;
+      li.read_loop = L.read_loop;
+      li.read_width = L.read_width;
+      li.coal_loop = L.coal_loop;
+      li.grid = L.grid;
+      li.block = L.block;
+    }
+    o->workspace_bytes = p.ws_bytes;
+    return FOP_OK;
+  });
+}
+
+size_t fop_plan_workspace_bytes(const fop_plan_t* plan) { return plan ? plan->p.ws_bytes : 0; }
+
+fop_status fop_plan_source(const fop_plan_t* plan, int32_t i, const char** src) {
+  return guarded([&] {
+    if (!plan || !src || i < 0 || i >= (int)plan->p.launches.size()) fop::fail(FOP_E_INVALID, "bad launch index");
+    *src = plan->p.launches[i].src.c_str();
+    return FOP_OK;
+  });
+}
+
+fop_status fop_plan_cubin(const fop_plan_t* plan, int32_t i, const void** data, size_t* size) {
+  return guarded([&] {
+    if (!plan || !data || !size || i < 0 || i >= (int)plan->p.launches.size())
+      fop::fail(FOP_E_INVALID, "bad launch index");
+    *data = plan->p.launches[i].cubin.data();
+    *size = plan->p.launches[i].cubin.size();
+    return FOP_OK;
+  });
+}
+
+fop_status fop_run(const fop_plan_t* plan, void* const* dev_ptrs, int32_t nptrs, void* workspace, void* stream) {
+  return guarded([&] {
+    if (!plan || !dev_ptrs) fop::fail(FOP_E_INVALID, "NULL plan or pointer table");
+    return fop::run_plan(const_cast<fop_plan_t*>(plan)->p, dev_ptrs, nptrs, workspace, stream, nullptr);
+  });
+}
+
+fop_status fop_run_host(const fop_plan_t* plan, void* const* host_ptrs, void* const* dev_ptrs, int32_t nptrs,
+                        void* workspace, void* stream) {
+  return guarded([&] {
+    if (!plan || !dev_ptrs || !host_ptrs) fop::fail(FOP_E_INVALID, "NULL plan or pointer table");
+    return fop::run_plan(const_cast<fop_plan_t*>(plan)->p, dev_ptrs, nptrs, workspace, stream, host_ptrs);
+  });
+}
+
+void fop_plan_destroy(fop_plan_t* plan) { delete plan; }
+
+const char* fop_status_str(fop_status s) {
+  switch (s) {
+    case FOP_OK: return "FOP_OK";
+    case FOP_E_INVALID: return "FOP_E_INVALID";
+    case FOP_E_UNSUPPORTED: return "FOP_E_UNSUPPORTED";
+    case FOP_E_ALIGN: return "FOP_E_ALIGN";
+    case FOP_E_CUDA: return "FOP_E_CUDA";
+    case FOP_E_NOMEM: return "FOP_E_NOMEM";
+    case FOP_E_JIT: return "FOP_E_JIT";
+  }
+  return "FOP_E_UNKNOWN";
+}
+
+const char* fop_last_error(void) { return fop::g_err.c_str(); }
+
+}  // extern "C"

@@ -1,0 +1,344 @@
+// fop_device.cuh — hand-written sm_100a device primitives of libfop.
+//
+// Every kernel libfop launches is one of four skeletons (EW, TRANSPOSE,
+// ROW_REDUCE, COL_REDUCE, see codegen.cpp) instantiated by the planner with
+// compile-time shapes, strides and the fused expression, then compiled by
+// NVRTC for sm_100a.  This header holds the pieces they are made of:
+//   * explicit vector loads/stores — the "explicit vector types" of the
+//     paper's backend vectorisation pass on B200:
+//     LDG/STG.128 (16 B) and LDG/STG.256 (32 B, sm_100a only) issued as PTX;
+//     streaming tensors bypass L1 (ld.global.nc.L1::no_allocate);
+//   * exact fp16/bf16 <-> fp32 conversions (cvt.rn, packed f16x2/bf16x2);
+//   * the fp32 operator set of the descriptor DAG (IEEE add/sub/mul/div/sqrt
+//     via the _rn intrinsics: never contracted, bit-identical to the oracle);
+//   * warp butterfly reductions (every lane gets the same bits).
+// No CUDA headers: NVRTC compiles this with only its built-ins.
+#pragma once
+
+typedef unsigned int u32;
+typedef unsigned short u16;
+typedef unsigned long long u64;
+
+namespace fop {
+
+enum { F32 = 0, F16 = 1, BF16 = 2, I32 = 3 };
+enum { LD_STREAM = 0, LD_CACHED = 1, LD_COHERENT = 2 };
+enum { ST_DEFAULT = 0, ST_STREAM = 1 };
+
+template <int DT> struct ES { enum { v = (DT == F16 || DT == BF16) ? 2 : 4 }; };
+
+// ------------------------------------------------------------------ loads
+template <int CB, int POL>
+__device__ __forceinline__ void ldraw(u32* w, const char* p) {
+  if constexpr (CB == 32) {
+    if constexpr (POL == LD_STREAM)
+      asm volatile("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                   : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]),
+                     "=r"(w[6]), "=r"(w[7]) : "l"(p));
+    else if constexpr (POL == LD_CACHED)
+      asm volatile("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                   : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]),
+                     "=r"(w[6]), "=r"(w[7]) : "l"(p));
+    else
+      asm volatile("ld.global.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                   : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]),
+                     "=r"(w[6]), "=r"(w[7]) : "l"(p) : "memory");
+  } else if constexpr (CB == 16) {
+    if constexpr (POL == LD_STREAM)
+      asm volatile("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]) : "l"(p));
+    else if constexpr (POL == LD_CACHED)
+      asm volatile("ld.global.nc.v4.b32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]) : "l"(p));
+    else
+      asm volatile("ld.global.v4.b32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]) : "l"(p) : "memory");
+  } else if constexpr (CB == 8) {
+    if constexpr (POL == LD_STREAM)
+      asm volatile("ld.global.nc.L1::no_allocate.v2.b32 {%0,%1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "l"(p));
+    else if constexpr (POL == LD_CACHED)
+      asm volatile("ld.global.nc.v2.b32 {%0,%1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "l"(p));
+    else
+      asm volatile("ld.global.v2.b32 {%0,%1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "l"(p) : "memory");
+  } else {
+    static_assert(CB == 4, "chunk");
+    if constexpr (POL == LD_STREAM)
+      asm volatile("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(w[0]) : "l"(p));
+    else if constexpr (POL == LD_CACHED)
+      asm volatile("ld.global.nc.b32 %0, [%1];" : "=r"(w[0]) : "l"(p));
+    else
+      asm volatile("ld.global.b32 %0, [%1];" : "=r"(w[0]) : "l"(p) : "memory");
+  }
+}
+
+template <int POL>
+__device__ __forceinline__ u16 ld16(const char* p) {
+  u16 h;
+  if constexpr (POL == LD_STREAM)
+    asm volatile("ld.global.nc.L1::no_allocate.b16 %0, [%1];" : "=h"(h) : "l"(p));
+  else if constexpr (POL == LD_CACHED)
+    asm volatile("ld.global.nc.b16 %0, [%1];" : "=h"(h) : "l"(p));
+  else
+    asm volatile("ld.global.b16 %0, [%1];" : "=h"(h) : "l"(p) : "memory");
+  return h;
+}
+
+// ------------------------------------------------------------------ stores
+template <int CB, int POL>
+__device__ __forceinline__ void straw(char* p, const u32* w) {
+  if constexpr (CB == 32) {
+    if constexpr (POL == ST_STREAM)
+      asm volatile("st.global.cs.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(w[0]), "r"(w[1]),
+                   "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7]) : "memory");
+    else
+      asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(w[0]), "r"(w[1]),
+                   "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7]) : "memory");
+  } else if constexpr (CB == 16) {
+    if constexpr (POL == ST_STREAM)
+      asm volatile("st.global.cs.v4.b32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(w[0]), "r"(w[1]), "r"(w[2]),
+                   "r"(w[3]) : "memory");
+    else
+      asm volatile("st.global.v4.b32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(w[0]), "r"(w[1]), "r"(w[2]),
+                   "r"(w[3]) : "memory");
+  } else if constexpr (CB == 8) {
+    if constexpr (POL == ST_STREAM)
+      asm volatile("st.global.cs.v2.b32 [%0], {%1,%2};" ::"l"(p), "r"(w[0]), "r"(w[1]) : "memory");
+    else
+      asm volatile("st.global.v2.b32 [%0], {%1,%2};" ::"l"(p), "r"(w[0]), "r"(w[1]) : "memory");
+  } else {
+    static_assert(CB == 4, "chunk");
+    if constexpr (POL == ST_STREAM)
+      asm volatile("st.global.cs.b32 [%0], %1;" ::"l"(p), "r"(w[0]) : "memory");
+    else
+      asm volatile("st.global.b32 [%0], %1;" ::"l"(p), "r"(w[0]) : "memory");
+  }
+}
+
+__device__ __forceinline__ void st16(char* p, u16 h) {
+  asm volatile("st.global.b16 [%0], %1;" ::"l"(p), "h"(h) : "memory");
+}
+
+// ------------------------------------------------------------------ conversions
+__device__ __forceinline__ float h2f(u16 h) {
+  float f;
+  asm("cvt.f32.f16 %0, %1;" : "=f"(f) : "h"(h));
+  return f;
+}
+__device__ __forceinline__ float b2f(u16 h) { return __uint_as_float(((u32)h) << 16); }
+__device__ __forceinline__ u16 f2h(float f) {
+  u16 h;
+  asm("cvt.rn.f16.f32 %0, %1;" : "=h"(h) : "f"(f));
+  return h;
+}
+__device__ __forceinline__ u16 f2b(float f) {
+  u16 h;
+  asm("cvt.rn.bf16.f32 %0, %1;" : "=h"(h) : "f"(f));
+  return h;
+}
+// packed pairs: lo in bits 0..15
+__device__ __forceinline__ u32 f2h2(float lo, float hi) {
+  u32 r;
+  asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+__device__ __forceinline__ u32 f2b2(float lo, float hi) {
+  u32 r;
+  asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+
+template <int DT>
+__device__ __forceinline__ float round_to(float v) {
+  if constexpr (DT == F16) return h2f(f2h(v));
+  else if constexpr (DT == BF16) return b2f(f2b(v));
+  else return v;
+}
+
+// ------------------------------------------------------------------ typed vectors
+// N elements of type DT at p (aligned to CB bytes) -> fp32
+template <int DT, int N, int CB, int POL>
+__device__ __forceinline__ void vload(float* v, const char* p) {
+  constexpr int TOT = N * ES<DT>::v;
+  if constexpr (CB >= 4) {
+    u32 w[TOT / 4];
+#pragma unroll
+    for (int c = 0; c < TOT / CB; ++c) ldraw<CB, POL>(w + c * (CB / 4), p + c * CB);
+#pragma unroll
+    for (int i = 0; i < TOT / 4; ++i) {
+      if constexpr (DT == F32 || DT == I32) {
+        v[i] = __uint_as_float(w[i]);
+      } else if constexpr (DT == F16) {
+        v[2 * i] = h2f((u16)(w[i] & 0xffffu));
+        v[2 * i + 1] = h2f((u16)(w[i] >> 16));
+      } else {
+        v[2 * i] = __uint_as_float(w[i] << 16);
+        v[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u);
+      }
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+      u16 h = ld16<POL>(p + 2 * i);
+      v[i] = DT == F16 ? h2f(h) : b2f(h);
+    }
+  }
+}
+
+// fp32 -> N elements of type DT at p (RNE conversion)
+template <int DT, int N, int CB, int POL>
+__device__ __forceinline__ void vstore(char* p, const float* v) {
+  constexpr int TOT = N * ES<DT>::v;
+  if constexpr (CB >= 4) {
+    u32 w[TOT / 4];
+#pragma unroll
+    for (int i = 0; i < TOT / 4; ++i) {
+      if constexpr (DT == F32 || DT == I32) w[i] = __float_as_uint(v[i]);
+      else if constexpr (DT == F16) w[i] = f2h2(v[2 * i], v[2 * i + 1]);
+      else w[i] = f2b2(v[2 * i], v[2 * i + 1]);
+    }
+#pragma unroll
+    for (int c = 0; c < TOT / CB; ++c) straw<CB, POL>(p + c * CB, w + c * (CB / 4));
+  } else {
+#pragma unroll
+    for (int i = 0; i < N; ++i) st16(p + 2 * i, DT == F16 ? f2h(v[i]) : f2b(v[i]));
+  }
+}
+
+// raw element moves (pure copies/transposes keep every bit, NaN payloads too)
+template <int ESZ, int N, int CB, int POL>
+__device__ __forceinline__ void vload_raw(u32* e, const char* p) {  // one element per u32
+  constexpr int TOT = N * ESZ;
+  if constexpr (CB >= 4) {
+    u32 w[TOT / 4];
+#pragma unroll
+    for (int c = 0; c < TOT / CB; ++c) ldraw<CB, POL>(w + c * (CB / 4), p + c * CB);
+#pragma unroll
+    for (int i = 0; i < TOT / 4; ++i) {
+      if constexpr (ESZ == 4) {
+        e[i] = w[i];
+      } else {
+        e[2 * i] = w[i] & 0xffffu;
+        e[2 * i + 1] = w[i] >> 16;
+      }
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < N; ++i) e[i] = ld16<POL>(p + 2 * i);
+  }
+}
+
+template <int ESZ, int N, int CB, int POL>
+__device__ __forceinline__ void vstore_raw(char* p, const u32* e) {
+  constexpr int TOT = N * ESZ;
+  if constexpr (CB >= 4) {
+    u32 w[TOT / 4];
+#pragma unroll
+    for (int i = 0; i < TOT / 4; ++i) {
+      if constexpr (ESZ == 4) w[i] = e[i];
+      else w[i] = (e[2 * i] & 0xffffu) | (e[2 * i + 1] << 16);
+    }
+#pragma unroll
+    for (int c = 0; c < TOT / CB; ++c) straw<CB, POL>(p + c * CB, w + c * (CB / 4));
+  } else {
+#pragma unroll
+    for (int i = 0; i < N; ++i) st16(p + 2 * i, (u16)e[i]);
+  }
+}
+
+template <int DT, int POL>
+__device__ __forceinline__ float sload(const char* p) {
+  if constexpr (DT == F32 || DT == I32) {
+    u32 w;
+    ldraw<4, POL>(&w, p);
+    return __uint_as_float(w);
+  } else {
+    u16 h = ld16<POL>(p);
+    return DT == F16 ? h2f(h) : b2f(h);
+  }
+}
+
+template <int DT>
+__device__ __forceinline__ void sstore(char* p, float v) {
+  if constexpr (DT == F32 || DT == I32) {
+    u32 w = __float_as_uint(v);
+    straw<4, ST_DEFAULT>(p, &w);
+  } else {
+    st16(p, DT == F16 ? f2h(v) : f2b(v));
+  }
+}
+
+template <int ESZ, int POL>
+__device__ __forceinline__ u32 sload_raw(const char* p) {
+  if constexpr (ESZ == 4) {
+    u32 w;
+    ldraw<4, POL>(&w, p);
+    return w;
+  } else {
+    return ld16<POL>(p);
+  }
+}
+
+template <int ESZ>
+__device__ __forceinline__ void sstore_raw(char* p, u32 e) {
+  if constexpr (ESZ == 4) straw<4, ST_DEFAULT>(p, &e);
+  else st16(p, (u16)e);
+}
+
+// ------------------------------------------------------------------ operators
+// fp32 semantics shared with the oracle (include/fop.h); + - * / sqrt are the
+// _rn intrinsics, which the compiler never fuses into FMA.
+__device__ __forceinline__ float op_relu(float a) { return a > 0.f ? a : 0.f; }
+__device__ __forceinline__ float op_max(float a, float b) {
+  if (a != a) return b;
+  if (b != b) return a;
+  if (a == 0.f && b == 0.f) return (signbit(a) && signbit(b)) ? -0.f : 0.f;
+  return a > b ? a : b;
+}
+__device__ __forceinline__ float op_min(float a, float b) {
+  if (a != a) return b;
+  if (b != b) return a;
+  if (a == 0.f && b == 0.f) return (signbit(a) || signbit(b)) ? -0.f : 0.f;
+  return a < b ? a : b;
+}
+__device__ __forceinline__ float ex2_approx(float x) {
+  float r;
+  asm("ex2.approx.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float rcp_approx(float x) {
+  float r;
+  asm("rcp.approx.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+// GELU, tanh form: 0.5 v (1 + tanh u) == v * sigmoid(2u), u = sqrt(2/pi)(v + 0.044715 v^3).
+// MUFU.EX2 + MUFU.RCP: relative error ~1e-6, far inside one fp16/bf16 ulp
+// (the <= 1 ulp lemma); the precise tanhf form costs ~4x the
+// ALU work and would make cfg4a ALU-bound on B200.
+__device__ __forceinline__ float op_gelu_tanh(float v) {
+  const float k2log2e = 2.0f * 0.7978845608028654f * 1.4426950408889634f;
+  float v2 = v * v;
+  float inner = fmaf(0.044715f * v2, v, v);
+  float e = ex2_approx(-k2log2e * inner);
+  return v * rcp_approx(1.0f + e);
+}
+__device__ __forceinline__ float op_gelu_erf(float v) { return 0.5f * v * erfcf(-0.70710678118654752f * v); }
+__device__ __forceinline__ float op_sigmoid(float v) { return __frcp_rn(1.0f + expf(-v)); }
+
+// ------------------------------------------------------------------ reductions
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = op_max(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+}  // namespace fop
+
+struct FopArgs {
+  char* p[16];
+  char* ws;
+};

@@ -1,0 +1,152 @@
+// fop_internal.h — host-side data structures of libfop (planner, codegen, runtime).
+//
+// Pipeline:  a1 validate  -> a2 analyse strides  ->
+// a3 Algorithm 2 scenarios  -> a4 widths  -> a5 groups/classes/launches
+// (+ a7 fusion)  -> codegen  -> NVRTC (sm_100a)  -> fop_run launches.
+#pragma once
+
+#include <cstdint>
+#include <mutex>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "../../include/fop.h"
+
+namespace fop {
+
+// ---------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+struct Error {
+  fop_status status;
+  std::string msg;
+};
+[[noreturn]] void fail(fop_status s, const std::string& msg);
+
+inline int esize(int dtype) { return (dtype == FOP_F16 || dtype == FOP_BF16) ? 2 : 4; }
+
+// ---------------------------------------------------------------- a2
+// An access as an affine function of the loop iterators (element units):
+//   offset = base + sum_l coef[l] * i_l          (P:355 access functions)
+struct Affine {
+  int tensor = -1;
+  int64_t base = 0;
+  int64_t coef[FOP_MAX_LOOPS] = {0};
+  bool same(const Affine& o) const {
+    if (tensor != o.tensor || base != o.base) return false;
+    for (int l = 0; l < FOP_MAX_LOOPS; l++)
+      if (coef[l] != o.coef[l]) return false;
+    return true;
+  }
+};
+
+Affine affine_of(const fop_desc& d, const fop_access& a);
+
+// ---------------------------------------------------------------- a3
+struct Scenarios {
+  int nscen = 0;
+  int len[FOP_MAX_SCEN] = {0};
+  int loops[FOP_MAX_SCEN][3] = {{0}};          // outermost -> innermost
+  double inner_score[FOP_MAX_LOOPS] = {0};     // by statement loop position
+};
+Scenarios rank_scenarios(const fop_desc& d, int s, const fop_plan_opts& o);
+
+// ---------------------------------------------------------------- a5/a7
+enum XOp {  // expanded DAG node kinds (fop_opcode values + internal ones)
+  X_FWD = 100,     // value of an earlier ASSIGN statement of the same launch (registers)
+  X_SCALAR = 101   // value of an earlier REDUCE statement of the same launch (per row)
+};
+
+struct XNode {
+  int op = 0;       // fop_opcode or XOp
+  int a = -1, b = -1;
+  int cvt = 0;
+  float imm = 0.f;
+  int acc = -1;     // FOP_OP_LOAD: index into Launch::loads
+  int src = -1;     // X_FWD / X_SCALAR: index into Launch::stmts
+};
+
+struct XStmt {
+  int stmt = -1;            // descriptor statement index
+  int kind = FOP_ASSIGN;
+  int redop = FOP_RED_SUM;
+  std::vector<XNode> nodes; // expanded DAG (inlined producers substituted)
+  std::vector<XNode> fin;   // REDUCE finalize
+  int result = -1;          // index of the statement value in nodes
+  Affine write;
+  int out_dtype = FOP_F32;
+  bool store = true;        // result written to memory
+  bool fwd = false;         // consumed later in the same launch
+  bool move = false;        // pure element move (raw bits)
+};
+
+// a kernel loop: adjacent launch loops collapsed into one (loops
+// contiguous for ALL accesses are merged); coefficient = that of members[0]
+struct KLoop {
+  std::vector<int> members;   // loop ids, innermost first
+  int64_t extent = 1;
+};
+
+struct Launch {
+  int kclass = FOP_CLASS_EW;
+  int main_stmt = -1;
+  uint32_t mask = 0;
+  std::vector<XStmt> stmts;
+  std::vector<Affine> loads;      // distinct load accesses (after inlining)
+  std::vector<int> loops;         // loop ids the launch iterates (main statement loops)
+  int vec_loop = -1;              // d_v
+  int width = 1;                  // W (elements along d_v)
+  int read_loop = -1, read_width = 0;  // TRANSPOSE
+  int trans_load = -1;            // TRANSPOSE: index into loads of the transposed access
+  int coal_loop = -1;
+  std::vector<int> order;         // launch loop order, innermost first (before collapse)
+  std::vector<KLoop> kl;          // kernel loops (see geometry.cpp for the per-class layout)
+  int nsplit = 0;                 // ROW: #reduction kloops; COL: #parallel kloops; TR: 2
+  std::vector<int> load_cb;       // per load: vector chunk bytes (0 = not contiguous along d_v)
+  std::vector<int> load_cb_r;     // TRANSPOSE: per load chunk bytes along d_r
+  std::vector<int> store_cb;      // per stmt: vector chunk bytes of the store (0 = scalar)
+  int unroll = 1;
+  int gv = 1, gr = 1;             // lanes along d_v / along the other tiled dim
+  int64_t nchunks = 1;            // COL: row chunks
+  int64_t work = 0;               // total work items (threads' units)
+  // codegen / runtime
+  std::string name, src;
+  std::vector<char> cubin;
+  int64_t grid = 1;
+  int block = 256;
+  size_t smem = 0;
+  size_t ws_off = 0, ws_bytes = 0;  // COL_REDUCE partials + counters
+  std::vector<int> align;         // per tensor: byte alignment the vector variant assumes
+  bool scalar_variant = false;    // this launch is the narrow (W=1) variant
+};
+
+struct Plan {
+  fop_desc desc;
+  fop_plan_opts opts;
+  Scenarios scen[FOP_MAX_STMTS];
+  std::vector<Launch> launches;
+  std::vector<int64_t> temp_off;  // per tensor: workspace byte offset (-1 = not materialised)
+  size_t ws_bytes = 0;
+  // lazily built narrow variants (misaligned pointers), guarded by mu
+  std::mutex mu;
+  std::vector<Launch> narrow;     // same indexing as launches (empty src = not built)
+  struct Loaded { void* ctx; std::vector<void*> mods, fns, nmods, nfns; };
+  std::vector<Loaded> loaded;
+};
+
+// validate.cpp
+void validate(const fop_desc& d);
+// planner.cpp
+void plan_launches(Plan& p);
+void finalize_launch_geometry(const Plan& p, Launch& L);
+// codegen.cpp
+std::string generate(const Plan& p, Launch& L, int launch_index);
+extern const char* kDeviceHeader;   // device/fop_device.cuh, embedded at build time
+// jit.cpp
+void jit_compile(Launch& L);
+bool jit_available();
+// runtime.cpp
+fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream,
+                    void* const* host_ptrs);
+
+}  // namespace fop

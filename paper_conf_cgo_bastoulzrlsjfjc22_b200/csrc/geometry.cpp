@@ -1,0 +1,303 @@
+// geometry.cpp — rows a4 (vector width, divisibility, alignment) and a5
+// (mapping and launch geometry) for one launch.
+//
+// a4: the paper's vector dimension must be innermost, of size 2 or 4, with
+// accesses "aligned and either constant or contiguous", carried by
+// 64/128-bit transactions.  On B200 the width is byte based: the
+// narrowest element type among the accesses contiguous along d_v gets a full
+// max_vec_bytes vector (16 B = LDG/STG.128, or 32 B = LDG/STG.256 on
+// sm_100a); wider types move several chunks.  Divisibility: the vector
+// loop's extent must be a multiple of W (halve W otherwise — down to 1, the
+// paper's "novec").  Alignment: each access gets the largest chunk
+// its base and the other loops' strides keep aligned ("we may mix vector
+// types with scalar types"); base pointers are checked at fop_run.
+//
+// a5: "dimensions marked as vectorized" are not mapped to blocks/threads
+// — each thread owns W consecutive iterations of d_v; consecutive
+// threads take consecutive vectors, then the next loops of the thread order
+// (coalescing, goal (ii) of P:297).  Loops that are contiguous for every
+// access are collapsed (a B200 step beyond the paper).
+#include <algorithm>
+#include <string>
+
+#include "fop_internal.h"
+
+namespace fop {
+
+namespace {
+
+std::vector<const Affine*> all_accesses(const Launch& L) {
+  std::vector<const Affine*> v;
+  for (const auto& a : L.loads) v.push_back(&a);
+  for (const auto& x : L.stmts) v.push_back(&x.write);
+  return v;
+}
+
+// order a set of loops innermost first
+std::vector<int> order_rest(const Plan& p, const Launch& L, std::vector<int> rest) {
+  const fop_stmt& st = p.desc.s[L.main_stmt];
+  auto pos = [&](int l) {
+    for (int k = 0; k < st.nloops; k++)
+      if (st.loop[k] == l) return k;
+    return -1;
+  };
+  const Affine& w = L.stmts[0].write;
+  if (p.opts.coalesce_order == FOP_ORDER_MEMORY) {
+    // memory order of the write; loops the write does not use (the reduction
+    // loops of COL) are ordered by the first load instead
+    auto key = [&](int l) {
+      if (w.coef[l] != 0 || L.loads.empty()) return w.coef[l];
+      return L.loads[0].coef[l];
+    };
+    std::stable_sort(rest.begin(), rest.end(), [&](int a, int b) {
+      int64_t ca = key(a), cb = key(b);
+      if (ca != cb) return ca < cb;
+      return pos(a) > pos(b);
+    });
+    return rest;
+  }
+  // FOP_ORDER_PAPER: the best scenario (outer -> inner) gives the innermost
+  // loops after d_v; loops outside the scenario follow, innermost first
+  std::vector<int> out;
+  const Scenarios& sc = p.scen[L.main_stmt];
+  for (int q = sc.len[0] - 1; q >= 0; q--) {
+    int l = sc.loops[0][q];
+    if (std::find(rest.begin(), rest.end(), l) != rest.end()) out.push_back(l);
+  }
+  for (int k = st.nloops - 1; k >= 0; k--) {
+    int l = st.loop[k];
+    if (std::find(rest.begin(), rest.end(), l) != rest.end() &&
+        std::find(out.begin(), out.end(), l) == out.end())
+      out.push_back(l);
+  }
+  return out;
+}
+
+// collapse adjacent loops of a segment: merge l into K iff for every access
+// coef(l) == coef(K.members[0]) * K.extent
+void collapse_into(const Plan& p, const std::vector<const Affine*>& acc, const std::vector<int>& seg,
+                   std::vector<KLoop>& out) {
+  for (size_t i = 0; i < seg.size(); i++) {
+    int l = seg[i];
+    if (i > 0) {
+      KLoop& K = out.back();
+      bool ok = true;
+      for (const Affine* a : acc)
+        if (a->coef[l] != a->coef[K.members[0]] * K.extent) ok = false;
+      if (ok) {
+        K.members.push_back(l);
+        K.extent *= p.desc.extent[l];
+        continue;
+      }
+    }
+    KLoop K;
+    K.members.push_back(l);
+    K.extent = p.desc.extent[l];
+    out.push_back(K);
+  }
+}
+
+int pow2_floor(int64_t x) {
+  int r = 1;
+  while ((int64_t)r * 2 <= x) r *= 2;
+  return r;
+}
+
+// largest power-of-two chunk (bytes) <= cap keeping `a` aligned, given the
+// kernel loops other than `vk` (whose steps are multiples of the vector)
+int chunk_bytes(const Plan& p, const Launch& L, const Affine& a, int vk, int cap) {
+  int es = esize(p.desc.t[a.tensor].dtype);
+  int cb = cap;
+  auto fits = [&](int64_t elems) { return ((elems * es) % cb) == 0; };
+  while (cb > es) {
+    bool ok = fits(a.base);
+    for (int k = 0; k < (int)L.kl.size() && ok; k++)
+      if (k != vk) ok = fits(a.coef[L.kl[k].members[0]]);
+    if (ok) break;
+    cb /= 2;
+  }
+  return std::max(cb, es);
+}
+
+int64_t coef(const Launch& L, const Affine& a, int k) { return a.coef[L.kl[k].members[0]]; }
+
+}  // namespace
+
+void finalize_launch_geometry(const Plan& p, Launch& L) {
+  const fop_desc& d = p.desc;
+  const fop_plan_opts& o = p.opts;
+  auto acc = all_accesses(L);
+  int sms = o.sm_count > 0 ? o.sm_count : 148;
+  int vmax = o.max_vec_bytes >= 32 ? 32 : 16;
+
+  // ---- loop order + collapse
+  L.kl.clear();
+  std::vector<int> rest;
+  for (int l : L.loops)
+    if (l != L.vec_loop && l != L.read_loop) rest.push_back(l);
+  if (L.kclass == FOP_CLASS_EW || L.kclass == FOP_CLASS_TRANSPOSE) {
+    std::vector<int> ord = {L.vec_loop};
+    if (L.kclass == FOP_CLASS_TRANSPOSE) ord.push_back(L.read_loop);
+    for (int l : order_rest(p, L, rest)) ord.push_back(l);
+    L.order = ord;
+    std::vector<int> seg0 = {ord[0]};
+    collapse_into(p, acc, seg0, L.kl);
+    std::vector<int> seg1(ord.begin() + 1, ord.end());
+    // V never absorbs loops in TRANSPOSE (d_r follows it); in EW it may
+    if (L.kclass == FOP_CLASS_EW) {
+      L.kl.clear();
+      collapse_into(p, acc, ord, L.kl);
+    } else {
+      collapse_into(p, acc, seg1, L.kl);
+    }
+    L.nsplit = L.kclass == FOP_CLASS_TRANSPOSE ? 2 : 1;
+  } else {
+    // ROW: [d_v, other reduction loops | parallel loops]
+    // COL: [d_v, other parallel loops  | reduction loops]
+    const Affine* wp = &L.stmts.back().write;  // a REDUCE target
+    for (const auto& x : L.stmts)
+      if (x.kind == FOP_REDUCE) wp = &x.write;
+    const Affine& w = *wp;
+    std::vector<int> red, par;
+    for (int l : rest) (w.coef[l] == 0 ? red : par).push_back(l);
+    std::vector<int> seg1 = {L.vec_loop}, seg2;
+    std::vector<int> first = L.kclass == FOP_CLASS_ROW_REDUCE ? red : par;
+    std::vector<int> second = L.kclass == FOP_CLASS_ROW_REDUCE ? par : red;
+    for (int l : order_rest(p, L, first)) seg1.push_back(l);
+    for (int l : order_rest(p, L, second)) seg2.push_back(l);
+    L.order = seg1;
+    L.order.insert(L.order.end(), seg2.begin(), seg2.end());
+    collapse_into(p, acc, seg1, L.kl);
+    L.nsplit = (int)L.kl.size();
+    collapse_into(p, acc, seg2, L.kl);
+  }
+
+  // ---- a4: width
+  int min_es = 16;
+  bool any_vec = false;
+  for (const Affine* a : acc)
+    if (coef(L, *a, 0) == 1) {
+      min_es = std::min(min_es, esize(d.t[a->tensor].dtype));
+      any_vec = true;
+    }
+  int W = any_vec ? std::max(1, o.max_vec_bytes / min_es) : 1;
+  if (o.force_width > 0) W = std::min(W, pow2_floor(o.force_width));
+  if (L.scalar_variant) W = 1;
+  int64_t EV = L.kl[0].extent;
+  bool tail_ok = L.kclass == FOP_CLASS_EW && L.kl.size() == 1;
+  if (tail_ok) {
+    if (EV < W) W = pow2_floor(EV);
+  } else {
+    while (W > 1 && EV % W) W /= 2;
+  }
+  L.width = W;
+
+  if (L.kclass == FOP_CLASS_TRANSPOSE) {
+    const Affine& t = L.loads[L.trans_load];
+    int wr = std::max(1, o.max_vec_bytes / esize(d.t[t.tensor].dtype));
+    if (o.force_width > 0) wr = std::min(wr, pow2_floor(o.force_width));
+    if (L.scalar_variant) wr = 1;
+    while (wr > 1 && L.kl[1].extent % wr) wr /= 2;
+    L.read_width = wr;
+    if (W == 1 || wr == 1) {  // degenerate tile: plain elementwise with gathers
+      L.kclass = FOP_CLASS_EW;
+      L.read_loop = -1;
+      L.trans_load = -1;
+      L.read_width = 0;
+      finalize_launch_geometry(p, L);
+      return;
+    }
+  }
+
+  // ---- a4: per-access chunks
+  auto vec_cb = [&](const Affine& a, int vk, int w) {
+    int es = esize(d.t[a.tensor].dtype);
+    return chunk_bytes(p, L, a, vk, std::min(vmax, w * es));
+  };
+  L.load_cb.assign(L.loads.size(), 0);
+  L.load_cb_r.assign(L.loads.size(), 0);
+  for (size_t k = 0; k < L.loads.size(); k++) {
+    if (coef(L, L.loads[k], 0) == 1) L.load_cb[k] = vec_cb(L.loads[k], 0, W);
+    if (L.kclass == FOP_CLASS_TRANSPOSE && coef(L, L.loads[k], 0) != 1 && coef(L, L.loads[k], 1) == 1)
+      L.load_cb_r[k] = vec_cb(L.loads[k], 1, L.read_width);
+  }
+  L.store_cb.assign(L.stmts.size(), 0);
+  for (size_t k = 0; k < L.stmts.size(); k++)
+    if (coef(L, L.stmts[k].write, 0) == 1) L.store_cb[k] = vec_cb(L.stmts[k].write, 0, W);
+  L.align.assign(d.ntensors, 1);
+  for (size_t k = 0; k < L.loads.size(); k++) {
+    int t = L.loads[k].tensor;
+    L.align[t] = std::max({L.align[t], L.load_cb[k], L.load_cb_r[k], esize(d.t[t].dtype)});
+  }
+  for (size_t k = 0; k < L.stmts.size(); k++) {
+    int t = L.stmts[k].write.tensor;
+    L.align[t] = std::max({L.align[t], L.store_cb[k], esize(d.t[t].dtype)});
+  }
+
+  // ---- a5: launch geometry
+  int64_t prod_rest = 1;
+  L.block = 256;
+  L.ws_bytes = 0;
+  if (L.kclass == FOP_CLASS_EW) {
+    for (size_t k = 1; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
+    int64_t nv = (EV + W - 1) / W;
+    L.work = nv * prod_rest;
+    int bytes = 0;
+    for (size_t k = 0; k < L.loads.size(); k++)
+      if (L.load_cb[k]) bytes += W * esize(d.t[L.loads[k].tensor].dtype);
+    for (size_t k = 0; k < L.stmts.size(); k++)
+      if (L.store_cb[k]) bytes += W * esize(L.stmts[k].out_dtype);
+    L.unroll = bytes <= 32 ? 4 : (bytes <= 64 ? 2 : 1);
+    int64_t need = (L.work + (int64_t)L.block * L.unroll - 1) / ((int64_t)L.block * L.unroll);
+    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * (2048 / L.block)));
+  } else if (L.kclass == FOP_CLASS_TRANSPOSE) {
+    for (size_t k = 2; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
+    int64_t ntv = EV / W, ntr = L.kl[1].extent / L.read_width;
+    int es_out = esize(L.stmts[0].out_dtype);
+    int gv = (int)std::min<int64_t>(32, std::max<int64_t>(1, 128 / (W * es_out)));
+    gv = std::min(gv, pow2_floor(ntv));
+    L.gv = gv;
+    L.gr = 32 / gv;
+    int64_t tvh = (ntv + gv - 1) / gv, trh = (ntr + L.gr - 1) / L.gr;
+    L.work = (int64_t)gv * L.gr * tvh * trh * prod_rest;
+    L.unroll = 1;
+    int64_t need = (L.work + L.block - 1) / L.block;
+    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * (2048 / L.block)));
+  } else if (L.kclass == FOP_CLASS_ROW_REDUCE) {
+    int64_t rows = 1;
+    for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
+    L.work = rows;  // one warp per row
+    int64_t need = (rows + L.block / 32 - 1) / (L.block / 32);
+    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * (2048 / L.block)));
+    L.unroll = 1;
+  } else {  // COL_REDUCE
+    int64_t nvd = EV / W;
+    const Affine* big = nullptr;
+    for (const auto& a : L.loads)
+      if (coef(L, a, 0) == 1) big = &a;
+    int es_ld = big ? esize(d.t[big->tensor].dtype) : 4;
+    int gv = (int)std::min<int64_t>(32, std::max<int64_t>(1, 128 / (W * es_ld)));
+    gv = std::min(gv, pow2_floor(nvd));
+    L.gv = gv;
+    L.gr = L.block / gv;
+    int64_t slabs = (nvd + gv - 1) / gv;
+    for (int k = 1; k < L.nsplit; k++) slabs *= L.kl[k].extent;
+    int64_t rows = 1;
+    for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
+    int64_t target = (int64_t)sms * 4;
+    int64_t nch = std::max<int64_t>(1, (target + slabs / 2) / std::max<int64_t>(1, slabs));
+    nch = std::min<int64_t>(nch, std::max<int64_t>(1, (rows + L.gr - 1) / L.gr));
+    L.nchunks = nch;
+    L.work = rows;
+    L.grid = slabs * nch;
+    L.unroll = 4;
+    if (nch > 1) {
+      size_t part = (size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(float);
+      part = (part + 255) & ~size_t(255);
+      L.ws_bytes = part + (size_t)slabs * sizeof(unsigned);
+    }
+    L.smem = (size_t)L.block * W * sizeof(float) + 16;
+  }
+}
+
+}  // namespace fop

@@ -1,0 +1,207 @@
+// runtime.cpp — loads the compiled kernels into the caller's CUDA context and
+// launches them on the caller's stream (the hot path of fop_run).
+//
+// The CUDA driver API is reached through dlopen("libcuda.so.1") so the library
+// loads on hosts without a driver (planning/compiling works there; running
+// returns FOP_E_CUDA).  The caller (PyTorch) owns every device buffer and the
+// stream; fop_run only enqueues: one kernel per launch of the plan.
+#include <dlfcn.h>
+
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "fop_internal.h"
+
+namespace fop {
+
+namespace {
+typedef int CUresult;
+typedef void* CUcontext;
+typedef void* CUmodule;
+typedef void* CUfunction;
+typedef void* CUstream;
+typedef int CUdevice;
+typedef unsigned long long CUdeviceptr;
+enum { CU_POINTER_ATTRIBUTE_CONTEXT = 1, CU_POINTER_ATTRIBUTE_DEVICE_ORDINAL = 9 };
+
+struct Cuda {
+  bool ok = false;
+  std::string why;
+  CUresult (*init)(unsigned);
+  CUresult (*ctx_get)(CUcontext*);
+  CUresult (*ctx_set)(CUcontext);
+  CUresult (*primary_retain)(CUcontext*, CUdevice);
+  CUresult (*ptr_attr)(void*, int, CUdeviceptr);
+  CUresult (*mod_load)(CUmodule*, const void*);
+  CUresult (*mod_func)(CUfunction*, CUmodule, const char*);
+  CUresult (*launch)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, CUstream,
+                     void**, void**);
+  CUresult (*h2d)(CUdeviceptr, const void*, size_t, CUstream);
+  CUresult (*d2h)(void*, CUdeviceptr, size_t, CUstream);
+  CUresult (*errstr)(CUresult, const char**);
+};
+
+Cuda& cuda() {
+  static Cuda c;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) {
+      c.why = "cannot dlopen libcuda.so.1 (no NVIDIA driver on this host)";
+      return;
+    }
+#define SYM(field, name)                               \
+  *(void**)(&c.field) = dlsym(h, name);                \
+  if (!c.field) {                                      \
+    c.why = std::string("libcuda lacks ") + name;      \
+    return;                                            \
+  }
+    SYM(init, "cuInit");
+    SYM(ctx_get, "cuCtxGetCurrent");
+    SYM(ctx_set, "cuCtxSetCurrent");
+    SYM(primary_retain, "cuDevicePrimaryCtxRetain");
+    SYM(ptr_attr, "cuPointerGetAttribute");
+    SYM(mod_load, "cuModuleLoadData");
+    SYM(mod_func, "cuModuleGetFunction");
+    SYM(launch, "cuLaunchKernel");
+    SYM(h2d, "cuMemcpyHtoDAsync_v2");
+    SYM(d2h, "cuMemcpyDtoHAsync_v2");
+    SYM(errstr, "cuGetErrorString");
+#undef SYM
+    if (c.init(0) != 0) {
+      c.why = "cuInit failed";
+      return;
+    }
+    c.ok = true;
+  });
+  return c;
+}
+
+void check(CUresult r, const char* what) {
+  if (r == 0) return;
+  const char* s = nullptr;
+  cuda().errstr(r, &s);
+  fail(FOP_E_CUDA, std::string(what) + ": " + (s ? s : "unknown CUDA error") + " (" + std::to_string(r) + ")");
+}
+
+CUcontext current_context(void* const* ptrs, int n) {
+  Cuda& c = cuda();
+  CUcontext ctx = nullptr;
+  check(c.ctx_get(&ctx), "cuCtxGetCurrent");
+  if (ctx) return ctx;
+  for (int i = 0; i < n; i++) {
+    if (!ptrs[i]) continue;
+    int dev = -1;
+    if (c.ptr_attr(&dev, CU_POINTER_ATTRIBUTE_DEVICE_ORDINAL, (CUdeviceptr)ptrs[i]) == 0 && dev >= 0) {
+      check(c.primary_retain(&ctx, dev), "cuDevicePrimaryCtxRetain");
+      check(c.ctx_set(ctx), "cuCtxSetCurrent");
+      return ctx;
+    }
+  }
+  fail(FOP_E_CUDA, "no current CUDA context and no device pointer to infer one from");
+}
+
+int64_t span_bytes(const fop_tensor& t) {
+  int64_t n = 1;
+  for (int r = 0; r < t.rank; r++) n += (t.shape[r] - 1) * t.stride[r];
+  return n * esize(t.dtype);
+}
+
+Plan::Loaded& loaded_for(Plan& p, CUcontext ctx) {
+  for (auto& l : p.loaded)
+    if (l.ctx == ctx) return l;
+  Plan::Loaded l;
+  l.ctx = ctx;
+  for (auto& L : p.launches) {
+    CUmodule m = nullptr;
+    CUfunction f = nullptr;
+    check(cuda().mod_load(&m, L.cubin.data()), "cuModuleLoadData");
+    check(cuda().mod_func(&f, m, L.name.c_str()), "cuModuleGetFunction");
+    l.mods.push_back(m);
+    l.fns.push_back(f);
+    l.nmods.push_back(nullptr);
+    l.nfns.push_back(nullptr);
+  }
+  p.loaded.push_back(l);
+  return p.loaded.back();
+}
+
+CUfunction narrow_fn(Plan& p, Plan::Loaded& l, size_t i) {
+  if (l.nfns[i]) return l.nfns[i];
+  Launch& N = p.narrow[i];
+  if (N.cubin.empty()) {
+    generate(p, N, (int)i);
+    jit_compile(N);
+  }
+  CUmodule m = nullptr;
+  CUfunction f = nullptr;
+  check(cuda().mod_load(&m, N.cubin.data()), "cuModuleLoadData(narrow)");
+  check(cuda().mod_func(&f, m, N.name.c_str()), "cuModuleGetFunction(narrow)");
+  l.nmods[i] = m;
+  l.nfns[i] = f;
+  return f;
+}
+}  // namespace
+
+fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream, void* const* host_ptrs) {
+  const fop_desc& d = p.desc;
+  if (nptrs != d.ntensors) fail(FOP_E_INVALID, "nptrs must equal desc.ntensors");
+  for (auto& L : p.launches)
+    if (L.cubin.empty()) fail(FOP_E_INVALID, "plan was built with opts.jit = 0: nothing to run");
+  Cuda& c = cuda();
+  if (!c.ok) fail(FOP_E_CUDA, c.why);
+  if (p.ws_bytes && !ws) fail(FOP_E_INVALID, "this plan needs a workspace of fop_plan_workspace_bytes() bytes");
+  for (int t = 0; t < d.ntensors; t++) {
+    if (!ptrs[t] && d.t[t].role != FOP_TEMP) fail(FOP_E_INVALID, "NULL pointer for tensor " + std::to_string(t));
+    if (ptrs[t] && ((uintptr_t)ptrs[t] % esize(d.t[t].dtype)))
+      fail(FOP_E_ALIGN, "tensor " + std::to_string(t) + " is not aligned to its element size");
+  }
+  CUcontext ctx = current_context(ptrs, nptrs);
+  CUstream st = (CUstream)stream;
+
+  if (host_ptrs) {  // end-to-end: inputs host -> device
+    for (int t = 0; t < d.ntensors; t++)
+      if ((d.t[t].role == FOP_IN || d.t[t].role == FOP_INOUT) && host_ptrs[t])
+        check(c.h2d((CUdeviceptr)ptrs[t], host_ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyHtoDAsync");
+  }
+
+  struct Args {  // mirrors FopArgs of fop_device.cuh
+
+    char* p[16];
+    char* ws;
+  } args;
+  std::memset(&args, 0, sizeof args);
+  for (int t = 0; t < d.ntensors; t++) {
+    args.p[t] = (char*)ptrs[t];
+    if (d.t[t].role == FOP_TEMP && p.temp_off[t] >= 0) args.p[t] = (char*)ws + p.temp_off[t];
+  }
+  args.ws = (char*)ws;
+
+  std::lock_guard<std::mutex> g(p.mu);
+  Plan::Loaded& l = loaded_for(p, ctx);
+  for (size_t i = 0; i < p.launches.size(); i++) {
+    const Launch& L = p.launches[i];
+    bool aligned = true;
+    for (int t = 0; t < d.ntensors; t++)
+      if (args.p[t] && ((uintptr_t)args.p[t] % (uintptr_t)L.align[t])) aligned = false;
+    CUfunction f = l.fns[i];
+    const Launch* G = &L;
+    if (!aligned) {
+      f = narrow_fn(p, l, i);
+      G = &p.narrow[i];
+    }
+    void* params[] = {&args};
+    check(c.launch(f, (unsigned)G->grid, 1, 1, (unsigned)G->block, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
+  }
+
+  if (host_ptrs) {  // device -> host results
+    for (int t = 0; t < d.ntensors; t++)
+      if ((d.t[t].role == FOP_OUT || d.t[t].role == FOP_INOUT) && host_ptrs[t])
+        check(c.d2h(host_ptrs[t], (CUdeviceptr)ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyDtoHAsync");
+  }
+  return FOP_OK;
+}
+
+}  // namespace fop

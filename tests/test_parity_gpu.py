@@ -1,0 +1,298 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the oracle, element by
+element, on the same seeded inputs (BASELINE.json north_star tolerances):
+  * bit-exact: transposes, copies, integer moves, fp32 elementwise (same op
+    order, no contraction) and every output that is a deterministic function
+    of IEEE-correct ops (cfg2's BN: / sqrt * + relu, RNE cast);
+  * <= 1 fp16/bf16 ulp where a transcendental (GELU) precedes the cast;
+  * reductions: normwise |gpu - ref| <= tol * fin(sum |term|) (reading R16).
+Sizes span several tiles plus ragged tails; full-size runs sample batch
+slices (the operators are independent along the batch loop).
+"""
+import copy
+
+import numpy as np
+import pytest
+import torch
+
+import workloads as W
+from oracle import oracle as O
+
+from harness import (abs_terms_desc, assert_bitexact, assert_normwise, assert_ulp, run_gpu,
+                     device_tensors, to_host)
+
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+
+def _outs(desc):
+    return [n for n, t in desc["tensors"].items() if t["role"] in ("out", "inout")]
+
+
+# ---------------------------------------------------------------- EW
+@pytest.mark.parametrize("shape", [(4, 8, 16), (3, 5, 7), (2, 3, 1000003 // 6), (1, 1, 1), (64, 33, 40)])
+def test_cfg1_ew_bitexact(shape):
+    d = W.cfg1(*shape)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    ref = O.run(d, x)
+    assert_bitexact(got["out"], ref["out"], "out")
+
+
+def test_cfg1_bias_b_and_novec_and_orders():
+    d = W.cfg1_bias_b(4, 8, 16)
+    x = W.make_inputs(d)
+    ref = O.run(d, x)
+    for opts in [{}, {"force_width": 1}, {"coalesce_order": "memory"}, {"max_vec_bytes": 32}]:
+        got, op = run_gpu(d, x, **opts)
+        assert_bitexact(got["out"], ref["out"], f"out {opts}")
+
+
+def test_cfg1_misaligned_pointers_use_narrow_variant():
+    d = W.cfg1(4, 8, 16)
+    x = W.make_inputs(d)
+    ref = O.run(d, x)
+    got, op = run_gpu(d, x, offset=1)      # base pointers 4 B off a 16 B boundary
+    assert_bitexact(got["out"], ref["out"], "out")
+
+
+@pytest.mark.parametrize("dims", [(2, 64, 112, 112), (1, 3, 7, 13), (3, 5, 4, 24)])
+def test_cfg2_bn_relu_cast_bitexact(dims):
+    d = W.cfg2(*dims)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    ref = O.run(d, x)
+    assert_bitexact(got["y"], ref["y"], "y")
+
+
+def test_cfg2_orders_widths_agree():
+    d = W.cfg2(2, 64, 28, 28)
+    x = W.make_inputs(d)
+    ref = O.run(d, x)
+    for opts in [{"coalesce_order": "memory"}, {"force_width": 2}, {"max_vec_bytes": 32}]:
+        got, op = run_gpu(d, x, **opts)
+        assert_bitexact(got["y"], ref["y"], f"y {opts}")
+
+
+def test_bf16_and_casts():
+    d = W.cfg1(4, 8, 64)
+    d["tensors"]["out"]["dtype"] = "bf16"
+    d["stmts"][0]["expr"] = d["stmts"][0]["expr"] + [("cast", 5, "f16"), ("sigmoid", 6),
+                                                     ("add", 7, 5)]
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    ref = O.run(d, x)
+    from harness import ordered16
+    diff = np.abs(ordered16(got["out"]) - ordered16(ref["out"]))   # bf16 has fp16's sign/magnitude order
+    assert diff.max() <= 1, diff.max()
+
+
+# ---------------------------------------------------------------- TRANSPOSE
+@pytest.mark.parametrize("dims", [(2, 256, 56, 56), (1, 24, 5, 7), (2, 40, 3, 16), (1, 8, 1, 8)])
+def test_cfg3_transpose_bitexact(dims):
+    d = W.cfg3(*dims)
+    d["tensors"]["x"]["init"] = ("special", 9)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    ref = O.run(d, x)
+    assert_bitexact(got["out"], ref["out"], "out")
+
+
+def test_cfg3_classifies_as_transpose_with_both_sides_vectorised():
+    d = W.cfg3(2, 256, 56, 56)
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    info = FusedOp(d).info()["launches"][0]
+    assert info["class"] == "transpose" and info["vec_loop"] == "c" and info["read_loop"] == "w"
+    assert info["width"] == 8 and info["read_width"] == 8
+
+
+def test_pure_move_transposes_keep_nan_payloads():
+    d = W.cfg3(2, 64, 8, 8)
+    d["stmts"][0]["expr"] = [("load", 0)]
+    d["tensors"]["x"]["init"] = ("special", 3)
+    x = W.make_inputs(d)
+    x["x"].view(np.uint16)[::97] = 0x7D01           # signalling-style NaN payload
+    got, _ = run_gpu(d, x)
+    ref = O.run(d, x)
+    assert np.array_equal(got["out"].view(np.uint16), ref["out"].view(np.uint16))
+
+
+@pytest.mark.parametrize("dtype", ["f32", "i32", "bf16"])
+def test_transpose2d_dtypes(dtype):
+    d = W.transpose2d(64, 96, dtype)
+    if dtype == "i32":
+        d["tensors"]["inp"]["init"] = ("randint", -1000000, 1000000, 5)
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    ref = O.run(d, x)
+    assert np.array_equal(got["out"].view(np.uint8), ref["out"].view(np.uint8))
+
+
+def test_transpose_roundtrip_on_gpu():
+    N, C, H, Wd = 2, 32, 6, 10
+    d = W.cfg3(N, C, H, Wd, s=1.0)
+    d["tensors"]["x"]["init"] = ("special", 4)
+    x = W.make_inputs(d)
+    t, _ = run_gpu(d, x)
+    d2 = W.cfg3(N, C, H, Wd, s=1.0)
+    d2["tensors"]["x"]["shape"] = [N, H, Wd, C]
+    d2["tensors"]["out"]["shape"] = [N, C, H, Wd]
+    d2["stmts"][0]["write"] = ("out", ["n", "c", "h", "w"])
+    d2["stmts"][0]["reads"] = [("x", ["n", "h", "w", "c"])]
+    back, _ = run_gpu(d2, {"x": t["out"]})
+    assert_bitexact(back["out"], x["x"], "roundtrip")
+
+
+# ---------------------------------------------------------------- ROW_REDUCE
+def _check_rowstats(d, x, got):
+    ref = O.run(d, x)
+    assert_ulp(got["y"], ref["y"], 1, "y")
+    # statistics of the GPU's own y, recomputed by the oracle: isolates the
+    # reduction from the GELU's last-bit rounding
+    d2 = copy.deepcopy(d)
+    d2["tensors"]["y"]["role"] = "in"
+    xin = dict(x)
+    xin["y"] = got["y"]
+    ref2 = O.run(d2, xin, stmts=[1, 2])
+    for si, name in [(1, "mean"), (2, "var")]:
+        scale = O.run(abs_terms_desc(d2, si), xin, stmts=[1, 2])[name]
+        assert_normwise(got[name], ref2[name], scale, 1e-5, name)
+        assert_normwise(got[name], ref[name], O.run(abs_terms_desc(d, si), x)[name], 2e-3, name)
+
+
+@pytest.mark.parametrize("dims", [(2, 64, 768), (1, 7, 200), (3, 5, 100), (1, 3, 24), (1, 2, 4096)])
+def test_cfg4a_bias_gelu_rowstats(dims):
+    d = W.cfg4a(*dims)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.info()["launches"][0]["class"] == "row_reduce"
+    _check_rowstats(d, x, got)
+
+
+def test_row_closed_forms_on_gpu():
+    d = W.cfg4a(1, 4, 768)
+    d["stmts"][0]["expr"] = [("load", 0)]
+    d["stmts"][0]["reads"] = [("x", ["b", "s", "h"])]
+    x = {"x": np.tile(np.arange(768, dtype=np.float16), 4), "bias": np.zeros(768, np.float16)}
+    got, _ = run_gpu(d, x)
+    assert np.all(got["mean"] == np.float32(383.5))
+    assert np.allclose(got["var"], (768 ** 2 - 1) / 12, rtol=1e-6)
+
+
+# ---------------------------------------------------------------- COL_REDUCE
+@pytest.mark.parametrize("dims", [(4096, 1024), (1000, 40), (65536, 8), (33, 1024), (5, 3)])
+def test_cfg4b_colsum(dims):
+    d = W.cfg4b(*dims)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    ref = O.run(d, x)
+    scale = O.run(abs_terms_desc(d, 0), x)["out"]
+    assert_normwise(got["out"], ref["out"], scale, 1e-5, "out")
+
+
+def test_colsum_ones_exact_and_deterministic():
+    d = W.cfg4b(65536, 1024, init=("ones",))
+    x = W.make_inputs(d)
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    op = FusedOp(d)
+    dev = device_tensors(d, x)
+    op.run(dev)
+    first = dev["out"].clone()
+    assert torch.all(first == 65536.0)
+    d2 = W.cfg4b(65536, 1024)
+    x2 = W.make_inputs(d2)
+    op2 = FusedOp(d2)
+    dev2 = device_tensors(d2, x2)
+    runs = []
+    for _ in range(3):
+        op2.run(dev2)
+        runs.append(dev2["out"].clone())
+    torch.cuda.synchronize()
+    assert all(torch.equal(runs[0], r) for r in runs[1:])   # fixed-order trees
+
+
+def test_reduce_max_col_and_row():
+    d = W.cfg4b(3000, 72)
+    d["stmts"][0]["op"] = "max"
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    assert_bitexact(got["out"], O.run(d, x)["out"], "colmax")
+    d = W.cfg4a(2, 8, 256)
+    d["stmts"][1]["op"] = "max"
+    d["stmts"][1]["finalize"] = []
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    ref = O.run(d, x)
+    assert_ulp(got["y"], ref["y"], 1, "y")
+
+
+# ---------------------------------------------------------------- full sizes (launch config of bench.py)
+def _slice_batch(desc, x, got, loop, idx):
+    """Oracle on batch index `idx` of `loop` vs the GPU's full-size output."""
+    d1 = copy.deepcopy(desc)
+    d1["loops"][loop] = 1
+    xs, gs = {}, {}
+    for n, t in desc["tensors"].items():
+        st = W.tensor_strides(t)
+        # the batch loop indexes dim 0 of every batched tensor in these configs
+        if t["shape"][0] == desc["loops"][loop] and len(t["shape"]) > 1:
+            d1["tensors"][n]["shape"] = [1] + t["shape"][1:]
+            sl = slice(idx * st[0], (idx + 1) * st[0])
+        else:
+            sl = slice(None)
+        if t["role"] in ("in", "inout"):
+            xs[n] = x[n][sl]
+        if t["role"] in ("out", "inout"):
+            gs[n] = got[n][sl]
+    return d1, xs, gs
+
+
+@pytest.mark.parametrize("cfg,loop,out", [("cfg2", "n", "y"), ("cfg3", "n", "out")])
+def test_full_size_sampled_bitexact(cfg, loop, out):
+    d = W.CONFIGS[cfg]()
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    for idx in (0, d["loops"][loop] // 2 + 3, d["loops"][loop] - 1):
+        d1, xs, gs = _slice_batch(d, x, got, loop, idx)
+        assert_bitexact(gs[out], O.run(d1, xs)[out], f"{cfg} {loop}={idx}")
+
+
+def test_full_size_cfg4a_sampled():
+    d = W.cfg4a()
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    for idx in (0, 40, 63):
+        d1, xs, gs = _slice_batch(d, x, got, "b", idx)
+        gs["mean"] = got["mean"][idx * 512:(idx + 1) * 512]
+        gs["var"] = got["var"][idx * 512:(idx + 1) * 512]
+        d1["tensors"]["mean"]["shape"] = [1, 512]
+        d1["tensors"]["var"]["shape"] = [1, 512]
+        _check_rowstats(d1, xs, gs)
+
+
+def test_full_size_cfg4b():
+    d = W.cfg4b()
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    ref = O.run(d, x)
+    scale = O.run(abs_terms_desc(d, 0), x)["out"]
+    assert_normwise(got["out"], ref["out"], scale, 1e-5, "out")
+
+
+# ---------------------------------------------------------------- end-to-end ABI path
+def test_run_host_end_to_end():
+    d = W.cfg2(2, 8, 16, 16)
+    x = W.make_inputs(d)
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    from harness import TORCH_DT
+    op = FusedOp(d)
+    dev = device_tensors(d, x)
+    host = {"x": torch.from_numpy(x["x"]).pin_memory()}
+    for n in ("gamma", "beta", "mean", "var"):
+        host[n] = torch.from_numpy(x[n]).pin_memory()
+    host["y"] = torch.empty(dev["y"].numel(), dtype=TORCH_DT["f16"]).pin_memory()
+    dev["x"].zero_()
+    op.run_host(host, dev)
+    torch.cuda.synchronize()
+    assert_bitexact(host["y"].numpy(), O.run(d, x)["y"], "y")
