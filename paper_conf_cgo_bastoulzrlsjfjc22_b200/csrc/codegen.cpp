@@ -193,7 +193,8 @@ struct Gen {
     return "(" + idx + ")(" + s + ")";
   }
 
-  void header(const std::string& name, int minblocks) {
+  void header(const std::string& name, int /*unused*/) {
+    const int minblocks = std::max(1, L.minblocks);
     o.l("// generated by libfop (planner + codegen); skeleton: " + name);
     o.l("#include \"fop_device.cuh\"");
     o.l("typedef " + idx + " idx_t;");
@@ -374,12 +375,14 @@ struct Gen {
   // ------------------------------------------------------------ TRANSPOSE
   void gen_transpose() {
     const int W = L.width, WR = L.read_width;
+    const int U = std::max(1, L.unroll);
     const int64_t NTV = L.kl[0].extent / W, NTR = L.kl[1].extent / WR;
-    const int64_t TVH = (NTV + L.gv - 1) / L.gv, TRH = (NTR + L.gr - 1) / L.gr;
+    const int64_t TVH = (NTV + L.gv - 1) / L.gv;
+    const int64_t TRH = (NTR + (int64_t)L.gr * U - 1) / ((int64_t)L.gr * U);
     const int64_t STRIDE = L.grid * L.block;
     const XStmt& x = L.stmts[0];
     bool raw = x.move && es(x.write.tensor) == 2;
-    header("TRANSPOSE (register tile W x WR; both sides vectorised)", 1);
+    header("TRANSPOSE (register tiles W x WR, U per thread; both sides vectorised)", 1);
     o.l("const idx_t tid = (idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x;");
     o.l("#pragma unroll 1");
     o.l("for (idx_t g = tid; g < (idx_t)" + num(L.work) + "ull; g += (idx_t)" + num(STRIDE) + "ull) {");
@@ -390,95 +393,134 @@ struct Gen {
     o.l("const idx_t tv_hi = t % " + num(TVH) + "u; t /= " + num(TVH) + "u;");
     if (L.kl.size() > 2) o.l("const idx_t tr_hi = t % " + num(TRH) + "u; t /= " + num(TRH) + "u;");
     else o.l("const idx_t tr_hi = t;");
-    o.l("const idx_t tv = tv_hi * " + num(L.gv) + "u + tv_lo, tr = tr_hi * " + num(L.gr) + "u + tr_lo;");
-    o.l("if (tv >= " + num(NTV) + "u || tr >= " + num(NTR) + "u) continue;");
-    o.l("const idx_t iv = tv * " + num(W) + "u, ir = tr * " + num(WR) + "u;");
-    std::vector<std::pair<int, std::string>> its = {{0, "iv"}, {1, "ir"}};
-    decompose("t", 2, (int)L.kl.size(), "", its);
+    o.l("const idx_t tv = tv_hi * " + num(L.gv) + "u + tv_lo;");
+    o.l("if (tv >= " + num(NTV) + "u) continue;");
+    o.l("const idx_t iv = tv * " + num(W) + "u;");
+    std::vector<std::pair<int, std::string>> outer;
+    decompose("t", 2, (int)L.kl.size(), "", outer);
     // loads: A = vector along d_v [b][a]; B = vector along d_r [a][b]; S = scalar; G = gather [a][b]
+    // A/B vectors are kept as raw words until the tile is computed (fewer registers per byte in flight)
     std::vector<char> kind(L.loads.size());
-    for (size_t k = 0; k < L.loads.size(); k++) {
-      const Affine& a = L.loads[k];
-      int64_t cv = C(a, 0), cr = C(a, 1);
-      std::string off = affine(a, its);
-      std::string nm = "L" + num(k);
-      std::string dt = dtn(d.t[a.tensor].dtype);
-      std::string ety = raw ? "u32" : "float";
-      if (cv == 1) {
-        kind[k] = 'A';
-        o.l(ety + " " + nm + "[" + num(WR) + "][" + num(W) + "];");
-        o.l("#pragma unroll");
-        o.l("for (int b = 0; b < " + num(WR) + "; ++b) " +
-            (raw ? "fop::vload_raw<" + num(es(a.tensor)) + ", "
-                 : "fop::vload<" + dt + ", ") +
-            num(W) + ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + nm + "[b], " +
-            ptr(a.tensor, off + " + b * " + num(cr)) + ");");
-      } else if (cr == 1) {
-        kind[k] = 'B';
-        o.l(ety + " " + nm + "[" + num(W) + "][" + num(WR) + "];");
-        o.l("#pragma unroll");
-        o.l("for (int a = 0; a < " + num(W) + "; ++a) " +
-            (raw ? "fop::vload_raw<" + num(es(a.tensor)) + ", "
-                 : "fop::vload<" + dt + ", ") +
-            num(WR) + ", " + num(L.load_cb_r[k]) + ", " + pol(a, false) + ">(" + nm + "[a], " +
-            ptr(a.tensor, off + " + a * " + num(cv)) + ");");
-      } else if (cv == 0 && cr == 0) {
-        kind[k] = 'S';
-        o.l("const float " + nm + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
-      } else {
-        kind[k] = 'G';
-        o.l("float " + nm + "[" + num(W) + "][" + num(WR) + "];");
-        o.l("#pragma unroll");
-        o.l("for (int a = 0; a < " + num(W) + "; ++a)");
-        o.l("#pragma unroll");
-        o.l("for (int b = 0; b < " + num(WR) + "; ++b) " + nm + "[a][b] = fop::sload<" + dt + ", " +
-            pol(a, false) + ">(" + ptr(a.tensor, off + " + a * " + num(cv) + " + b * " + num(cr)) + ");");
+    std::vector<int> wpv(L.loads.size(), 0);
+    std::vector<std::vector<std::pair<int, std::string>>> its(U);
+    for (int u = 0; u < U; u++) {
+      std::string t = "_" + num(u);
+      o.l("const idx_t tr" + t + " = tr_hi * " + num((int64_t)L.gr * U) + "u + " + num((int64_t)u * L.gr) +
+          "u + tr_lo;");
+      o.l("const bool ok" + t + " = tr" + t + " < " + num(NTR) + "u;");
+      o.l("const idx_t ir" + t + " = tr" + t + " * " + num(WR) + "u;");
+      its[u] = {{0, "iv"}, {1, "ir" + t}};
+      its[u].insert(its[u].end(), outer.begin(), outer.end());
+      for (size_t k = 0; k < L.loads.size(); k++) {
+        const Affine& a = L.loads[k];
+        int64_t cv = C(a, 0), cr = C(a, 1);
+        std::string off = affine(a, its[u]);
+        std::string nm = "L" + num(k) + t;
+        std::string dt = dtn(d.t[a.tensor].dtype);
+        int eb = es(a.tensor);
+        if (cv == 1 || cr == 1) {
+          kind[k] = cv == 1 ? 'A' : 'B';
+          int n_in = cv == 1 ? W : WR, n_out = cv == 1 ? WR : W;   // vector length, vector count
+          int cb = cv == 1 ? L.load_cb[k] : L.load_cb_r[k];
+          int64_t step = cv == 1 ? cr : cv;
+          std::string vloop = cv == 1 ? "b" : "a";
+          if (raw) {
+            o.l("u32 " + nm + "[" + num(n_out) + "][" + num(n_in) + "];");
+            o.l("#pragma unroll");
+            o.l("for (int " + vloop + " = 0; " + vloop + " < " + num(n_out) + "; ++" + vloop + ") if (ok" + t +
+                ") fop::vload_raw<" + num(eb) + ", " + num(n_in) + ", " + num(cb) + ", " + pol(a, false) + ">(" +
+                nm + "[" + vloop + "], " + ptr(a.tensor, off + " + " + vloop + " * " + num(step)) + ");");
+          } else if (n_in * eb >= 4 && cb >= 4) {
+            wpv[k] = n_in * eb / 4;
+            o.l("u32 W" + nm + "[" + num(n_out) + "][" + num(wpv[k]) + "];");
+            o.l("#pragma unroll");
+            o.l("for (int " + vloop + " = 0; " + vloop + " < " + num(n_out) + "; ++" + vloop + ") if (ok" + t +
+                ") fop::vload_words<" + dt + ", " + num(n_in) + ", " + num(cb) + ", " + pol(a, false) + ">(W" + nm +
+                "[" + vloop + "], " + ptr(a.tensor, off + " + " + vloop + " * " + num(step)) + ");");
+          } else {
+            o.l("float " + nm + "[" + num(n_out) + "][" + num(n_in) + "];");
+            o.l("#pragma unroll");
+            o.l("for (int " + vloop + " = 0; " + vloop + " < " + num(n_out) + "; ++" + vloop + ") if (ok" + t +
+                ") fop::vload<" + dt + ", " + num(n_in) + ", " + num(cb) + ", " + pol(a, false) + ">(" + nm + "[" +
+                vloop + "], " + ptr(a.tensor, off + " + " + vloop + " * " + num(step)) + ");");
+          }
+        } else if (cv == 0 && cr == 0) {
+          kind[k] = 'S';
+          o.l("float " + nm + " = 0.f;");
+          o.l("if (ok" + t + ") " + nm + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
+        } else {
+          kind[k] = 'G';
+          o.l("float " + nm + "[" + num(W) + "][" + num(WR) + "];");
+          o.l("#pragma unroll");
+          o.l("for (int a = 0; a < " + num(W) + "; ++a)");
+          o.l("#pragma unroll");
+          o.l("for (int b = 0; b < " + num(WR) + "; ++b) if (ok" + t + ") " + nm + "[a][b] = fop::sload<" + dt +
+              ", " + pol(a, false) + ">(" + ptr(a.tensor, off + " + a * " + num(cv) + " + b * " + num(cr)) + ");");
+        }
       }
     }
-    std::string woff = affine(x.write, its);
     int64_t cwr = C(x.write, 1);
     std::string dto = dtn(x.out_dtype);
-    if (raw) {
-      int k = x.nodes[x.result].acc;
-      o.l("u32 O[" + num(WR) + "][" + num(W) + "];");
-      o.l("#pragma unroll");
-      o.l("for (int b = 0; b < " + num(WR) + "; ++b)");
-      o.l("#pragma unroll");
-      o.l("for (int a = 0; a < " + num(W) + "; ++a) O[b][a] = " +
-          std::string(kind[k] == 'A' ? "L" + num(k) + "[b][a]" : "L" + num(k) + "[a][b]") + ";");
-      o.l("#pragma unroll");
-      o.l("for (int b = 0; b < " + num(WR) + "; ++b) fop::vstore_raw<" + num(es(x.write.tensor)) + ", " + num(W) +
-          ", " + num(L.store_cb[0]) + ", " + spol() + ">(" + ptr(x.write.tensor, woff + " + b * " + num(cwr)) +
-          ", O[b]);");
-    } else {
-      DagCtx c;
-      c.tag = "";
-      c.load_varies = [&](int k) { return kind[k] != 'S'; };
-      c.load = [&](int k) {
-        std::string nm = "L" + num(k);
-        switch (kind[k]) {
-          case 'A': return nm + "[b][a]";
-          case 'S': return nm;
-          default: return nm + "[a][b]";
-        }
-      };
-      c.fwd = [&](int) { return std::string("0.f"); };
-      c.scalar = [&](int) { return std::string("0.f"); };
-      auto var = varies(x, c);
-      emit_nodes(o, x, var, false, c);
-      o.l("float O[" + num(WR) + "][" + num(W) + "];");
-      o.l("#pragma unroll");
-      o.l("for (int b = 0; b < " + num(WR) + "; ++b) {");
-      o.l("#pragma unroll");
-      o.l("for (int a = 0; a < " + num(W) + "; ++a) {");
+    for (int u = 0; u < U; u++) {
+      std::string t = "_" + num(u);
+      std::string woff = affine(x.write, its[u]);
+      o.l("if (ok" + t + ") {");
       o.ind++;
-      emit_nodes(o, x, var, true, c);
-      o.l("O[b][a] = " + node_name(x, var, x.result, c) + ";");
+      if (raw) {
+        int k = x.nodes[x.result].acc;
+        o.l("u32 O[" + num(WR) + "][" + num(W) + "];");
+        o.l("#pragma unroll");
+        o.l("for (int b = 0; b < " + num(WR) + "; ++b)");
+        o.l("#pragma unroll");
+        o.l("for (int a = 0; a < " + num(W) + "; ++a) O[b][a] = " +
+            std::string(kind[k] == 'A' ? "L" + num(k) + t + "[b][a]" : "L" + num(k) + t + "[a][b]") + ";");
+        o.l("#pragma unroll");
+        o.l("for (int b = 0; b < " + num(WR) + "; ++b) fop::vstore_raw<" + num(es(x.write.tensor)) + ", " +
+            num(W) + ", " + num(L.store_cb[0]) + ", " + spol() + ">(" +
+            ptr(x.write.tensor, woff + " + b * " + num(cwr)) + ", O[b]);");
+      } else {
+        for (size_t k = 0; k < L.loads.size(); k++) {
+          if (!wpv[k]) continue;
+          bool A = kind[k] == 'A';
+          int n_in = A ? W : WR, n_out = A ? WR : W;
+          std::string nm = "L" + num(k) + t;
+          o.l("float " + nm + "[" + num(n_out) + "][" + num(n_in) + "];");
+          o.l("#pragma unroll");
+          o.l("for (int q = 0; q < " + num(n_out) + "; ++q) fop::cvt_words<" +
+              std::string(dtn(d.t[L.loads[k].tensor].dtype)) + ", " + num(n_in) + ">(" + nm + "[q], W" + nm + "[q]);");
+        }
+        DagCtx c;
+        c.tag = t;
+        c.load_varies = [&](int k) { return kind[k] != 'S'; };
+        c.load = [&, t](int k) {
+          std::string nm = "L" + num(k) + t;
+          switch (kind[k]) {
+            case 'A': return nm + "[b][a]";
+            case 'S': return nm;
+            default: return nm + "[a][b]";
+          }
+        };
+        c.fwd = [&](int) { return std::string("0.f"); };
+        c.scalar = [&](int) { return std::string("0.f"); };
+        auto var = varies(x, c);
+        emit_nodes(o, x, var, false, c);
+        o.l("float O[" + num(WR) + "][" + num(W) + "];");
+        o.l("#pragma unroll");
+        o.l("for (int b = 0; b < " + num(WR) + "; ++b) {");
+        o.l("#pragma unroll");
+        o.l("for (int a = 0; a < " + num(W) + "; ++a) {");
+        o.ind++;
+        emit_nodes(o, x, var, true, c);
+        o.l("O[b][a] = " + node_name(x, var, x.result, c) + ";");
+        o.ind--;
+        o.l("}}");
+        o.l("#pragma unroll");
+        o.l("for (int b = 0; b < " + num(WR) + "; ++b) fop::vstore<" + dto + ", " + num(W) + ", " +
+            num(L.store_cb[0]) + ", " + spol() + ">(" + ptr(x.write.tensor, woff + " + b * " + num(cwr)) +
+            ", O[b]);");
+      }
       o.ind--;
-      o.l("}}");
-      o.l("#pragma unroll");
-      o.l("for (int b = 0; b < " + num(WR) + "; ++b) fop::vstore<" + dto + ", " + num(W) + ", " +
-          num(L.store_cb[0]) + ", " + spol() + ">(" + ptr(x.write.tensor, woff + " + b * " + num(cwr)) + ", O[b]);");
+      o.l("}");
     }
     o.ind--;
     o.l("}");
@@ -503,12 +545,101 @@ struct Gen {
       if (x.kind == FOP_ASSIGN && x.fwd && !regmode && !x.store)
         fail(FOP_E_UNSUPPORTED, "ROW_REDUCE: a long forwarded row must be stored to be re-read");
     if (NRO > 64) fail(FOP_E_UNSUPPORTED, "ROW_REDUCE: too many outer reduction iterations");
+    const int NP = (int)(NRO * K);   // vectors per lane per row
+    // per-load treatment: hoisted (independent of the row: e.g. a bias, loaded
+    // once per warp), prefetched (streaming vector of the first phase, loaded
+    // one row ahead so the reductions overlap the next row's HBM latency), or
+    // plain
+    std::vector<char> mode(L.loads.size(), 'L');
+    std::vector<bool> used0(L.loads.size(), false);
+    for (auto& n : L.stmts[0].nodes)
+      if (n.op == FOP_OP_LOAD) used0[n.acc] = true;
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      const Affine& a = L.loads[k];
+      bool row_inv = true;
+      for (size_t q = L.nsplit; q < L.kl.size(); q++) row_inv &= C(a, (int)q) == 0;
+      int64_t cv = C(a, 0);
+      int es_k = es(a.tensor);
+      if (row_inv && regmode && (cv == 0 || cv == 1) && !written_here(a.tensor)) mode[k] = 'H';
+      else if (L.row_prefetch && used0[k] && cv == 1 && W * es_k >= 4 && L.load_cb[k] >= 4 &&
+               NP * W * es_k / 4 <= 32 && !written_here(a.tensor))
+        mode[k] = 'P';
+    }
+    auto ro_its = [&](int64_t ro, const std::vector<std::pair<int, std::string>>& base) {
+      std::vector<std::pair<int, std::string>> its = base;
+      int64_t rem = ro;
+      for (int k = 1; k < L.nsplit; k++) {
+        its.push_back({k, num(rem % L.kl[k].extent) + "u"});
+        rem /= L.kl[k].extent;
+      }
+      return its;
+    };
+    auto lane_guard = [&](int kk) {
+      return jguard ? "if (lane + " + num(32 * kk) + "u < " + num(NVD) + "u) " : std::string("");
+    };
     header("ROW_REDUCE (one warp per row, lanes across d_v vectors, butterfly)", 1);
     o.l("const idx_t lane = threadIdx.x & 31u;");
+    // hoisted row-invariant loads
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      if (mode[k] != 'H') continue;
+      const Affine& a = L.loads[k];
+      std::string dt = dtn(d.t[a.tensor].dtype);
+      bool vec = C(a, 0) == 1;
+      o.l("float H" + num(k) + "[" + num(NP) + "]" + (vec ? "[" + num(W) + "]" : "") + ";");
+      for (int64_t ro = 0; ro < NRO; ro++)
+        for (int kk = 0; kk < K; kk++) {
+          auto its = ro_its(ro, {});
+          its.push_back({0, "((lane + " + num(32 * kk) + "u) * " + num(W) + "u)"});
+          std::string off = affine(a, its);
+          std::string dst = "H" + num(k) + "[" + num(ro * K + kk) + "]";
+          if (vec)
+            o.l(lane_guard(kk) + "fop::vload<" + dt + ", " + num(W) + ", " + num(L.load_cb[k]) + ", " +
+                pol(a, true) + ">(" + dst + ", " + ptr(a.tensor, off) + ");");
+          else
+            o.l(dst + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
+        }
+    }
+    // prefetch of the first row's streaming loads
+    auto emit_prefetch = [&](const std::string& rowvar, const std::string& tag) {
+      bool any = false;
+      for (size_t k = 0; k < L.loads.size(); k++) any |= mode[k] == 'P';
+      if (!any) return;
+      o.l("if (" + rowvar + " < (idx_t)" + num(rows) + "ull) {");
+      o.ind++;
+      o.l("idx_t pr = " + rowvar + ";");
+      std::vector<std::pair<int, std::string>> pits;
+      decompose("pr", L.nsplit, (int)L.kl.size(), tag, pits);
+      for (size_t k = 0; k < L.loads.size(); k++) {
+        if (mode[k] != 'P') continue;
+        const Affine& a = L.loads[k];
+        int wpv = W * es(a.tensor) / 4;
+        for (int64_t ro = 0; ro < NRO; ro++)
+          for (int kk = 0; kk < K; kk++) {
+            auto its = ro_its(ro, pits);
+            its.push_back({0, "((lane + " + num(32 * kk) + "u) * " + num(W) + "u)"});
+            o.l(lane_guard(kk) + "fop::vload_words<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + num(W) +
+                ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(&P" + num(k) + "[" +
+                num((ro * K + kk) * wpv) + "], " + ptr(a.tensor, affine(a, its)) + ");");
+          }
+      }
+      o.ind--;
+      o.l("}");
+    };
+    for (size_t k = 0; k < L.loads.size(); k++)
+      if (mode[k] == 'P') o.l("u32 P" + num(k) + "[" + num(NP * W * es(L.loads[k].tensor) / 4) + "];");
+    o.l("idx_t row = ((idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x) >> 5;");
+    emit_prefetch("row", "_p");
     o.l("#pragma unroll 1");
-    o.l("for (idx_t row = ((idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x) >> 5; row < (idx_t)" +
-        num(rows) + "ull; row += (idx_t)" + num(WSTRIDE) + "ull) {");
+    o.l("for (; row < (idx_t)" + num(rows) + "ull; row += (idx_t)" + num(WSTRIDE) + "ull) {");
     o.ind++;
+    for (size_t k = 0; k < L.loads.size(); k++)
+      if (mode[k] == 'P') {
+        int n = NP * W * es(L.loads[k].tensor) / 4;
+        o.l("u32 Q" + num(k) + "[" + num(n) + "];");
+        o.l("#pragma unroll");
+        o.l("for (int i = 0; i < " + num(n) + "; ++i) Q" + num(k) + "[i] = P" + num(k) + "[i];");
+      }
+    emit_prefetch("row + (idx_t)" + num(WSTRIDE) + "ull", "_n");
     o.l("idx_t rr = row;");
     std::vector<std::pair<int, std::string>> rits;
     decompose("rr", L.nsplit, (int)L.kl.size(), "", rits);
@@ -517,7 +648,7 @@ struct Gen {
       const XStmt& x = L.stmts[si];
       bool red = x.kind == FOP_REDUCE;
       o.l("// statement " + num(x.stmt) + (red ? " (REDUCE)" : " (ASSIGN)"));
-      if (red) o.l(std::string("float acc") + num(x.stmt) + " = " + (x.redop == FOP_RED_MAX ? "-INFINITY" : "0.f") + ";");
+      if (red) o.l(std::string("float acc") + num(x.stmt) + " = " + (x.redop == FOP_RED_MAX ? "__uint_as_float(0xff800000u)" : "0.f") + ";");
       if (x.kind == FOP_ASSIGN && x.fwd && regmode) o.l("float F" + num(x.stmt) + "[" + num(NRO * K * W) + "];");
       for (int64_t ro = 0; ro < NRO; ro++) {
         // compile-time decomposition of ro over the outer reduction kloops
@@ -546,7 +677,15 @@ struct Gen {
             std::string off = affine(a, its2);
             std::string nm = "L" + num(k);
             std::string dt = dtn(d.t[a.tensor].dtype);
-            if (cv == 0) {
+            int64_t vi = ro * K + kk;
+            if (mode[k] == 'H') {
+              if (cv == 0) o.l("const float " + nm + " = H" + num(k) + "[" + num(vi) + "];");
+              else o.l("const float* " + nm + " = H" + num(k) + "[" + num(vi) + "];");
+            } else if (mode[k] == 'P') {
+              int wpv = W * es(a.tensor) / 4;
+              o.l("float " + nm + "[" + num(W) + "];");
+              o.l("fop::cvt_words<" + dt + ", " + num(W) + ">(" + nm + ", &Q" + num(k) + "[" + num(vi * wpv) + "]);");
+            } else if (cv == 0) {
               o.l("const float " + nm + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
             } else if (cv == 1) {
               o.l("float " + nm + "[" + num(W) + "];");
@@ -650,7 +789,7 @@ struct Gen {
     const int64_t RPC = (ROWS + NCH - 1) / NCH;
     const int SW = L.gv * W;
     bool isMax = x.redop == FOP_RED_MAX;
-    std::string init = isMax ? "-INFINITY" : "0.f";
+    std::string init = isMax ? "__uint_as_float(0xff800000u)" : "0.f";
     auto comb = [&](const std::string& a, const std::string& b) {
       return isMax ? "fop::op_max(" + a + ", " + b + ")" : "__fadd_rn(" + a + ", " + b + ")";
     };

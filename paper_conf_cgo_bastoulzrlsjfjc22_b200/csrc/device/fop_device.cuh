@@ -184,6 +184,31 @@ __device__ __forceinline__ void vload(float* v, const char* p) {
   }
 }
 
+// split form of vload for software prefetch: raw words now, conversion later
+template <int DT, int N, int CB, int POL>
+__device__ __forceinline__ void vload_words(u32* w, const char* p) {
+  constexpr int TOT = N * ES<DT>::v;
+  static_assert(CB >= 4 && TOT % CB == 0, "word-granular vectors only");
+#pragma unroll
+  for (int c = 0; c < TOT / CB; ++c) ldraw<CB, POL>(w + c * (CB / 4), p + c * CB);
+}
+template <int DT, int N>
+__device__ __forceinline__ void cvt_words(float* v, const u32* w) {
+  constexpr int TOT = N * ES<DT>::v;
+#pragma unroll
+  for (int i = 0; i < TOT / 4; ++i) {
+    if constexpr (DT == F32 || DT == I32) {
+      v[i] = __uint_as_float(w[i]);
+    } else if constexpr (DT == F16) {
+      v[2 * i] = h2f((u16)(w[i] & 0xffffu));
+      v[2 * i + 1] = h2f((u16)(w[i] >> 16));
+    } else {
+      v[2 * i] = __uint_as_float(w[i] << 16);
+      v[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u);
+    }
+  }
+}
+
 // fp32 -> N elements of type DT at p (RNE conversion)
 template <int DT, int N, int CB, int POL>
 __device__ __forceinline__ void vstore(char* p, const float* v) {

@@ -106,6 +106,8 @@ struct Launch {
   std::vector<int> load_cb_r;     // TRANSPOSE: per load chunk bytes along d_r
   std::vector<int> store_cb;      // per stmt: vector chunk bytes of the store (0 = scalar)
   int unroll = 1;
+  int minblocks = 1;              // __launch_bounds__ min blocks/SM; grid-stride grids = SMs x minblocks
+  int row_prefetch = 0;           // ROW: prefetch the next row's streaming loads
   int gv = 1, gr = 1;             // lanes along d_v / along the other tiled dim
   int64_t nchunks = 1;            // COL: row chunks
   int64_t work = 0;               // total work items (threads' units)

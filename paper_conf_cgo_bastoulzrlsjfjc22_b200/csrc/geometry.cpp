@@ -18,6 +18,7 @@
 // (coalescing, goal (ii) of P:297).  Loops that are contiguous for every
 // access are collapsed (a B200 step beyond the paper).
 #include <algorithm>
+#include <cstdlib>
 #include <string>
 
 #include "fop_internal.h"
@@ -234,22 +235,31 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.align[t] = std::max({L.align[t], L.store_cb[k], esize(d.t[t].dtype)});
   }
 
-  // ---- a5: launch geometry
+  // ---- a5: launch geometry.  Grid-stride classes launch exactly the blocks
+  // that are resident at once (SMs x minblocks, guaranteed by
+  // __launch_bounds__(block, minblocks)): one wave, no tail wave.
+  // FOP_<CLASS>_U / FOP_<CLASS>_MINB override the defaults (tuning sweeps).
   int64_t prod_rest = 1;
-  L.block = 256;
   L.ws_bytes = 0;
+  auto knob = [](const char* name, int dflt) {
+    const char* e = std::getenv(name);
+    return e && *e ? std::atoi(e) : dflt;
+  };
+  L.block = knob("FOP_BLOCK", 256);
   if (L.kclass == FOP_CLASS_EW) {
     for (size_t k = 1; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
     int64_t nv = (EV + W - 1) / W;
     L.work = nv * prod_rest;
+    // bytes each work item loads; ~128 B of loads in flight per thread at
+    // 512-768 threads/SM measured best on B200 (tools/sweep.py)
     int bytes = 0;
     for (size_t k = 0; k < L.loads.size(); k++)
-      if (L.load_cb[k]) bytes += W * esize(d.t[L.loads[k].tensor].dtype);
-    for (size_t k = 0; k < L.stmts.size(); k++)
-      if (L.store_cb[k]) bytes += W * esize(L.stmts[k].out_dtype);
-    L.unroll = bytes <= 32 ? 4 : (bytes <= 64 ? 2 : 1);
+      if (coef(L, L.loads[k], 0) != 0) bytes += W * esize(d.t[L.loads[k].tensor].dtype);
+    int u = bytes > 0 ? std::max(1, std::min(8, pow2_floor(std::max(1, 128 / bytes)))) : 4;
+    L.unroll = knob("FOP_EW_U", u);
+    L.minblocks = knob("FOP_EW_MINB", L.unroll >= 4 ? 2 : 3);
     int64_t need = (L.work + (int64_t)L.block * L.unroll - 1) / ((int64_t)L.block * L.unroll);
-    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * (2048 / L.block)));
+    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
   } else if (L.kclass == FOP_CLASS_TRANSPOSE) {
     for (size_t k = 2; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
     int64_t ntv = EV / W, ntr = L.kl[1].extent / L.read_width;
@@ -259,16 +269,22 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.gv = gv;
     L.gr = 32 / gv;
     int64_t tvh = (ntv + gv - 1) / gv, trh = (ntr + L.gr - 1) / L.gr;
+    // U tiles per thread, adjacent along d_r (tr, tr+gr, ...): a warp's loads
+    // of consecutive tiles complete the same 128 B lines back to back
+    L.unroll = std::max(1, knob("FOP_TR_U", 2));
+    trh = (ntr + (int64_t)L.gr * L.unroll - 1) / ((int64_t)L.gr * L.unroll);
     L.work = (int64_t)gv * L.gr * tvh * trh * prod_rest;
-    L.unroll = 1;
+    L.minblocks = knob("FOP_TR_MINB", L.unroll >= 2 ? 1 : 2);
     int64_t need = (L.work + L.block - 1) / L.block;
-    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * (2048 / L.block)));
+    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
   } else if (L.kclass == FOP_CLASS_ROW_REDUCE) {
     int64_t rows = 1;
     for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
     L.work = rows;  // one warp per row
+    L.minblocks = knob("FOP_ROW_MINB", 3);
+    L.row_prefetch = knob("FOP_ROW_PREFETCH", 1);
     int64_t need = (rows + L.block / 32 - 1) / (L.block / 32);
-    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * (2048 / L.block)));
+    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
     L.unroll = 1;
   } else {  // COL_REDUCE
     int64_t nvd = EV / W;
@@ -284,13 +300,14 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     for (int k = 1; k < L.nsplit; k++) slabs *= L.kl[k].extent;
     int64_t rows = 1;
     for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
-    int64_t target = (int64_t)sms * 4;
-    int64_t nch = std::max<int64_t>(1, (target + slabs / 2) / std::max<int64_t>(1, slabs));
+    L.minblocks = knob("FOP_COL_MINB", 2);
+    L.unroll = knob("FOP_COL_U", 8);
+    int64_t target = (int64_t)sms * L.minblocks;   // one resident wave
+    int64_t nch = std::max<int64_t>(1, target / std::max<int64_t>(1, slabs));
     nch = std::min<int64_t>(nch, std::max<int64_t>(1, (rows + L.gr - 1) / L.gr));
     L.nchunks = nch;
     L.work = rows;
     L.grid = slabs * nch;
-    L.unroll = 4;
     if (nch > 1) {
       size_t part = (size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(float);
       part = (part + 255) & ~size_t(255);
