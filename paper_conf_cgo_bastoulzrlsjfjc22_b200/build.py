@@ -68,7 +68,7 @@ def nvcc_check(sources, out_dir=None):
             f.write(src)
         cub = os.path.join(out_dir, name + ".cubin")
         subprocess.check_call(["nvcc", "-cubin", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a",
-                               "-lineinfo", "-O3", "-I", inc, "-o", cub, cu])
+                               "-lineinfo", "-O3", "-fmad=false", "-I", inc, "-o", cub, cu])
         cubins.append(cub)
     return cubins
 

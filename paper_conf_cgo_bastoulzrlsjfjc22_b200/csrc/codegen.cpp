@@ -76,13 +76,16 @@ std::string op_expr(const XNode& n, const std::string& a, const std::string& b) 
   return "0.f";
 }
 
-// Emission context for one statement at one "point" (work item)
+// Emission context for one statement at one "point" (work item).  Element
+// expressions are built for an element index expression `e` (a loop variable
+// in the scalar loop, 2*p / 2*p+1 in the packed loop).
 struct DagCtx {
-  std::function<std::string(int)> load;       // element expression of load k
+  std::function<std::string(int, const std::string&)> load;  // element expression of load k
   std::function<bool(int)> load_varies;
-  std::function<std::string(int)> fwd;        // element expression of forwarded stmt
-  std::function<std::string(int)> scalar;     // per-row scalar of a REDUCE
-  std::string tag;                            // name suffix
+  std::function<std::string(int, const std::string&)> fwd;   // element expression of forwarded stmt
+  std::function<std::string(int)> scalar;                    // per-row scalar of a REDUCE
+  std::string tag;                                           // name suffix
+  std::string ev = "e";                                      // scalar element loop variable
 };
 
 std::vector<bool> varies(const XStmt& x, const DagCtx& c) {
@@ -114,15 +117,16 @@ std::vector<bool> reachable(const XStmt& x) {
   return r;
 }
 
-// emit nodes with var==want; returns nothing, defines names
-void emit_nodes(Out& o, const XStmt& x, const std::vector<bool>& var, bool want, const DagCtx& c) {
+// emit nodes with var==want (scalar form); defines names
+void emit_nodes(Out& o, const XStmt& x, const std::vector<bool>& var, bool want, const DagCtx& c,
+                int skip = -1) {
   std::vector<bool> reach = reachable(x);
   for (size_t i = 0; i < x.nodes.size(); i++) {
-    if (!reach[i] || var[i] != want) continue;
+    if (!reach[i] || var[i] != want || (int)i == skip) continue;
     const XNode& n = x.nodes[i];
     std::string e;
-    if (n.op == FOP_OP_LOAD) e = c.load(n.acc);
-    else if (n.op == X_FWD) e = c.fwd(n.src);
+    if (n.op == FOP_OP_LOAD) e = c.load(n.acc, c.ev);
+    else if (n.op == X_FWD) e = c.fwd(n.src, c.ev);
     else if (n.op == X_SCALAR) e = c.scalar(n.src);
     else {
       std::string a = n.a >= 0 ? node_name(x, var, n.a, c) : "";
@@ -131,6 +135,83 @@ void emit_nodes(Out& o, const XStmt& x, const std::vector<bool>& var, bool want,
     }
     o.l("const float " + node_name(x, var, (int)i, c) + " = " + e + ";");
   }
+}
+
+// packed (fp32x2) form of the varying nodes: one value = elements (2p, 2p+1)
+std::string pair_name(const XStmt& x, int i, const DagCtx& c) {
+  return "w" + num(x.stmt) + "_" + num(i) + c.tag;
+}
+void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, const DagCtx& c, const std::string& p,
+                       int skip = -1) {
+  std::vector<bool> reach = reachable(x);
+  const std::string e0 = "2 * " + p, e1 = "2 * " + p + " + 1";
+  auto opnd = [&](int i) { return var[i] ? pair_name(x, i, c) : "fop::pk1(" + node_name(x, var, i, c) + ")"; };
+  // a packed product feeding a packed add/sub must not be contracted (see fop::nofuse)
+  auto addend = [&](int i) {
+    return var[i] && x.nodes[i].op == FOP_OP_MUL ? "fop::nofuse(" + pair_name(x, i, c) + ", fop_zero)" : opnd(i);
+  };
+  for (size_t i = 0; i < x.nodes.size(); i++) {
+    if (!reach[i] || !var[i] || (int)i == skip) continue;
+    const XNode& n = x.nodes[i];
+    std::string e;
+    switch (n.op) {
+      case FOP_OP_LOAD: e = "fop::pk(" + c.load(n.acc, e0) + ", " + c.load(n.acc, e1) + ")"; break;
+      case X_FWD: e = "fop::pk(" + c.fwd(n.src, e0) + ", " + c.fwd(n.src, e1) + ")"; break;
+      case FOP_OP_ADD: e = "fop::add2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
+      case FOP_OP_SUB: e = "fop::sub2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
+      case FOP_OP_MUL: e = "fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + ")"; break;
+      case FOP_OP_GELU_TANH: e = "fop::op_gelu_tanh2(" + opnd(n.a) + ")"; break;
+      default: {  // no packed form: per lane
+        auto lane = [&](const char* f, int k) {
+          return k < 0 ? std::string("") : (var[k] ? std::string("fop::") + f + "(" + pair_name(x, k, c) + ")"
+                                                   : node_name(x, var, k, c));
+        };
+        e = "fop::pk(" + op_expr(n, lane("lo", n.a), lane("lo", n.b)) + ", " +
+            op_expr(n, lane("hi", n.a), lane("hi", n.b)) + ")";
+      }
+    }
+    o.l("const u64 " + pair_name(x, (int)i, c) + " = " + e + ";");
+  }
+}
+
+// The element loop of one statement.  W even and packing on: pairs with
+// FADD2/FMUL2/FFMA2; otherwise scalar.  A SUM reduction whose term ends in a
+// product hands the two factors to `fma` (contracted into the accumulator,
+// reading R23) instead of materialising the product.
+struct Sink {
+  std::function<void(const std::string&)> scalar;                          // value, element var c.ev
+  std::function<void(const std::string&, const std::string&)> pair;        // packed value, pair var
+  std::function<void(const std::string&, const std::string&, const std::string&)> pair_fma;  // a, b, pair var
+};
+bool g_packed = true;
+void emit_elems(Out& o, const XStmt& x, const std::vector<bool>& var, const DagCtx& c, int W, const Sink& s) {
+  bool packed = g_packed && W % 2 == 0 && s.pair;
+  if (!packed) {
+    o.l("#pragma unroll");
+    o.l("for (int " + c.ev + " = 0; " + c.ev + " < " + num(W) + "; ++" + c.ev + ") {");
+    o.ind++;
+    emit_nodes(o, x, var, true, c);
+    s.scalar(node_name(x, var, x.result, c));
+    o.ind--;
+    o.l("}");
+    return;
+  }
+  std::string p = c.ev + "p";
+  const XNode& r = x.nodes[x.result];
+  bool fma = s.pair_fma && r.op == FOP_OP_MUL && var[x.result];
+  int uses = 0;
+  for (auto& n : x.nodes) uses += (n.a == x.result) + (n.b == x.result);
+  fma = fma && uses == 0;
+  o.l("#pragma unroll");
+  o.l("for (int " + p + " = 0; " + p + " < " + num(W / 2) + "; ++" + p + ") {");
+  o.ind++;
+  emit_nodes_packed(o, x, var, c, p, fma ? x.result : -1);
+  auto opnd = [&](int i) { return var[i] ? pair_name(x, i, c) : "fop::pk1(" + node_name(x, var, i, c) + ")"; };
+  if (fma) s.pair_fma(opnd(r.a), opnd(r.b), p);
+  else if (var[x.result]) s.pair(pair_name(x, x.result, c), p);
+  else s.pair("fop::pk1(" + node_name(x, var, x.result, c) + ")", p);
+  o.ind--;
+  o.l("}");
 }
 
 std::string fin_expr(Out& o, const XStmt& x, const std::string& acc, const std::string& tag) {
@@ -209,6 +290,7 @@ struct Gen {
       o.l((written_here(t) ? std::string("char* __restrict__ T") : std::string("const char* __restrict__ T")) +
           num(t) + " = args.p[" + num(t) + "];");
     }
+    o.l("const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;");
   }
   void footer() {
     o.ind--;
@@ -328,20 +410,21 @@ struct Gen {
         DagCtx c;
         c.tag = t;
         c.load_varies = [&](int k) { return C(L.loads[k], 0) != 0; };
-        c.load = [&, t](int k) { return C(L.loads[k], 0) != 0 ? "L" + num(k) + t + "[e]" : "L" + num(k) + t; };
-        c.fwd = [&, t](int s) { return "F" + num(L.stmts[s].stmt) + t + "[e]"; };
+        c.load = [&, t](int k, const std::string& e) {
+          return C(L.loads[k], 0) != 0 ? "L" + num(k) + t + "[" + e + "]" : "L" + num(k) + t;
+        };
+        c.fwd = [&, t](int s, const std::string& e) { return "F" + num(L.stmts[s].stmt) + t + "[" + e + "]"; };
         c.scalar = [&](int) { return std::string("0.f"); };
         auto var = varies(x, c);
         emit_nodes(o, x, var, false, c);
         std::string R = "R" + num(x.stmt) + t;
         o.l("float " + R + "[" + num(W) + "];");
-        o.l("#pragma unroll");
-        o.l("for (int e = 0; e < " + num(W) + "; ++e) {");
-        o.ind++;
-        emit_nodes(o, x, var, true, c);
-        o.l(R + "[e] = " + node_name(x, var, x.result, c) + ";");
-        o.ind--;
-        o.l("}");
+        Sink sk;
+        sk.scalar = [&](const std::string& v) { o.l(R + "[e] = " + v + ";"); };
+        sk.pair = [&](const std::string& v, const std::string& p) {
+          o.l("fop::upk(" + v + ", " + R + "[2 * " + p + "], " + R + "[2 * " + p + " + 1]);");
+        };
+        emit_elems(o, x, var, c, W, sk);
         if (x.fwd) {
           o.l("float F" + num(x.stmt) + t + "[" + num(W) + "];");
           o.l("#pragma unroll");
@@ -491,29 +574,32 @@ struct Gen {
         }
         DagCtx c;
         c.tag = t;
+        c.ev = "a";
         c.load_varies = [&](int k) { return kind[k] != 'S'; };
-        c.load = [&, t](int k) {
+        c.load = [&, t](int k, const std::string& e) {
           std::string nm = "L" + num(k) + t;
           switch (kind[k]) {
-            case 'A': return nm + "[b][a]";
+            case 'A': return nm + "[b][" + e + "]";
             case 'S': return nm;
-            default: return nm + "[a][b]";
+            default: return nm + "[" + e + "][b]";
           }
         };
-        c.fwd = [&](int) { return std::string("0.f"); };
+        c.fwd = [&](int, const std::string&) { return std::string("0.f"); };
         c.scalar = [&](int) { return std::string("0.f"); };
         auto var = varies(x, c);
         emit_nodes(o, x, var, false, c);
         o.l("float O[" + num(WR) + "][" + num(W) + "];");
         o.l("#pragma unroll");
         o.l("for (int b = 0; b < " + num(WR) + "; ++b) {");
-        o.l("#pragma unroll");
-        o.l("for (int a = 0; a < " + num(W) + "; ++a) {");
         o.ind++;
-        emit_nodes(o, x, var, true, c);
-        o.l("O[b][a] = " + node_name(x, var, x.result, c) + ";");
+        Sink sk;
+        sk.scalar = [&](const std::string& v) { o.l("O[b][a] = " + v + ";"); };
+        sk.pair = [&](const std::string& v, const std::string& p) {
+          o.l("fop::upk(" + v + ", O[b][2 * " + p + "], O[b][2 * " + p + " + 1]);");
+        };
+        emit_elems(o, x, var, c, W, sk);
         o.ind--;
-        o.l("}}");
+        o.l("}");
         o.l("#pragma unroll");
         o.l("for (int b = 0; b < " + num(WR) + "; ++b) fop::vstore<" + dto + ", " + num(W) + ", " +
             num(L.store_cb[0]) + ", " + spol() + ">(" + ptr(x.write.tensor, woff + " + b * " + num(cwr)) +
@@ -648,7 +734,11 @@ struct Gen {
       const XStmt& x = L.stmts[si];
       bool red = x.kind == FOP_REDUCE;
       o.l("// statement " + num(x.stmt) + (red ? " (REDUCE)" : " (ASSIGN)"));
-      if (red) o.l(std::string("float acc") + num(x.stmt) + " = " + (x.redop == FOP_RED_MAX ? "__uint_as_float(0xff800000u)" : "0.f") + ";");
+      if (red) {
+        o.l(std::string("float acc") + num(x.stmt) + " = " +
+            (x.redop == FOP_RED_MAX ? "__uint_as_float(0xff800000u)" : "0.f") + ";");
+        if (x.redop == FOP_RED_SUM) o.l("u64 acc" + num(x.stmt) + "p = fop::pk1(0.f);");
+      }
       if (x.kind == FOP_ASSIGN && x.fwd && regmode) o.l("float F" + num(x.stmt) + "[" + num(NRO * K * W) + "];");
       for (int64_t ro = 0; ro < NRO; ro++) {
         // compile-time decomposition of ro over the outer reduction kloops
@@ -720,31 +810,48 @@ struct Gen {
           DagCtx c;
           c.tag = "";
           c.load_varies = load_varies_e;
-          c.load = [&](int k) { return C(L.loads[k], 0) != 0 ? "L" + num(k) + "[e]" : "L" + num(k); };
+          c.load = [&](int k, const std::string& e) {
+            return C(L.loads[k], 0) != 0 ? "L" + num(k) + "[" + e + "]" : "L" + num(k);
+          };
           int64_t base_idx = (ro * K + kk) * W;
-          c.fwd = [&, base_idx](int s) {
-            return regmode ? "F" + num(L.stmts[s].stmt) + "[" + num(base_idx) + " + e]"
-                           : "FW" + num(L.stmts[s].stmt) + "[e]";
+          c.fwd = [&, base_idx](int s, const std::string& e) {
+            return regmode ? "F" + num(L.stmts[s].stmt) + "[" + num(base_idx) + " + " + e + "]"
+                           : "FW" + num(L.stmts[s].stmt) + "[" + e + "]";
           };
           c.scalar = [&](int s) { return "S" + num(L.stmts[s].stmt); };
           auto var = varies(x, c);
           emit_nodes(o, x, var, false, c);
           if (!red) o.l("float R[" + num(W) + "];");
-          o.l("#pragma unroll");
-          o.l("for (int e = 0; e < " + num(W) + "; ++e) {");
-          o.ind++;
-          emit_nodes(o, x, var, true, c);
-          std::string v = node_name(x, var, x.result, c);
+          std::string A = "acc" + num(x.stmt);
+          Sink sk;
           if (red) {
-            if (x.redop == FOP_RED_MAX) o.l("acc" + num(x.stmt) + " = fop::op_max(acc" + num(x.stmt) + ", " + v + ");");
-            else o.l("acc" + num(x.stmt) + " = __fadd_rn(acc" + num(x.stmt) + ", " + v + ");");
+            bool mx = x.redop == FOP_RED_MAX;
+            sk.scalar = [&, A, mx](const std::string& v) {
+              o.l(A + " = " + (mx ? "fop::op_max(" : "__fadd_rn(") + A + ", " + v + ");");
+            };
+            if (!mx) {
+              sk.pair = [&, A](const std::string& v, const std::string&) { o.l(A + "p = fop::add2(" + A + "p, " + v + ");"); };
+              sk.pair_fma = [&, A](const std::string& a, const std::string& b, const std::string&) {
+                o.l(A + "p = fop::fma2(" + a + ", " + b + ", " + A + "p);");
+              };
+            }
           } else {
-            o.l("R[e] = " + v + ";");
-            if (x.fwd && regmode)
-              o.l("F" + num(x.stmt) + "[" + num(base_idx) + " + e] = fop::round_to<" + dtn(x.out_dtype) + ">(" + v + ");");
+            std::string F = "F" + num(x.stmt) + "[" + num(base_idx) + " + ";
+            bool keep = x.fwd && regmode;
+            std::string dto = dtn(x.out_dtype);
+            sk.scalar = [&, F, keep, dto](const std::string& v) {
+              o.l("R[e] = " + v + ";");
+              if (keep) o.l(F + "e] = fop::round_to<" + dto + ">(" + v + ");");
+            };
+            sk.pair = [&, F, keep, dto](const std::string& v, const std::string& p) {
+              o.l("fop::upk(" + v + ", R[2 * " + p + "], R[2 * " + p + " + 1]);");
+              if (keep) {
+                o.l(F + "2 * " + p + "] = fop::round_to<" + dto + ">(R[2 * " + p + "]);");
+                o.l(F + "2 * " + p + " + 1] = fop::round_to<" + dto + ">(R[2 * " + p + " + 1]);");
+              }
+            };
           }
-          o.ind--;
-          o.l("}");
+          emit_elems(o, x, var, c, W, sk);
           if (!red && x.store) {
             std::string off = affine(x.write, its2);
             int64_t cw = C(x.write, 0);
@@ -763,6 +870,8 @@ struct Gen {
       }
       if (red) {
         std::string a = "acc" + num(x.stmt);
+        if (x.redop == FOP_RED_SUM)
+          o.l(a + " = __fadd_rn(" + a + ", __fadd_rn(fop::lo(" + a + "p), fop::hi(" + a + "p)));");
         o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::warp_max(" : "fop::warp_sum(") + a + ");");
         std::string res = fin_expr(o, x, a, "");
         if (x.fwd) o.l("const float S" + num(x.stmt) + " = fop::round_to<" + dtn(x.out_dtype) + ">(" + res + ");");
@@ -809,9 +918,15 @@ struct Gen {
     o.l("const idx_t r0 = chunk * " + num(RPC) + "u;");
     o.l("const idx_t r1 = (r0 + " + num(RPC) + "u < " + num(ROWS) + "u) ? r0 + " + num(RPC) + "u : " + num(ROWS) +
         "u;");
+    const bool packed = !isMax && W % 2 == 0 && g_packed;
     o.l("float acc[" + num(W) + "];");
     o.l("#pragma unroll");
     o.l("for (int e = 0; e < " + num(W) + "; ++e) acc[e] = " + init + ";");
+    if (packed) {
+      o.l("u64 accp[" + num(W / 2) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) accp[p] = fop::pk1(0.f);");
+    }
     o.l("#pragma unroll 1");
     o.l("for (idx_t r = r0 + rl; r < r1; r += " + num((int64_t)L.gr * U) + "u) {");
     o.ind++;
@@ -848,25 +963,34 @@ struct Gen {
       DagCtx c;
       c.tag = t;
       c.load_varies = [&](int k) { return C(L.loads[k], 0) != 0; };
-      c.load = [&, t](int k) { return C(L.loads[k], 0) != 0 ? "L" + num(k) + t + "[e]" : "L" + num(k) + t; };
-      c.fwd = [&](int) { return std::string("0.f"); };
+      c.load = [&, t](int k, const std::string& e) {
+        return C(L.loads[k], 0) != 0 ? "L" + num(k) + t + "[" + e + "]" : "L" + num(k) + t;
+      };
+      c.fwd = [&](int, const std::string&) { return std::string("0.f"); };
       c.scalar = [&](int) { return std::string("0.f"); };
       auto var = varies(x, c);
       o.l("if (ok" + t + ") {");
       o.ind++;
       emit_nodes(o, x, var, false, c);
-      o.l("#pragma unroll");
-      o.l("for (int e = 0; e < " + num(W) + "; ++e) {");
-      o.ind++;
-      emit_nodes(o, x, var, true, c);
-      o.l("acc[e] = " + comb("acc[e]", node_name(x, var, x.result, c)) + ";");
-      o.ind--;
-      o.l("}");
+      Sink sk;
+      sk.scalar = [&](const std::string& v) { o.l("acc[e] = " + comb("acc[e]", v) + ";"); };
+      if (packed) {
+        sk.pair = [&](const std::string& v, const std::string& p) { o.l("accp[" + p + "] = fop::add2(accp[" + p + "], " + v + ");"); };
+        sk.pair_fma = [&](const std::string& a, const std::string& b, const std::string& p) {
+          o.l("accp[" + p + "] = fop::fma2(" + a + ", " + b + ", accp[" + p + "]);");
+        };
+      }
+      emit_elems(o, x, var, c, W, sk);
       o.ind--;
       o.l("}");
     }
     o.ind--;
     o.l("}");
+    if (packed) {  // pairs of partial sums back to one accumulator per column
+      o.l("#pragma unroll");
+      o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) { float a0_, a1_; fop::upk(accp[p], a0_, a1_); "
+          "acc[2 * p] = __fadd_rn(acc[2 * p], a0_); acc[2 * p + 1] = __fadd_rn(acc[2 * p + 1], a1_); }");
+    }
     // block tree over the row lanes (fixed order => deterministic)
     auto tree = [&]() {
       o.l("#pragma unroll");
@@ -958,6 +1082,10 @@ const char* class_name(int c) {
 }  // namespace
 
 std::string generate(const Plan& p, Launch& L, int launch_index) {
+  {
+    const char* e = std::getenv("FOP_PACKED");   // 0: scalar fp32 DAG evaluation (ablation)
+    g_packed = !(e && *e == '0');
+  }
   Gen g(p, L);
   // 32-bit index arithmetic when every offset and work index fits
   int64_t maxv = L.work + L.grid * L.block * 8;

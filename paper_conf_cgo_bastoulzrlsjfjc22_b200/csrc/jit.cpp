@@ -94,8 +94,11 @@ void jit_compile(Launch& L) {
   std::string fname = L.name + ".cu";
   if (n.create(&prog, L.src.c_str(), fname.c_str(), 1, hdr_src, hdr_name) != 0)
     fail(FOP_E_JIT, "nvrtcCreateProgram failed");
-  const char* opts[] = {"-arch=sm_100a", "-std=c++17", "-lineinfo"};
-  nvrtcResult r = n.compile(prog, 3, opts);
+  // -fmad=false: ptxas may not contract a multiply and an add into one FMA,
+  // even for the packed mul/add.rn.f32x2 forms (it does without this flag);
+  // every FMA the kernels use is an explicit fma instruction.
+  const char* opts[] = {"-arch=sm_100a", "-std=c++17", "-lineinfo", "-fmad=false"};
+  nvrtcResult r = n.compile(prog, 4, opts);
   if (r != 0) {
     size_t ls = 0;
     n.logsize(prog, &ls);
