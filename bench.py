@@ -37,6 +37,9 @@ import workloads as W  # noqa: E402
 
 OPS = [("cfg2", W.cfg2, "ew"), ("cfg3", W.cfg3, "transpose"), ("cfg4a", W.cfg4a, "row_reduce"),
        ("cfg4b", W.cfg4b, "col_reduce")]
+# global operator at `world` GPUs (batch loop scaled by world) and the loop it is sharded along
+GLOBAL = {"cfg2": (lambda w: W.cfg2(N=128 * w), "n"), "cfg3": (lambda w: W.cfg3(N=256 * w), "n"),
+          "cfg4a": (lambda w: W.cfg4a(B=64 * w), "b"), "cfg4b": (lambda w: W.cfg4b(R=65536 * w), "r")}
 FALLBACK_HBM = 6650.0
 
 
@@ -178,9 +181,11 @@ def run_fop(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
 
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc, allreduce_partials
     ops = []
     for name, mk, cls in OPS:
-        d = mk()
+        gmk, loop = GLOBAL[name]
+        d, shard_info = shard_desc(gmk(world), loop, rank, world)   # == mk() per rank
         op = FusedOp(d, **({"max_vec_bytes": args.vec_bytes} if args.vec_bytes else {}),
                      **({"coalesce_order": args.order} if args.order else {}))
         x = W.make_inputs(d, seed_offset=rank * 1000)
@@ -196,15 +201,15 @@ def run_fop(args):
                   if t["role"] in ("in", "inout"))
         d2h = sum(host[n].numel() * host[n].element_size() for n, t in d["tensors"].items()
                   if t["role"] in ("out", "inout"))
-        ops.append({"name": name, "cls": cls, "desc": d, "op": op, "dev": tens, "host": host,
+        ops.append({"name": name, "cls": cls, "desc": d, "op": op, "dev": tens, "host": host, "shard": shard_info,
                     "bytes": W.algorithmic_bytes(d), "h2d": h2d, "d2h": d2h,
                     "launches": len(op.info()["launches"]), "kernel": op.info()["launches"][0]})
         del x, outs
     stream = torch.cuda.current_stream(dev)
 
-    def allreduce(o):
-        if world > 1 and o["name"] == "cfg4b":
-            dist.all_reduce(o["dev"]["out"], op=dist.ReduceOp.SUM)
+    def allreduce(o):   # only cfg4b has partials: its rows are the sharded (reduced) axis
+        if world > 1:
+            allreduce_partials(o["dev"], o["shard"])
 
     def step(events=None):
         for i, o in enumerate(ops):
