@@ -277,6 +277,7 @@ struct Gen {
   void header(const std::string& name, int /*unused*/) {
     const int minblocks = std::max(1, L.minblocks);
     o.l("// generated by libfop (planner + codegen); skeleton: " + name);
+    if (const char* g = std::getenv("FOP_GELU_NR"); g && *g == '1') o.l("#define FOP_GELU_NR 1");
     o.l("#include \"fop_device.cuh\"");
     o.l("typedef " + idx + " idx_t;");
     o.l("extern \"C\" __global__ void __launch_bounds__(" + num(L.block) + ", " + num(minblocks) + ") " +
@@ -646,7 +647,7 @@ struct Gen {
       for (size_t q = L.nsplit; q < L.kl.size(); q++) row_inv &= C(a, (int)q) == 0;
       int64_t cv = C(a, 0);
       int es_k = es(a.tensor);
-      if (row_inv && regmode && (cv == 0 || cv == 1) && !written_here(a.tensor)) mode[k] = 'H';
+      if (L.row_hoist && row_inv && regmode && (cv == 0 || cv == 1) && !written_here(a.tensor)) mode[k] = 'H';
       else if (L.row_prefetch && used0[k] && cv == 1 && W * es_k >= 4 && L.load_cb[k] >= 4 &&
                NP * W * es_k / 4 <= 32 && !written_here(a.tensor))
         mode[k] = 'P';
@@ -845,10 +846,9 @@ struct Gen {
             };
             sk.pair = [&, F, keep, dto](const std::string& v, const std::string& p) {
               o.l("fop::upk(" + v + ", R[2 * " + p + "], R[2 * " + p + " + 1]);");
-              if (keep) {
-                o.l(F + "2 * " + p + "] = fop::round_to<" + dto + ">(R[2 * " + p + "]);");
-                o.l(F + "2 * " + p + " + 1] = fop::round_to<" + dto + ">(R[2 * " + p + " + 1]);");
-              }
+              if (keep)
+                o.l("fop::round2<" + dto + ">(R[2 * " + p + "], R[2 * " + p + " + 1], " + F + "2 * " + p + "], " + F +
+                    "2 * " + p + " + 1]);");
             };
           }
           emit_elems(o, x, var, c, W, sk);
@@ -927,9 +927,53 @@ struct Gen {
       o.l("#pragma unroll");
       o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) accp[p] = fop::pk1(0.f);");
     }
+    // Software pipeline (default): the U row loads of batch i+1 are issued as
+    // raw words before batch i is converted and accumulated, so HBM requests
+    // stay in flight across the accumulation instead of draining each batch.
+    bool pipe = L.col_pipe;
+    std::vector<int> wpv(L.loads.size(), 0);
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      int64_t cv = C(L.loads[k], 0);
+      int eb = es(L.loads[k].tensor);
+      if (cv == 1 && W * eb >= 4 && L.load_cb[k] >= 4 && !written_here(L.loads[k].tensor)) wpv[k] = W * eb / 4;
+      else if (cv != 0) pipe = false;
+    }
+    const int64_t BSTEP = (int64_t)L.gr * U;
+    auto batch_loads = [&](const std::string& rbase, const std::string& buf, const std::string& tg) {
+      for (int u = 0; u < U; u++) {
+        std::string t = tg + num(u);
+        o.l("{");
+        o.ind++;
+        o.l("const idx_t rr = " + rbase + " + " + num((int64_t)L.gr * u) + "u;");
+        o.l("idx_t q = rr;");
+        std::vector<std::pair<int, std::string>> bits = cits;
+        decompose("q", L.nsplit, (int)L.kl.size(), t, bits);
+        for (size_t k = 0; k < L.loads.size(); k++) {
+          if (!wpv[k]) continue;
+          const Affine& a = L.loads[k];
+          o.l("if (okc && rr < r1) fop::vload_words<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + num(W) + ", " +
+              num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + buf + num(k) + "_" + num(u) + ", " +
+              ptr(a.tensor, affine(a, bits)) + ");");
+        }
+        o.ind--;
+        o.l("}");
+      }
+    };
+    if (pipe) {
+      for (int u = 0; u < U; u++)
+        for (size_t k = 0; k < L.loads.size(); k++)
+          if (wpv[k]) o.l("u32 A" + num(k) + "_" + num(u) + "[" + num(wpv[k]) + "];");
+      batch_loads("(r0 + rl)", "A", "_a");
+    }
     o.l("#pragma unroll 1");
-    o.l("for (idx_t r = r0 + rl; r < r1; r += " + num((int64_t)L.gr * U) + "u) {");
+    o.l("for (idx_t r = r0 + rl; r < r1; r += " + num(BSTEP) + "u) {");
     o.ind++;
+    if (pipe) {
+      for (int u = 0; u < U; u++)
+        for (size_t k = 0; k < L.loads.size(); k++)
+          if (wpv[k]) o.l("u32 B" + num(k) + "_" + num(u) + "[" + num(wpv[k]) + "];");
+      batch_loads("(r + " + num(BSTEP) + "u)", "B", "_b");
+    }
     std::vector<std::vector<std::pair<int, std::string>>> its(U);
     for (int u = 0; u < U; u++) {
       std::string t = "_" + num(u);
@@ -939,6 +983,12 @@ struct Gen {
       its[u] = cits;
       decompose("q" + t, L.nsplit, (int)L.kl.size(), t, its[u]);
       for (size_t k = 0; k < L.loads.size(); k++) {
+        if (pipe && wpv[k]) {
+          o.l("float L" + num(k) + t + "[" + num(W) + "];");
+          o.l("fop::cvt_words<" + std::string(dtn(d.t[L.loads[k].tensor].dtype)) + ", " + num(W) + ">(L" + num(k) + t +
+              ", A" + num(k) + t + ");");
+          continue;
+        }
         const Affine& a = L.loads[k];
         int64_t cv = C(a, 0);
         std::string off = affine(a, its[u]);
@@ -983,6 +1033,13 @@ struct Gen {
       emit_elems(o, x, var, c, W, sk);
       o.ind--;
       o.l("}");
+    }
+    if (pipe) {  // batch i+1 becomes the current batch
+      for (int u = 0; u < U; u++)
+        for (size_t k = 0; k < L.loads.size(); k++)
+          if (wpv[k])
+            o.l("#pragma unroll\nfor (int i = 0; i < " + num(wpv[k]) + "; ++i) A" + num(k) + "_" + num(u) + "[i] = B" +
+                num(k) + "_" + num(u) + "[i];");
     }
     o.ind--;
     o.l("}");

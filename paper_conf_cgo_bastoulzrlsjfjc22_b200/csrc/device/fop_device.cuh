@@ -405,12 +405,48 @@ __device__ __forceinline__ float op_gelu_tanh(float v) {
   float e = ex2_approx(t * v);
   return v * rcp_approx(1.0f + e);
 }
+#ifndef FOP_GELU_NR
+#define FOP_GELU_NR 0
+#endif
 __device__ __forceinline__ u64 op_gelu_tanh2(u64 v) {
   u64 t = fma2(mul2(v, v), pk1(FOP_GELU_C1), pk1(FOP_GELU_C2));
   u64 a = mul2(t, v);
+#if FOP_GELU_NR
+  // 1/(1+e) on the FMA pipe: MUFU.EX2 only (the XU pipe is the cfg4a limiter).
+  // Clamp the exponent so 1+e stays below 2^127 (the magic-constant seed needs
+  // a finite input; 1/(1+2^126) vs 0 is below fp16/bf16 resolution), seed by
+  // the integer reciprocal trick, three Newton steps y <- y (2 - d y).
+  u64 e = pk(ex2_approx(fminf(lo(a), 126.f)), ex2_approx(fminf(hi(a), 126.f)));
+  u64 dn = add2(e, pk1(1.0f));
+  u64 y = 0x7EF311C37EF311C3ull - dn;
+  u64 nd = dn ^ 0x8000000080000000ull;
+  y = mul2(y, fma2(nd, y, pk1(2.0f)));
+  y = mul2(y, fma2(nd, y, pk1(2.0f)));
+  y = mul2(y, fma2(nd, y, pk1(2.0f)));
+  return mul2(v, y);
+#else
   u64 e = pk(ex2_approx(lo(a)), ex2_approx(hi(a)));
   u64 dn = add2(e, pk1(1.0f));
   return mul2(v, pk(rcp_approx(lo(dn)), rcp_approx(hi(dn))));
+#endif
+}
+
+// value rounded to DT and back, for a pair; the packed conversion is the same
+// instruction the vector store issues, so the compiler computes it once
+template <int DT>
+__device__ __forceinline__ void round2(float a, float b, float& ra, float& rb) {
+  if constexpr (DT == F16) {
+    u32 w = f2h2(a, b);
+    ra = h2f((u16)(w & 0xffffu));
+    rb = h2f((u16)(w >> 16));
+  } else if constexpr (DT == BF16) {
+    u32 w = f2b2(a, b);
+    ra = __uint_as_float(w << 16);
+    rb = __uint_as_float(w & 0xffff0000u);
+  } else {
+    ra = a;
+    rb = b;
+  }
 }
 __device__ __forceinline__ float op_gelu_erf(float v) { return 0.5f * v * erfcf(-0.70710678118654752f * v); }
 __device__ __forceinline__ float op_sigmoid(float v) { return __frcp_rn(1.0f + expf(-v)); }

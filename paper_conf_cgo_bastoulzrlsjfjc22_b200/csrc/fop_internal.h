@@ -108,6 +108,8 @@ struct Launch {
   int unroll = 1;
   int minblocks = 1;              // __launch_bounds__ min blocks/SM; grid-stride grids = SMs x minblocks
   int row_prefetch = 0;           // ROW: prefetch the next row's streaming loads
+  int col_pipe = 0;               // COL: software-pipelined row batches
+  int row_hoist = 1;              // ROW: keep row-invariant loads in registers across rows
   int gv = 1, gr = 1;             // lanes along d_v / along the other tiled dim
   int64_t nchunks = 1;            // COL: row chunks
   int64_t work = 0;               // total work items (threads' units)

@@ -283,6 +283,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.work = rows;  // one warp per row
     L.minblocks = knob("FOP_ROW_MINB", 3);
     L.row_prefetch = knob("FOP_ROW_PREFETCH", 1);
+    L.row_hoist = knob("FOP_ROW_HOIST", 1);
     int64_t need = (rows + L.block / 32 - 1) / (L.block / 32);
     L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
     L.unroll = 1;
@@ -292,7 +293,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     for (const auto& a : L.loads)
       if (coef(L, a, 0) == 1) big = &a;
     int es_ld = big ? esize(d.t[big->tensor].dtype) : 4;
-    int gv = (int)std::min<int64_t>(32, std::max<int64_t>(1, 128 / (W * es_ld)));
+    int gv = (int)std::min<int64_t>(32, std::max<int64_t>(1, knob("FOP_COL_SLAB_BYTES", 128) / (W * es_ld)));
     gv = std::min(gv, pow2_floor(nvd));
     L.gv = gv;
     L.gr = L.block / gv;
@@ -300,8 +301,9 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     for (int k = 1; k < L.nsplit; k++) slabs *= L.kl[k].extent;
     int64_t rows = 1;
     for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
+    L.col_pipe = knob("FOP_COL_PIPE", 0);   // measured: no gain over U=8 batches (sweep_r01_4)
     L.minblocks = knob("FOP_COL_MINB", 2);
-    L.unroll = knob("FOP_COL_U", 8);
+    L.unroll = knob("FOP_COL_U", L.col_pipe ? 4 : 8);
     int64_t target = (int64_t)sms * L.minblocks;   // one resident wave
     int64_t nch = std::max<int64_t>(1, target / std::max<int64_t>(1, slabs));
     nch = std::min<int64_t>(nch, std::max<int64_t>(1, (rows + L.gr - 1) / L.gr));

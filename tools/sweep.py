@@ -3,10 +3,11 @@
     python tools/sweep.py cfg2 "FOP_EW_U=2,FOP_EW_MINB=4" "FOP_EW_U=4,FOP_EW_MINB=3" ...
     python tools/sweep.py cfg3 "opt:max_vec_bytes=32" "opt:coalesce_order=memory"
 
-Each variant: plan under the given env knobs / plan options, 5 warm-up runs,
-then 30 timed runs (CUDA events around the launch on the current stream),
-L2 flushed (256 MiB memset) before every timed run.  Prints median/min GB/s
-(algorithmic bytes) per variant, one JSON line each.
+Timing: R copies of every tensor (R chosen so the copies exceed 3x the 126 MB
+L2), 5 warm-up launches, then 5 batches of 40 launches rotating over the
+copies, each batch bracketed by CUDA events on the current stream (event
+resolution is ~2 us, too coarse for one 20-40 us launch).  Per-launch time =
+batch time / 40; reported: median and best batch, GB/s of algorithmic bytes.
 """
 import json
 import os
@@ -22,6 +23,8 @@ import workloads as W  # noqa: E402
 from bench import to_device  # noqa: E402
 from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp  # noqa: E402
 
+L2 = 126 << 20
+
 
 def main():
     name = sys.argv[1]
@@ -29,10 +32,12 @@ def main():
     d = W.CONFIGS[name]()
     x = W.make_inputs(d)
     o = W.alloc_outputs(d, fill_nan=False)
-    tens = {n: to_device(x[n] if t["role"] in ("in", "inout") else o[n], t["dtype"], "cuda")
-            for n, t in d["tensors"].items() if t["role"] != "temp"}
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     nbytes = W.algorithmic_bytes(d)
+    copies = max(1, min(16, -(-3 * L2 // nbytes)))
+    sets = []
+    for _ in range(copies):
+        sets.append({n: to_device(x[n] if t["role"] in ("in", "inout") else o[n], t["dtype"], "cuda")
+                     for n, t in d["tensors"].items() if t["role"] != "temp"})
     for v in variants:
         env, opts = {}, {}
         for kv in filter(None, v.split(",")):
@@ -54,22 +59,25 @@ def main():
                     os.environ.pop(k, None)
                 else:
                     os.environ[k] = val
+        for i in range(5):
+            op.run(sets[i % copies])
+        torch.cuda.synchronize()
+        per = []
+        n = 40
         for _ in range(5):
-            op.run(tens)
-        times = []
-        for _ in range(30):
-            flush.zero_()
             s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             s.record()
-            op.run(tens)
+            for i in range(n):
+                op.run(sets[i % copies])
             e.record()
             torch.cuda.synchronize()
-            times.append(s.elapsed_time(e))
-        med = statistics.median(times)
+            per.append(s.elapsed_time(e) / n)
+        med = statistics.median(per)
         li = op.info()["launches"][0]
-        print(json.dumps({"op": name, "variant": v, "us_median": med * 1e3, "us_min": min(times) * 1e3,
-                          "GBs_median": nbytes / med / 1e6, "GBs_best": nbytes / min(times) / 1e6,
-                          "grid": li["grid"], "class": li["class"], "width": li["width"]}), flush=True)
+        print(json.dumps({"op": name, "variant": v, "us_median": med * 1e3, "us_min": min(per) * 1e3,
+                          "GBs_median": nbytes / med / 1e6, "GBs_best": nbytes / min(per) / 1e6,
+                          "grid": li["grid"], "class": li["class"], "width": li["width"], "copies": copies}),
+              flush=True)
 
 
 if __name__ == "__main__":
