@@ -614,6 +614,157 @@ struct Gen {
     footer();
   }
 
+  // ------------------------------------------------------------ TRANSPOSE via TMA
+  // 64x64 tiles of 16-bit data.  Per CTA (128 threads = two 64-thread tile
+  // groups): a pipeline of S smem stages, each holding two 8 KB input tiles
+  // loaded by cp.async.bulk.tensor (128B swizzle) and completed on an mbarrier;
+  // each thread transposes one 8x8 sub-tile through registers (8 LDS.128 ->
+  // compute -> 8 STS.128 into a swizzled output tile); one thread stores both
+  // output tiles with cp.async.bulk.tensor and refills the stage.  Sub-tiles
+  // are assigned along diagonals (ca = t, cb = t + d) so every quarter-warp
+  // LDS.128/STS.128 touches 8 distinct 16 B bank groups of the swizzle.
+  void gen_transpose_tma() {
+    const XStmt& x = L.stmts[0];
+    const int S = L.tma_stages, R = L.tma_rank;
+    const int64_t NP = L.work;   // tile pairs
+    bool raw = x.move;
+    const int ktr = L.trans_load;
+    std::string dti = dtn(d.t[L.loads[ktr].tensor].dtype), dto = dtn(x.out_dtype);
+    o.l("// generated by libfop (planner + codegen); skeleton: TRANSPOSE via TMA (64x64 tiles, " + num(S) +
+        "-stage mbarrier pipeline)");
+    if (const char* g = std::getenv("FOP_GELU_NR"); g && *g == '1') o.l("#define FOP_GELU_NR 1");
+    o.l("#include \"fop_device.cuh\"");
+    o.l("typedef " + idx + " idx_t;");
+    const int NW = L.block / 32;
+    o.l("extern \"C\" __global__ void __launch_bounds__(" + num(L.block) + ", " + num(std::max(1, L.minblocks)) + ") " +
+        L.name + "(const FopArgs args, const __grid_constant__ fop::TmaDesc tin, const __grid_constant__ fop::TmaDesc tout) {");
+    o.ind++;
+    o.l("extern __shared__ __align__(1024) unsigned char smem_raw[];");
+    o.l("unsigned char* smem = (unsigned char*)(((unsigned long long)smem_raw + 1023ull) & ~1023ull);");
+    o.l("const unsigned lane = threadIdx.x & 31u, wid = threadIdx.x >> 5;");
+    o.l("// per warp: S input stages (8 KB tiles) + 2 output tiles, own mbarriers: warps never wait for each other");
+    o.l("unsigned char* sin = smem + wid * " + num((S + 2) * 8192) + "u;");
+    o.l("unsigned char* sout = sin + " + num(S * 8192) + ";");
+    o.l("u64* full = (u64*)(smem + " + num(NW * (S + 2) * 8192) + ") + wid * " + num(S) + "u;");
+    o.l("const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;");
+    for (int t = 0; t < d.ntensors; t++) {
+      bool used = false;
+      for (size_t k = 0; k < L.loads.size(); k++) used |= (int)k != ktr && L.loads[k].tensor == t;
+      if (used) o.l("const char* __restrict__ T" + num(t) + " = args.p[" + num(t) + "];");
+    }
+    // constant (scalar) loads
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      if ((int)k == ktr) continue;
+      const Affine& a = L.loads[k];
+      o.l("const float L" + num(k) + " = fop::sload<" + std::string(dtn(d.t[a.tensor].dtype)) + ", fop::LD_CACHED>(" +
+          ptr(a.tensor, num(a.base)) + ");");
+    }
+    // tile -> coordinates (elements): tv fastest, then tr, then outer kloops
+    o.l("auto coords = [&](idx_t tile, int* ci, int* co) {");
+    o.l("  const int tv = (int)(tile % " + num(L.tma_ntv) + "u); tile /= " + num(L.tma_ntv) + "u;");
+    o.l("  const int tr = (int)(tile % " + num(L.tma_ntr) + "u); tile /= " + num(L.tma_ntr) + "u;");
+    o.l("  ci[0] = tr * 64; ci[1] = tv * 64; co[0] = tv * 64; co[1] = tr * 64;");
+    for (int q = 2; q < R; q++) {
+      if (q == R - 1) o.l("  ci[" + num(q) + "] = co[" + num(q) + "] = (int)tile;");
+      else o.l("  ci[" + num(q) + "] = co[" + num(q) + "] = (int)(tile % " + num(L.kl[q].extent) + "u); tile /= " +
+               num(L.kl[q].extent) + "u;");
+    }
+    o.l("};");
+    const int64_t T = L.tma_tiles;
+    o.l("const idx_t first = (idx_t)blockIdx.x * " + num(NW) + "u + wid, tstride = (idx_t)gridDim.x * " + num(NW) + "u;");
+    o.l("auto issue = [&](idx_t t, int s) {   // tile t into stage s");
+    o.l("  int ci[5], co[5];");
+    o.l("  coords(t, ci, co);");
+    o.l("  fop::mbar_expect_tx(&full[s], 8192u);");
+    o.l("  fop::tma_load(sin + s * 8192, &tin, &full[s], " + num(R) + ", ci);");
+    o.l("};");
+    o.l("if (lane == 0) {");
+    o.l("  for (int s = 0; s < " + num(S) + "; ++s) fop::mbar_init(&full[s], 1);");
+    o.l("  fop::fence_mbar_init();");
+    o.l("  for (int s = 0; s < " + num(S) + "; ++s) {");
+    o.l("    const idx_t t = first + (idx_t)s * tstride;");
+    o.l("    if (t < " + num(T) + "u) issue(t, s);");
+    o.l("  }");
+    o.l("}");
+    o.l("__syncwarp();");
+    o.l("#pragma unroll 1");
+    o.l("for (unsigned k = 0;; ++k) {");
+    o.ind++;
+    o.l("const idx_t tile = first + (idx_t)k * tstride;");
+    o.l("if (tile >= " + num(T) + "u) break;");
+    o.l("const int s = (int)(k % " + num(S) + "u);");
+    o.l("const unsigned ph = (k / " + num(S) + "u) & 1u;");
+    o.l("const int ob = (int)(k & 1u);");
+    o.l("if (lane == 0) fop::bulk_wait_read<1>();   // this warp's store of step k-2 has left buffer ob");
+    o.l("__syncwarp();");
+    o.l("fop::mbar_wait(&full[s], ph);");
+    o.l("const u32 ib = fop::smem_u32(sin + s * 8192), obase = fop::smem_u32(sout + ob * 8192);");
+    o.l("#pragma unroll");
+    o.l("for (int pass = 0; pass < 2; ++pass) {   // 64 sub-tiles, 2 per lane; quarter-warp = one diagonal");
+    o.ind++;
+    o.l("const unsigned tau = lane + 32u * pass;");
+    o.l("const unsigned ca = tau & 7u, cb = ((tau & 7u) + (tau >> 3)) & 7u;");
+    o.l("u32 w[8][4];");
+    o.l("#pragma unroll");
+    o.l("for (int i = 0; i < 8; ++i) fop::lds128(w[i], ib + (8u * ca + i) * 128u + ((cb ^ (unsigned)i) << 4));");
+    if (raw) {
+      // out row j (R = 8cb + j), chunk ca holds in[i][j] for i = 0..7
+      o.l("#pragma unroll");
+      o.l("for (int j = 0; j < 8; ++j) {");
+      o.l("  u32 h[8];");
+      o.l("  #pragma unroll");
+      o.l("  for (int i = 0; i < 8; ++i) h[i] = (w[i][j >> 1] >> ((j & 1) * 16)) & 0xffffu;");
+      o.l("  fop::sts128(obase + (8u * cb + j) * 128u + ((ca ^ (unsigned)j) << 4), h[0] | (h[1] << 16), h[2] | (h[3] << 16),"
+          " h[4] | (h[5] << 16), h[6] | (h[7] << 16));");
+      o.l("}");
+    } else {
+      o.l("float X[8][8];   // X[i][j]: V = 8ca+i, R = 8cb+j");
+      o.l("#pragma unroll");
+      o.l("for (int i = 0; i < 8; ++i) fop::cvt_words<" + dti + ", 8>(X[i], w[i]);");
+      DagCtx c;
+      c.tag = "";
+      c.ev = "i";
+      c.load_varies = [&](int k) { return k == ktr; };
+      c.load = [&](int k, const std::string& e) { return k == ktr ? "X[" + e + "][j]" : "L" + num(k); };
+      c.fwd = [&](int, const std::string&) { return std::string("0.f"); };
+      c.scalar = [&](int) { return std::string("0.f"); };
+      auto var = varies(x, c);
+      emit_nodes(o, x, var, false, c);
+      o.l("#pragma unroll");
+      o.l("for (int j = 0; j < 8; ++j) {");
+      o.ind++;
+      o.l("float O[8];");
+      Sink sk;
+      sk.scalar = [&](const std::string& v) { o.l("O[i] = " + v + ";"); };
+      sk.pair = [&](const std::string& v, const std::string& p) {
+        o.l("fop::upk(" + v + ", O[2 * " + p + "], O[2 * " + p + " + 1]);");
+      };
+      emit_elems(o, x, var, c, 8, sk);
+      std::string pack = x.out_dtype == FOP_BF16 ? "fop::f2b2" : "fop::f2h2";
+      o.l("fop::sts128(obase + (8u * cb + j) * 128u + ((ca ^ (unsigned)j) << 4), " + pack + "(O[0], O[1]), " + pack +
+          "(O[2], O[3]), " + pack + "(O[4], O[5]), " + pack + "(O[6], O[7]));");
+      o.ind--;
+      o.l("}");
+    }
+    o.ind--;
+    o.l("}");
+    o.l("fop::fence_async_smem();   // generic-proxy smem writes -> visible to the TMA store");
+    o.l("__syncwarp();");
+    o.l("if (lane == 0) {");
+    o.l("  int ci[5], co[5];");
+    o.l("  coords(tile, ci, co);");
+    o.l("  fop::tma_store(&tout, sout + ob * 8192, " + num(R) + ", co);");
+    o.l("  fop::bulk_commit();");
+    o.l("  const idx_t tn = tile + (idx_t)" + num(S) + "u * tstride;");
+    o.l("  if (tn < " + num(T) + "u) issue(tn, s);   // every lane has finished reading stage s");
+    o.l("}");
+    o.ind--;
+    o.l("}");
+    o.l("if (lane == 0) fop::bulk_wait<0>();");
+    footer();
+    (void)NP;
+  }
+
   // ------------------------------------------------------------ ROW_REDUCE
   void gen_row() {
     const int W = L.width;
@@ -1152,10 +1303,13 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
     maxv = std::max(maxv, span + 64);
   }
   g.idx = maxv < (int64_t(1) << 31) ? "unsigned" : "unsigned long long";
-  L.name = std::string("fop_") + class_name(L.kclass) + "_k" + std::to_string(launch_index) +
+  L.name = std::string("fop_") + class_name(L.kclass) + (L.tma ? "_tma" : "") + "_k" + std::to_string(launch_index) +
            (L.scalar_variant ? "_narrow" : "");
   switch (L.kclass) {
-    case FOP_CLASS_TRANSPOSE: g.gen_transpose(); break;
+    case FOP_CLASS_TRANSPOSE:
+      if (L.tma) g.gen_transpose_tma();
+      else g.gen_transpose();
+      break;
     case FOP_CLASS_ROW_REDUCE: g.gen_row(); break;
     case FOP_CLASS_COL_REDUCE: g.gen_col(); break;
     default: g.gen_ew();

@@ -110,6 +110,19 @@ struct Launch {
   int row_prefetch = 0;           // ROW: prefetch the next row's streaming loads
   int col_pipe = 0;               // COL: software-pipelined row batches
   int row_hoist = 1;              // ROW: keep row-invariant loads in registers across rows
+  // TRANSPOSE through TMA (16-bit data): 64x64 tiles, tensor maps encoded per run
+  int tma = 0;
+  int tma_rank = 0, tma_stages = 4;
+  int tma_in_tensor = -1, tma_out_tensor = -1;
+  int64_t tma_in_base = 0, tma_out_base = 0;     // access base offsets (elements)
+  uint64_t tma_in_dim[5] = {0}, tma_in_stride[5] = {0};    // strides in bytes of dims 1..rank-1
+  uint64_t tma_out_dim[5] = {0}, tma_out_stride[5] = {0};
+  int64_t tma_tiles = 0, tma_ntv = 0, tma_ntr = 0;
+  // per-run tensor maps (runtime; cached for the last pointer pair, guarded by Plan::mu)
+  struct alignas(64) TmaMap { uint64_t w[16]; };
+  TmaMap tma_map_in, tma_map_out;
+  const void* tma_last_in = nullptr;
+  const void* tma_last_out = nullptr;
   int gv = 1, gr = 1;             // lanes along d_v / along the other tiled dim
   int64_t nchunks = 1;            // COL: row chunks
   int64_t work = 0;               // total work items (threads' units)

@@ -8,6 +8,7 @@
 #include <dlfcn.h>
 
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -41,7 +42,12 @@ struct Cuda {
   CUresult (*h2d)(CUdeviceptr, const void*, size_t, CUstream);
   CUresult (*d2h)(void*, CUdeviceptr, size_t, CUstream);
   CUresult (*errstr)(CUresult, const char**);
+  CUresult (*func_attr)(CUfunction, int, int);
+  CUresult (*tmap_encode)(void*, int, unsigned, void*, const uint64_t*, const uint64_t*, const unsigned*,
+                          const unsigned*, int, int, int, int);
 };
+enum { CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES = 8 };
+enum { TMAP_UINT16 = 1, TMAP_INTERLEAVE_NONE = 0, TMAP_SWIZZLE_128B = 3, TMAP_L2_PROMO_256B = 3, TMAP_OOB_NONE = 0 };
 
 Cuda& cuda() {
   static Cuda c;
@@ -69,6 +75,8 @@ Cuda& cuda() {
     SYM(h2d, "cuMemcpyHtoDAsync_v2");
     SYM(d2h, "cuMemcpyDtoHAsync_v2");
     SYM(errstr, "cuGetErrorString");
+    SYM(func_attr, "cuFuncSetAttribute");
+    SYM(tmap_encode, "cuTensorMapEncodeTiled");
 #undef SYM
     if (c.init(0) != 0) {
       c.why = "cuInit failed";
@@ -119,6 +127,8 @@ Plan::Loaded& loaded_for(Plan& p, CUcontext ctx) {
     CUfunction f = nullptr;
     check(cuda().mod_load(&m, L.cubin.data()), "cuModuleLoadData");
     check(cuda().mod_func(&f, m, L.name.c_str()), "cuModuleGetFunction");
+    if (L.tma && L.smem > 48 * 1024)
+      check(cuda().func_attr(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)L.smem), "cuFuncSetAttribute");
     l.mods.push_back(m);
     l.fns.push_back(f);
     l.nmods.push_back(nullptr);
@@ -182,15 +192,36 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
   std::lock_guard<std::mutex> g(p.mu);
   Plan::Loaded& l = loaded_for(p, ctx);
   for (size_t i = 0; i < p.launches.size(); i++) {
-    const Launch& L = p.launches[i];
+    Launch& L = p.launches[i];
     bool aligned = true;
     for (int t = 0; t < d.ntensors; t++)
       if (args.p[t] && ((uintptr_t)args.p[t] % (uintptr_t)L.align[t])) aligned = false;
     CUfunction f = l.fns[i];
-    const Launch* G = &L;
+    Launch* G = &L;
     if (!aligned) {
       f = narrow_fn(p, l, i);
       G = &p.narrow[i];
+    }
+    if (G->tma) {  // tensor maps for this run's base addresses (cached for the last pair)
+      const char* gin = args.p[G->tma_in_tensor] + G->tma_in_base * 2;
+      const char* gout = args.p[G->tma_out_tensor] + G->tma_out_base * 2;
+      if (gin != G->tma_last_in || gout != G->tma_last_out) {
+        unsigned box[5] = {64, 64, 1, 1, 1}, es[5] = {1, 1, 1, 1, 1};
+        const char* pe = std::getenv("FOP_TMA_L2PROMO");   // 0 none, 1 64B, 2 128B, 3 256B
+        int promo = pe && *pe ? std::atoi(pe) : TMAP_L2_PROMO_256B;
+        check(c.tmap_encode(&G->tma_map_in, TMAP_UINT16, (unsigned)G->tma_rank, (void*)gin, G->tma_in_dim,
+                            G->tma_in_stride, box, es, TMAP_INTERLEAVE_NONE, TMAP_SWIZZLE_128B, promo,
+                            TMAP_OOB_NONE), "cuTensorMapEncodeTiled(in)");
+        check(c.tmap_encode(&G->tma_map_out, TMAP_UINT16, (unsigned)G->tma_rank, (void*)gout, G->tma_out_dim,
+                            G->tma_out_stride, box, es, TMAP_INTERLEAVE_NONE, TMAP_SWIZZLE_128B, promo,
+                            TMAP_OOB_NONE), "cuTensorMapEncodeTiled(out)");
+        G->tma_last_in = gin;
+        G->tma_last_out = gout;
+      }
+      void* params[] = {&args, &G->tma_map_in, &G->tma_map_out};
+      check(c.launch(f, (unsigned)G->grid, 1, 1, (unsigned)G->block, 1, 1, (unsigned)G->smem, st, params, nullptr),
+            "cuLaunchKernel(tma)");
+      continue;
     }
     void* params[] = {&args};
     check(c.launch(f, (unsigned)G->grid, 1, 1, (unsigned)G->block, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");

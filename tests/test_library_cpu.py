@@ -161,6 +161,22 @@ def test_config_kernels_compile_for_sm100a_with_vector_access(name, expect):
     assert "LDL" not in sass and "STL" not in sass      # no register spills
 
 
+def test_tma_transpose_variant(monkeypatch):
+    monkeypatch.setenv("FOP_TR_TMA", "1")
+    op = FusedOp(W.cfg3())
+    assert op.info()["launches"][0]["block"] == 128
+    sass = _sass(op.cubin(0))
+    for pat in (r"UTMALDG\.3D", r"UTMASTG\.3D", r"LDS\.128", r"STS\.128", r"SYNCS"):
+        assert re.search(pat, sass), pat
+    assert "LDL" not in sass
+    # raw 16-bit move; and a 4-D map: padded NCHW rows keep h and w from collapsing
+    d = W.cfg3(2, 64, 64, 64)
+    d["stmts"][0]["expr"] = [("load", 0)]
+    assert "UTMALDG.3D" in _sass(FusedOp(d).cubin(0))
+    d["tensors"]["x"]["strides"] = [64 * 64 * 72, 64 * 72, 72, 1]
+    assert "UTMALDG.4D" in _sass(FusedOp(d).cubin(0))
+
+
 def test_256bit_vectors_on_request():
     op = FusedOp(W.cfg2(), max_vec_bytes=32)
     assert re.search(r"LDG\.E\.NA\.ENL2\.256", _sass(op.cubin(0)))

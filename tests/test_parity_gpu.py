@@ -99,6 +99,41 @@ def test_cfg3_transpose_bitexact(dims):
     assert_bitexact(got["out"], ref["out"], "out")
 
 
+@pytest.mark.parametrize("dims,move", [((2, 256, 56, 56), False), ((1, 40, 9, 13), False), ((2, 128, 8, 64), True),
+                                       ((1, 64, 64, 64), False)])
+def test_cfg3_tma_transpose_bitexact(monkeypatch, dims, move):
+    """TMA path (cp.async.bulk.tensor, 128B swizzle, mbarrier pipeline; opt-in FOP_TR_TMA=1):
+    64x64 tiles with out-of-bounds edges (C=40, HW=117) must give the same bits."""
+    monkeypatch.setenv("FOP_TR_TMA", "1")
+    d = W.cfg3(*dims)
+    d["tensors"]["x"]["init"] = ("special", 9)
+    if move:
+        d["stmts"][0]["expr"] = [("load", 0)]
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    li = op.info()["launches"][0]
+    tma = min(dims[1], dims[2] * dims[3]) >= 64
+    assert (li["block"] == 128) == tma
+    ref = O.run(d, x)
+    if move:
+        assert np.array_equal(got["out"].view(np.uint16), ref["out"].view(np.uint16))
+    else:
+        assert_bitexact(got["out"], ref["out"], "out")
+
+
+@pytest.mark.parametrize("tma", ["0", "1"])
+def test_transpose_padded_input_rows(monkeypatch, tma):
+    """NCHW input with padded rows (w stride 72 > 64): h and w no longer collapse
+    (4-D tensor map on the TMA path, 3 kernel loops on the register path)."""
+    monkeypatch.setenv("FOP_TR_TMA", tma)
+    d = W.cfg3(2, 64, 64, 64)
+    d["tensors"]["x"]["strides"] = [64 * 64 * 72, 64 * 72, 72, 1]
+    d["tensors"]["x"]["init"] = ("special", 5)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+
+
 def test_cfg3_classifies_as_transpose_with_both_sides_vectorised():
     d = W.cfg3(2, 256, 56, 56)
     from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
