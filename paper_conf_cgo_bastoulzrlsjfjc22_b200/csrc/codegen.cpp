@@ -84,6 +84,7 @@ struct DagCtx {
   std::function<bool(int)> load_varies;
   std::function<std::string(int, const std::string&)> fwd;   // element expression of forwarded stmt
   std::function<std::string(int)> scalar;                    // per-row scalar of a REDUCE
+  std::function<std::string(const std::string&)> self;       // read-modify-write running value
   std::string tag;                                           // name suffix
   std::string ev = "e";                                      // scalar element loop variable
 };
@@ -93,7 +94,7 @@ std::vector<bool> varies(const XStmt& x, const DagCtx& c) {
   for (size_t i = 0; i < x.nodes.size(); i++) {
     const XNode& n = x.nodes[i];
     if (n.op == FOP_OP_LOAD) v[i] = c.load_varies(n.acc);
-    else if (n.op == X_FWD) v[i] = true;
+    else if (n.op == X_FWD || n.op == X_SELF) v[i] = true;
     else if (n.op == X_SCALAR || n.op == FOP_OP_CONST) v[i] = false;
     else v[i] = (n.a >= 0 && v[n.a]) || (n.b >= 0 && v[n.b]);
   }
@@ -127,6 +128,7 @@ void emit_nodes(Out& o, const XStmt& x, const std::vector<bool>& var, bool want,
     std::string e;
     if (n.op == FOP_OP_LOAD) e = c.load(n.acc, c.ev);
     else if (n.op == X_FWD) e = c.fwd(n.src, c.ev);
+    else if (n.op == X_SELF) e = c.self(c.ev);
     else if (n.op == X_SCALAR) e = c.scalar(n.src);
     else {
       std::string a = n.a >= 0 ? node_name(x, var, n.a, c) : "";
@@ -157,6 +159,7 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
     switch (n.op) {
       case FOP_OP_LOAD: e = "fop::pk(" + c.load(n.acc, e0) + ", " + c.load(n.acc, e1) + ")"; break;
       case X_FWD: e = "fop::pk(" + c.fwd(n.src, e0) + ", " + c.fwd(n.src, e1) + ")"; break;
+      case X_SELF: e = "fop::pk(" + c.self(e0) + ", " + c.self(e1) + ")"; break;
       case FOP_OP_ADD: e = "fop::add2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
       case FOP_OP_SUB: e = "fop::sub2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
       case FOP_OP_MUL: e = "fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + ")"; break;
@@ -451,6 +454,113 @@ struct Gen {
         o.l("}");
       }
     }
+    o.ind--;
+    o.l("}");
+    footer();
+  }
+
+  // ------------------------------------------------------------ EW, read-modify-write
+  // Fig. 2(c) of the paper: forall (parallel loops) / for (the
+  // loops the target ignores, in original order) / forvec (d_v).  Each thread
+  // owns W target elements, keeps their running values in registers across
+  // the sequential loops (rounded to the target dtype after every update, as
+  // the in-order program stores them) and stores once at the end.
+  void gen_ew_seq() {
+    const int W = L.width;
+    const int64_t EV = L.kl[0].extent;
+    const int64_t NV = (EV + W - 1) / W;
+    const bool tail = EV % W != 0;
+    const int64_t STRIDE = L.grid * L.block;
+    const XStmt& x = L.stmts[0];
+    const fop_desc& dd = d;
+    header("EW read-modify-write (forall / for in order / forvec, Fig. 2(c))", 1);
+    o.l("const idx_t tid = (idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x;");
+    o.l("#pragma unroll 1");
+    o.l("for (idx_t g = tid; g < (idx_t)" + num(L.work) + "ull; g += (idx_t)" + num(STRIDE) + "ull) {");
+    o.ind++;
+    o.l("idx_t r = g;");
+    if (L.kl.size() > 1) {
+      o.l("const idx_t j = r % " + num(NV) + "u;");
+      o.l("r /= " + num(NV) + "u;");
+    } else {
+      o.l("const idx_t j = r;");
+    }
+    o.l("const idx_t iv = j * " + num(W) + "u;");
+    std::vector<std::pair<int, std::string>> its = {{0, "iv"}};
+    decompose("r", 1, (int)L.kl.size(), "", its);
+    std::string guard = tail ? "if (iv + e < " + num(EV) + "u) " : "";
+    auto seq_terms = [&](const Affine& a) {
+      std::string s;
+      for (size_t q = 0; q < L.seq.size(); q++) {
+        int64_t cq = a.coef[L.seq[q]];
+        if (cq) s += " + s" + num(q) + (cq == 1 ? "" : " * " + num(cq));
+      }
+      return s;
+    };
+    // running values of the target, read once
+    std::string dto = dtn(x.out_dtype);
+    std::string woff = affine(x.write, its);
+    int64_t cw = C(x.write, 0);
+    o.l("float ACC[" + num(W) + "];");
+    o.l("#pragma unroll");
+    o.l("for (int e = 0; e < " + num(W) + "; ++e) ACC[e] = 0.f;");
+    o.l("#pragma unroll");
+    o.l("for (int e = 0; e < " + num(W) + "; ++e) " + guard + "ACC[e] = fop::sload<" + dto +
+        ", fop::LD_COHERENT>(" + ptr(x.write.tensor, woff + " + e * " + num(cw)) + ");");
+    for (size_t q = 0; q < L.seq.size(); q++) {
+      o.l("#pragma unroll 1");
+      o.l("for (idx_t s" + num(q) + " = 0; s" + num(q) + " < " + num(dd.extent[L.seq[q]]) + "u; ++s" + num(q) + ") {");
+      o.ind++;
+    }
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      const Affine& a = L.loads[k];
+      int64_t cv = C(a, 0);
+      std::string off = "(" + affine(a, its) + seq_terms(a) + ")";
+      std::string nm = "L" + num(k);
+      std::string dt = dtn(dd.t[a.tensor].dtype);
+      if (cv == 0) {
+        o.l("const float " + nm + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
+      } else if (cv == 1 && !tail && L.load_cb[k]) {
+        o.l("float " + nm + "[" + num(W) + "];");
+        o.l("fop::vload<" + dt + ", " + num(W) + ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + nm + ", " +
+            ptr(a.tensor, off) + ");");
+      } else {
+        o.l("float " + nm + "[" + num(W) + "];");
+        o.l("#pragma unroll");
+        o.l("for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = " + (tail ? "(iv + e < " + num(EV) + "u) ? " : "") +
+            "fop::sload<" + dt + ", " + pol(a, false) + ">(" + ptr(a.tensor, off + " + e * " + num(cv)) + ")" +
+            (tail ? " : 0.f" : "") + ";");
+      }
+    }
+    DagCtx c;
+    c.load_varies = [&](int k) { return C(L.loads[k], 0) != 0; };
+    c.load = [&](int k, const std::string& e) {
+      return C(L.loads[k], 0) != 0 ? "L" + num(k) + "[" + e + "]" : "L" + num(k);
+    };
+    c.fwd = [&](int, const std::string&) { return std::string("0.f"); };
+    c.scalar = [&](int) { return std::string("0.f"); };
+    c.self = [&](const std::string& e) { return "ACC[" + e + "]"; };
+    auto var = varies(x, c);
+    emit_nodes(o, x, var, false, c);
+    o.l("float R[" + num(W) + "];");
+    Sink sk;
+    sk.scalar = [&](const std::string& v) { o.l("R[e] = " + v + ";"); };
+    sk.pair = [&](const std::string& v, const std::string& p) {
+      o.l("fop::upk(" + v + ", R[2 * " + p + "], R[2 * " + p + " + 1]);");
+    };
+    emit_elems(o, x, var, c, W, sk);
+    o.l("#pragma unroll");
+    o.l("for (int e = 0; e < " + num(W) + "; ++e) ACC[e] = fop::round_to<" + dto + ">(R[e]);   // the stored value");
+    for (size_t q = 0; q < L.seq.size(); q++) {
+      o.ind--;
+      o.l("}");
+    }
+    if (cw == 1 && !tail && L.store_cb[0])
+      o.l("fop::vstore<" + dto + ", " + num(W) + ", " + num(L.store_cb[0]) + ", fop::ST_DEFAULT>(" +
+          ptr(x.write.tensor, woff) + ", ACC);");
+    else
+      o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) " + guard + "fop::sstore<" + dto + ">(" +
+          ptr(x.write.tensor, woff + " + e * " + num(cw)) + ", ACC[e]);");
     o.ind--;
     o.l("}");
     footer();
@@ -1312,7 +1422,9 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
       break;
     case FOP_CLASS_ROW_REDUCE: g.gen_row(); break;
     case FOP_CLASS_COL_REDUCE: g.gen_col(); break;
-    default: g.gen_ew();
+    default:
+      if (!L.seq.empty()) g.gen_ew_seq();
+      else g.gen_ew();
   }
   L.src = g.o.s.str();
   return L.src;

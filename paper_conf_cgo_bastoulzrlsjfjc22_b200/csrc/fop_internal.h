@@ -54,7 +54,8 @@ Scenarios rank_scenarios(const fop_desc& d, int s, const fop_plan_opts& o);
 // ---------------------------------------------------------------- a5/a7
 enum XOp {  // expanded DAG node kinds (fop_opcode values + internal ones)
   X_FWD = 100,     // value of an earlier ASSIGN statement of the same launch (registers)
-  X_SCALAR = 101   // value of an earlier REDUCE statement of the same launch (per row)
+  X_SCALAR = 101,  // value of an earlier REDUCE statement of the same launch (per row)
+  X_SELF = 102     // read-modify-write: the running value of the statement's own target
 };
 
 struct XNode {
@@ -100,6 +101,7 @@ struct Launch {
   int trans_load = -1;            // TRANSPOSE: index into loads of the transposed access
   int coal_loop = -1;
   std::vector<int> order;         // launch loop order, innermost first (before collapse)
+  std::vector<int> seq;           // EW read-modify-write: loops walked in order by each thread (outer first)
   std::vector<KLoop> kl;          // kernel loops (see geometry.cpp for the per-class layout)
   int nsplit = 0;                 // ROW: #reduction kloops; COL: #parallel kloops; TR: 2
   std::vector<int> load_cb;       // per load: vector chunk bytes (0 = not contiguous along d_v)

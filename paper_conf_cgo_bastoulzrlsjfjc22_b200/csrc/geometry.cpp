@@ -135,7 +135,8 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   L.kl.clear();
   std::vector<int> rest;
   for (int l : L.loops)
-    if (l != L.vec_loop && l != L.read_loop) rest.push_back(l);
+    if (l != L.vec_loop && l != L.read_loop && std::find(L.seq.begin(), L.seq.end(), l) == L.seq.end())
+      rest.push_back(l);
   if (L.kclass == FOP_CLASS_EW || L.kclass == FOP_CLASS_TRANSPOSE) {
     std::vector<int> ord = {L.vec_loop};
     if (L.kclass == FOP_CLASS_TRANSPOSE) ord.push_back(L.read_loop);
@@ -256,7 +257,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     for (size_t k = 0; k < L.loads.size(); k++)
       if (coef(L, L.loads[k], 0) != 0) bytes += W * esize(d.t[L.loads[k].tensor].dtype);
     int u = bytes > 0 ? std::max(1, std::min(8, pow2_floor(std::max(1, 128 / bytes)))) : 4;
-    L.unroll = knob("FOP_EW_U", u);
+    L.unroll = L.seq.empty() ? knob("FOP_EW_U", u) : 1;   // RMW: one target vector per thread
     L.minblocks = knob("FOP_EW_MINB", L.unroll >= 4 ? 2 : 3);
     int64_t need = (L.work + (int64_t)L.block * L.unroll - 1) / ((int64_t)L.block * L.unroll);
     L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));

@@ -222,7 +222,18 @@ struct Group {
   int kclass = FOP_CLASS_EW;
   int vec = -1;
   bool has_reduce = false;
+  bool closed = false;   // a read-modify-write launch: nothing joins it
 };
+
+// read-modify-write ASSIGN (Fig. 2's Y): some loop of extent > 1 leaves the target index unchanged
+bool is_rmw(const fop_desc& d, int s) {
+  const fop_stmt& st = d.s[s];
+  if (st.kind != FOP_ASSIGN) return false;
+  Affine w = affine_of(d, st.acc[0]);
+  for (int k = 0; k < st.nloops; k++)
+    if (w.coef[st.loop[k]] == 0 && d.extent[st.loop[k]] > 1) return true;
+  return false;
+}
 
 // reduction loops of a REDUCE statement: loops its target does not depend on
 uint32_t red_loops(const fop_desc& d, int s) {
@@ -250,6 +261,11 @@ static int expand(const Plan& p, Launch& L, const std::vector<bool>& inl, int s,
   x.imm = q.imm;
   if (q.op == FOP_OP_LOAD) {
     const fop_access& a = st.acc[q.a];
+    if (a.tensor == st.acc[0].tensor && is_rmw(d, s)) {  // read-modify-write: running value
+      x.op = X_SELF;
+      out.push_back(x);
+      return memo[node_idx] = (int)out.size() - 1;
+    }
     int w = writer_before(d, s, a.tensor);
     if (w >= 0 && inl[w]) {  // inlined producer: substitute its DAG once per consumer
       if (pmemo[w] < 0) {
@@ -301,7 +317,30 @@ void plan_launches(Plan& p) {
     bool is_red = st.kind == FOP_REDUCE;
     bool row = is_red && (red_loops(d, s) >> v & 1u);
     bool joined = false;
-    if (!groups.empty()) {
+    bool rmw = is_rmw(d, s);
+    if (rmw) {
+      // the vector loop must be one the target depends on (each thread owns W
+      // target elements); take the best-ranked scenario whose innermost loop
+      // is such a loop — the fallback order of the scenario list
+      Affine w = affine_of(d, st.acc[0]);
+      const Scenarios& sc = p.scen[s];
+      int pick = -1;
+      for (int k = 0; k < sc.nscen && pick < 0; k++) {
+        int l = sc.loops[k][sc.len[k] - 1];
+        if (w.coef[l] != 0) pick = l;
+      }
+      if (pick < 0)
+        for (int k = st.nloops - 1; k >= 0 && pick < 0; k--)
+          if (w.coef[st.loop[k]] != 0) pick = st.loop[k];
+      Group g;
+      g.stmts.push_back(s);
+      g.vec = pick;
+      g.kclass = FOP_CLASS_EW;
+      g.closed = true;
+      groups.push_back(g);
+      continue;
+    }
+    if (!groups.empty() && !groups.back().closed) {
       Group& g = groups.back();
       const fop_stmt& g0 = d.s[g.stmts[0]];
       bool ok = g.kclass != FOP_CLASS_COL_REDUCE && g.kclass != FOP_CLASS_TRANSPOSE;
@@ -420,6 +459,17 @@ void plan_launches(Plan& p) {
     // coalescing loop: next loop of the main scenario (goal (ii))
     const Scenarios& sc = p.scen[L.main_stmt];
     L.coal_loop = sc.len[0] >= 2 ? sc.loops[0][sc.len[0] - 2] : -1;
+    if (g.closed) {  // read-modify-write: loops the target ignores run in order inside each thread
+      L.kclass = FOP_CLASS_EW;
+      L.read_loop = -1;
+      L.trans_load = -1;
+      const fop_stmt& st = d.s[L.main_stmt];
+      for (int k = 0; k < st.nloops; k++)
+        if (L.stmts[0].write.coef[st.loop[k]] == 0) L.seq.push_back(st.loop[k]);
+      L.coal_loop = -1;
+      for (int q = sc.len[0] - 2; q >= 0 && L.coal_loop < 0; q--)
+        if (L.stmts[0].write.coef[sc.loops[0][q]] != 0) L.coal_loop = sc.loops[0][q];
+    }
     p.launches.push_back(L);
   }
 

@@ -148,9 +148,17 @@ void validate(const fop_desc& d) {
     }
     for (int l = 0; l < d.nloops; l++)
       if (uses[l] > 1) fail(FOP_E_UNSUPPORTED, where(s) + "write access uses one loop in two dims");
-    if (st.kind == FOP_ASSIGN && !injective)
-      fail(FOP_E_UNSUPPORTED, where(s) + "ASSIGN whose write does not depend on every loop is an "
-                                         "in-order read-modify-write (Fig. 2's Y, row N2): not implemented");
+    if (st.kind == FOP_ASSIGN && !injective) {
+      // In-order read-modify-write (Fig. 2's Y): every iteration of the
+      // loops the target ignores updates the same element, in lexicographic
+      // order.  Supported when the statement reads its target only through
+      // the write access itself (the running value) — then one thread owns
+      // each target element and walks those loops sequentially.
+      for (int a = 1; a < st.nacc; a++)
+        if (st.acc[a].tensor == st.acc[0].tensor && !affine_of(d, st.acc[a]).same(w))
+          fail(FOP_E_UNSUPPORTED, where(s) + "read-modify-write statement reads its target at another index");
+      if (wt.dtype == FOP_I32) fail(FOP_E_UNSUPPORTED, where(s) + "i32 read-modify-write");
+    }
     if (st.kind == FOP_REDUCE && !has_red)
       fail(FOP_E_UNSUPPORTED, where(s) + "REDUCE statement without a reduction loop (use ASSIGN)");
 

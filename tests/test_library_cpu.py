@@ -43,7 +43,9 @@ def test_library_has_no_hard_cuda_dependency():
     (lambda d: d["stmts"][0].__setitem__("expr", [("add", 0, 1)]), "FOP_E_INVALID"),
     (lambda d: d["tensors"]["x"].__setitem__("role", "out") or
         d["stmts"][0].__setitem__("write", ("x", ["a", "b", "c"])) or None, None),
-    (lambda d: d["stmts"][0].__setitem__("write", ("out", ["a", "b", 0])), "FOP_E_UNSUPPORTED"),
+    (lambda d: d["stmts"][0].__setitem__("write", ("out", ["a", "b", 0])), None),   # RMW, last write wins
+    (lambda d: d["stmts"][0].update(kind="reduce", op="sum"), "FOP_E_UNSUPPORTED"),  # no reduction loop
+    (lambda d: d["stmts"][0].__setitem__("write", ("x", ["a", "b", "c"])), "FOP_E_INVALID"),  # writes an IN tensor
 ])
 def test_validation_status(mutate, status):
     d = W.cfg1()
@@ -56,9 +58,19 @@ def test_validation_status(mutate, status):
     assert e.value.status == status
 
 
-def test_fig2_rmw_is_reported_unsupported_not_wrong():
+def test_fig2_plan_is_fig2c():
+    """Fig. 2(c): forall i / for k { X; forvec j { Y } } — X inlined,
+    one launch, vector loop j, k walked in order inside each thread."""
+    op = FusedOp(W.fig2_running_example(64))
+    li = op.info()["launches"]
+    assert len(li) == 1 and li[0]["stmts"] == [1] and li[0]["vec_loop"] == "j"
+    src = op.source(0)
+    assert "for (idx_t s0 = 0; s0 < 64u; ++s0)" in src      # the in-order k loop
+    # a read of the RMW target at another index is not supported (would need a dependence test)
+    d = W.fig2_running_example(16)
+    d["stmts"][1]["reads"][0] = ("C", ["j", "i"])
     with pytest.raises(FopError) as e:
-        FusedOp(W.fig2_running_example(16), jit=0)
+        FusedOp(d, jit=0)
     assert e.value.status == "FOP_E_UNSUPPORTED"
 
 

@@ -88,6 +88,31 @@ def test_bf16_and_casts():
     assert diff.max() <= 1, diff.max()
 
 
+# ---------------------------------------------------------------- Fig. 2 running example (N2)
+@pytest.mark.parametrize("N,order", [(64, ("i", "j", "k")), (64, ("i", "k", "j")), (37, ("i", "j", "k")),
+                                     (256, ("i", "j", "k"))])
+def test_fig2_running_example_bitexact(N, order):
+    """Y: C[i][j] = C[i][j] + B[i][k] * D[k][i][j] over k in order, X: B = A + 1
+    inlined — the sequential k order is preserved, so even real-valued data
+    gives the oracle's exact bits."""
+    d = W.fig2_running_example(N, order_y=order)
+    d["tensors"]["D"]["init"] = ("normal", 0.0, 1.0, 23)
+    d["tensors"]["C"]["init"] = ("normal", 0.0, 1.0, 22)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.info()["launches"][0]["vec_loop"] == "j"
+    assert_bitexact(got["C"], O.run(d, x)["C"], "C")
+
+
+def test_fig2_fp16_target_rounds_every_step():
+    d = W.fig2_running_example(48)
+    d["tensors"]["C"]["dtype"] = "f16"
+    d["tensors"]["D"]["init"] = ("normal", 0.0, 1.0, 23)
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    assert_bitexact(got["C"], O.run(d, x)["C"], "C")
+
+
 # ---------------------------------------------------------------- TRANSPOSE
 @pytest.mark.parametrize("dims", [(2, 256, 56, 56), (1, 24, 5, 7), (2, 40, 3, 16), (1, 8, 1, 8)])
 def test_cfg3_transpose_bitexact(dims):
