@@ -162,6 +162,11 @@ typedef struct {
   int32_t coalesce_order;        /* FOP_ORDER_PAPER: threads follow the scenario order; MEMORY: write-memory order */
   int32_t sm_count;              /* 0 = 148 (B200); used for grid sizing */
   int32_t jit;                   /* 1 = compile kernels at fop_plan (NVRTC, sm_100a); 0 = analysis only */
+  int32_t autotune;              /* 1 = compile a few geometry variants per launch; the first fop_run on a
+                                    context times them on the caller's stream (synchronising once) and
+                                    keeps the fastest (tile sizes are auto-tuned in the paper too).
+                                    Skipped for plans that are not idempotent (in-place / read-modify-write)
+                                    and while the stream is being captured into a CUDA graph. */
 } fop_plan_opts;
 
 typedef enum {

@@ -1,6 +1,7 @@
 // abi.cpp — the extern "C" entry points declared in include/fop.h.
 // Every entry point converts internal failures into a fop_status plus a
 // thread-local message; nothing throws or aborts across the ABI.
+#include <algorithm>
 #include <cstring>
 #include <exception>
 #include <new>
@@ -57,6 +58,7 @@ void fop_plan_opts_default(fop_plan_opts* o) {
   o->coalesce_order = FOP_ORDER_MEMORY;  // measured faster on B200; PAPER kept as ablation
   o->sm_count = 148;
   o->jit = 1;
+  o->autotune = 1;
 }
 
 fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t** out) {
@@ -94,6 +96,47 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
       for (size_t i = 0; i < p.launches.size(); i++) {
         fop::generate(p, p.launches[i], (int)i);
         if (p.opts.jit) fop::jit_compile(p.launches[i]);
+      }
+      // auto-tuning candidates (fop.h: opts.autotune), only for idempotent plans
+      p.tunable = true;
+      for (size_t i = 0; i < p.launches.size(); i++) {
+        const fop::Launch& L = p.launches[i];
+        if (!L.seq.empty()) p.tunable = false;
+        for (const auto& x : L.stmts) {
+          if (p.desc.t[x.write.tensor].role == FOP_INOUT) p.tunable = false;
+          for (size_t j = 0; j <= i; j++)
+            for (const auto& a : p.launches[j].loads)
+              if (a.tensor == x.write.tensor) p.tunable = false;
+        }
+      }
+      p.variants.assign(p.launches.size(), {});
+      if (p.opts.autotune && p.opts.jit && p.tunable) {
+        for (size_t i = 0; i < p.launches.size(); i++) {
+          auto vs = fop::tuning_variants(p.launches[i]);
+          std::vector<std::string> seen = {p.launches[i].src};
+          for (size_t k = 1; k < vs.size(); k++) {
+            fop::Launch V = p.launches[i];
+            V.knobs = vs[k];
+            V.cubin.clear();
+            V.src.clear();
+            V.name_suffix = "_v" + std::to_string(k);
+            fop::finalize_launch_geometry(p, V);
+            V.ws_off = p.launches[i].ws_off;
+            if (V.ws_bytes > p.launches[i].ws_bytes) {
+              V.ws_off = (p.ws_bytes + 255) & ~size_t(255);
+              p.ws_bytes = V.ws_off + V.ws_bytes;
+            }
+            fop::generate(p, V, (int)i);
+            // identical geometry up to the name: nothing to tune
+            std::string body = V.src;
+            for (size_t q = body.find(V.name_suffix); q != std::string::npos; q = body.find(V.name_suffix))
+              body.erase(q, V.name_suffix.size());
+            if (std::find(seen.begin(), seen.end(), body) != seen.end()) continue;
+            seen.push_back(body);
+            fop::jit_compile(V);
+            p.variants[i].push_back(V);
+          }
+        }
       }
     } catch (...) {
       delete h;

@@ -51,8 +51,16 @@ struct Out {
   }
 };
 
+// set per statement (see varies()): the statement's result is rounded to a
+// 16-bit type, so transcendental fast forms are within one ulp
+thread_local bool g_approx16 = false;
+
 // C expression of a fused-DAG node given its operand expressions
 std::string op_expr(const XNode& n, const std::string& a, const std::string& b) {
+  if (g_approx16) {
+    if (n.op == FOP_OP_EXP) return "fop::exp_fast(" + a + ")";
+    if (n.op == FOP_OP_SIGMOID) return "fop::sigmoid_fast(" + a + ")";
+  }
   switch (n.op) {
     case FOP_OP_CONST: return fimm(n.imm);
     case FOP_OP_ADD: return "__fadd_rn(" + a + ", " + b + ")";
@@ -90,6 +98,10 @@ struct DagCtx {
 };
 
 std::vector<bool> varies(const XStmt& x, const DagCtx& c) {
+  {  // every statement emission starts here: decide the 16-bit fast forms
+    const char* e = std::getenv("FOP_APPROX16");
+    g_approx16 = !(e && *e == '0') && x.kind == FOP_ASSIGN && esize(x.out_dtype) == 2 && x.out_dtype != FOP_I32;
+  }
   std::vector<bool> v(x.nodes.size(), false);
   for (size_t i = 0; i < x.nodes.size(); i++) {
     const XNode& n = x.nodes[i];
@@ -105,13 +117,18 @@ std::string node_name(const XStmt& x, const std::vector<bool>& var, int i, const
   return std::string(var[i] ? "v" : "c") + num(x.stmt) + "_" + num(i) + c.tag;
 }
 
-// reachable set from the result
+// per-statement node overrides: a non-empty entry replaces the node's whole
+// cone by that expression (e.g. a shared-memory table lookup)
+thread_local const std::vector<std::string>* g_over = nullptr;
+bool overridden(int i) { return g_over && i < (int)g_over->size() && !(*g_over)[i].empty(); }
+
+// reachable set from the result (not descending into overridden nodes)
 std::vector<bool> reachable(const XStmt& x) {
   std::vector<bool> r(x.nodes.size(), false);
   if (x.result < 0) return r;
   r[x.result] = true;
   for (int i = x.result; i >= 0; i--) {
-    if (!r[i]) continue;
+    if (!r[i] || overridden(i)) continue;
     if (x.nodes[i].a >= 0) r[x.nodes[i].a] = true;
     if (x.nodes[i].b >= 0) r[x.nodes[i].b] = true;
   }
@@ -126,7 +143,8 @@ void emit_nodes(Out& o, const XStmt& x, const std::vector<bool>& var, bool want,
     if (!reach[i] || var[i] != want || (int)i == skip) continue;
     const XNode& n = x.nodes[i];
     std::string e;
-    if (n.op == FOP_OP_LOAD) e = c.load(n.acc, c.ev);
+    if (overridden((int)i)) e = (*g_over)[i];
+    else if (n.op == FOP_OP_LOAD) e = c.load(n.acc, c.ev);
     else if (n.op == X_FWD) e = c.fwd(n.src, c.ev);
     else if (n.op == X_SELF) e = c.self(c.ev);
     else if (n.op == X_SCALAR) e = c.scalar(n.src);
@@ -164,6 +182,12 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
       case FOP_OP_SUB: e = "fop::sub2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
       case FOP_OP_MUL: e = "fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + ")"; break;
       case FOP_OP_GELU_TANH: e = "fop::op_gelu_tanh2(" + opnd(n.a) + ")"; break;
+      case FOP_OP_DIV:
+        if (g_approx16 && !var[n.b]) {  // ÷ loop-invariant -> × correctly rounded reciprocal
+          e = "fop::mul2(" + opnd(n.a) + ", fop::pk1(__frcp_rn(" + node_name(x, var, n.b, c) + ")))";
+          break;
+        }
+        [[fallthrough]];
       default: {  // no packed form: per lane
         auto lane = [&](const char* f, int k) {
           return k < 0 ? std::string("") : (var[k] ? std::string("fop::") + f + "(" + pair_name(x, k, c) + ")"
@@ -315,6 +339,98 @@ struct Gen {
     }
   }
 
+  // ------------------------------------------------------------ shared-memory tables
+  // An invariant sub-DAG (constant along the vector loop) that depends on ONE
+  // kernel loop of small extent and contains a costly op (÷, √, exp, ...) —
+  // BN's scale[c] = γ/√(var+ε), shift[c] — is evaluated once per CTA for every
+  // value of that loop into shared memory, then looked up per vector, instead
+  // of being recomputed for every vector.  Identical IEEE operations, so the
+  // bits are unchanged.
+  struct Table {
+    int si, node, k;
+    int64_t E;
+    std::string name;
+  };
+  std::vector<Table> tables;
+  std::vector<std::vector<std::string>> over;   // per statement: node -> lookup expression
+
+  void plan_tables() {
+    tables.clear();
+    over.assign(L.stmts.size(), {});
+    if (!geometry_knob(L, "FOP_SMEM_TABLES", 1)) return;
+    int64_t bytes = 0;
+    for (size_t si = 0; si < L.stmts.size(); si++) {
+      const XStmt& x = L.stmts[si];
+      size_t n = x.nodes.size();
+      std::vector<uint32_t> dep(n, 0);
+      std::vector<bool> costly(n, false), var(n, false);
+      for (size_t i = 0; i < n; i++) {
+        const XNode& q = x.nodes[i];
+        if (q.op == FOP_OP_LOAD) {
+          for (size_t k = 0; k < L.kl.size(); k++)
+            if (C(L.loads[q.acc], (int)k) != 0) dep[i] |= 1u << k;
+        } else if (q.op == X_FWD || q.op == X_SELF || q.op == X_SCALAR) {
+          dep[i] = ~0u;
+        } else if (q.op != FOP_OP_CONST) {
+          dep[i] = (q.a >= 0 ? dep[q.a] : 0) | (q.b >= 0 ? dep[q.b] : 0);
+          costly[i] = q.op == FOP_OP_DIV || q.op == FOP_OP_SQRT || (q.op >= FOP_OP_EXP && q.op <= FOP_OP_GELU_ERF) ||
+                      (q.a >= 0 && costly[q.a]) || (q.b >= 0 && costly[q.b]);
+        }
+        var[i] = dep[i] & 1u;
+      }
+      over[si].assign(n, "");
+      for (size_t i = 0; i < n; i++) {
+        bool frontier = false;   // an invariant operand of a varying node
+        for (size_t j = i + 1; j < n; j++)
+          if (var[j] && (x.nodes[j].a == (int)i || x.nodes[j].b == (int)i)) frontier = true;
+        if (var[i] || !costly[i] || !frontier || __builtin_popcount(dep[i]) != 1) continue;
+        int k = __builtin_ctz(dep[i]);
+        int64_t E = L.kl[k].extent;
+        if (k == 0 || E > 8192 || bytes + E * 4 > 32 * 1024) continue;
+        bytes += E * 4;
+        Table t{(int)si, (int)i, k, E, "tbl" + num(x.stmt) + "_" + num(i)};
+        tables.push_back(t);
+      }
+    }
+  }
+
+  // emit the table fills (before the grid-stride loop) and return whether any
+  void emit_tables() {
+    if (tables.empty()) return;
+    for (const Table& t : tables) {
+      const XStmt& x = L.stmts[t.si];
+      o.l("__shared__ float " + t.name + "[" + num(t.E) + "];");
+      o.l("for (unsigned ti = threadIdx.x; ti < " + num(t.E) + "u; ti += " + num(L.block) + "u) {");
+      o.ind++;
+      // the cone of the table node, with its single loop bound to ti
+      std::vector<bool> cone(x.nodes.size(), false);
+      cone[t.node] = true;
+      for (int i = t.node; i >= 0; i--) {
+        if (!cone[i]) continue;
+        if (x.nodes[i].a >= 0) cone[x.nodes[i].a] = true;
+        if (x.nodes[i].b >= 0) cone[x.nodes[i].b] = true;
+      }
+      std::vector<std::pair<int, std::string>> its = {{t.k, "(idx_t)ti"}};
+      for (int i = 0; i <= t.node; i++) {
+        if (!cone[i]) continue;
+        const XNode& q = x.nodes[i];
+        std::string nm = t.name + "_" + num(i), e;
+        if (q.op == FOP_OP_LOAD) {
+          const Affine& a = L.loads[q.acc];
+          e = "fop::sload<" + std::string(dtn(d.t[a.tensor].dtype)) + ", fop::LD_CACHED>(" +
+              ptr(a.tensor, affine(a, its)) + ")";
+        } else {
+          e = op_expr(q, q.a >= 0 ? t.name + "_" + num(q.a) : "", q.b >= 0 ? t.name + "_" + num(q.b) : "");
+        }
+        o.l("const float " + nm + " = " + e + ";");
+      }
+      o.l(t.name + "[ti] = " + t.name + "_" + num(t.node) + ";");
+      o.ind--;
+      o.l("}");
+    }
+    o.l("__syncthreads();");
+  }
+
   // ------------------------------------------------------------ EW
   void gen_ew() {
     const int W = L.width;
@@ -325,6 +441,52 @@ struct Gen {
     const int64_t STRIDE = L.grid * L.block;
     bool raw = L.stmts.size() == 1 && L.stmts[0].move && es(L.stmts[0].write.tensor) == 2;
     header("EW (elementwise/broadcast, grid-stride over vectors of d_v)", 1);
+    if (!raw) plan_tables();
+    if (!tables.empty()) {
+      // the table fill (cold parameter loads + ÷/√) delays each CTA's first
+      // streaming loads: start the first iteration's vectors towards L2 now
+      o.l("{");
+      o.ind++;
+      o.l("const idx_t tid0 = (idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x;");
+      for (int u = 0; u < U; u++) {
+        std::string t = "_p" + num(u);
+        o.l("if (tid0 + (idx_t)" + num(STRIDE * u) + "ull < (idx_t)" + num(L.work) + "ull) {");
+        o.ind++;
+        o.l("idx_t r" + t + " = tid0 + (idx_t)" + num(STRIDE * u) + "ull;");
+        std::vector<std::pair<int, std::string>> pits;
+        if (L.kl.size() > 1) {
+          o.l("const idx_t j" + t + " = r" + t + " % " + num(NV) + "u;");
+          o.l("r" + t + " /= " + num(NV) + "u;");
+        } else {
+          o.l("const idx_t j" + t + " = r" + t + ";");
+        }
+        pits.push_back({0, "(j" + t + " * " + num(W) + "u)"});
+        decompose("r" + t, 1, (int)L.kl.size(), t, pits);
+        for (size_t k = 0; k < L.loads.size(); k++)
+          if (C(L.loads[k], 0) == 1 && L.load_cb[k])
+            o.l("asm volatile(\"prefetch.global.L2 [%0];\" :: \"l\"(" + ptr(L.loads[k].tensor, affine(L.loads[k], pits)) +
+                "));");
+        o.ind--;
+        o.l("}");
+      }
+      o.ind--;
+      o.l("}");
+    }
+    emit_tables();
+    // loads still needed per vector once tabled cones are cut off
+    std::vector<bool> need(L.loads.size(), raw);
+    for (size_t si = 0; si < L.stmts.size() && !raw; si++) {
+      std::vector<std::string> probe = over.empty() ? std::vector<std::string>() : over[si];
+      for (const Table& t : tables)
+        if (t.si == (int)si) probe[t.node] = "x";
+      g_over = &probe;
+      std::vector<bool> r = reachable(L.stmts[si]);
+      g_over = nullptr;
+      for (size_t i = 0; i < r.size(); i++)
+        if (r[i] && !(si < over.size() && !probe.empty() && !probe[i].empty()) &&
+            L.stmts[si].nodes[i].op == FOP_OP_LOAD)
+          need[L.stmts[si].nodes[i].acc] = true;
+    }
     o.l("const idx_t tid = (idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x;");
     o.l("#pragma unroll 1");
     o.l("for (idx_t g = tid; g < (idx_t)" + num(L.work) + "ull; g += (idx_t)" + num(STRIDE * U) + "ull) {");
@@ -347,6 +509,7 @@ struct Gen {
       if (tail) o.l("const bool full" + t + " = iv" + t + " + " + num(W) + "u <= " + num(EV) + "u;");
       // loads
       for (size_t k = 0; k < L.loads.size(); k++) {
+        if (!need[k]) continue;
         const Affine& a = L.loads[k];
         int64_t cv = C(a, 0);
         std::string off = affine(a, its[u]);
@@ -419,6 +582,12 @@ struct Gen {
         };
         c.fwd = [&, t](int s, const std::string& e) { return "F" + num(L.stmts[s].stmt) + t + "[" + e + "]"; };
         c.scalar = [&](int) { return std::string("0.f"); };
+        std::vector<std::string> ov(x.nodes.size());
+        for (const Table& tb : tables)
+          if (tb.si == (int)si)
+            for (auto& kv : its[u])
+              if (kv.first == tb.k) ov[tb.node] = tb.name + "[" + kv.second + "]";
+        g_over = &ov;
         auto var = varies(x, c);
         emit_nodes(o, x, var, false, c);
         std::string R = "R" + num(x.stmt) + t;
@@ -429,6 +598,7 @@ struct Gen {
           o.l("fop::upk(" + v + ", " + R + "[2 * " + p + "], " + R + "[2 * " + p + " + 1]);");
         };
         emit_elems(o, x, var, c, W, sk);
+        g_over = nullptr;
         if (x.fwd) {
           o.l("float F" + num(x.stmt) + t + "[" + num(W) + "];");
           o.l("#pragma unroll");
@@ -1414,7 +1584,7 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
   }
   g.idx = maxv < (int64_t(1) << 31) ? "unsigned" : "unsigned long long";
   L.name = std::string("fop_") + class_name(L.kclass) + (L.tma ? "_tma" : "") + "_k" + std::to_string(launch_index) +
-           (L.scalar_variant ? "_narrow" : "");
+           (L.scalar_variant ? "_narrow" : "") + L.name_suffix;
   switch (L.kclass) {
     case FOP_CLASS_TRANSPOSE:
       if (L.tma) g.gen_transpose_tma();

@@ -313,18 +313,11 @@ __device__ __forceinline__ void sstore_raw(char* p, u32 e) {
 // fp32 semantics shared with the oracle (include/fop.h); + - * / sqrt are the
 // _rn intrinsics, which the compiler never fuses into FMA.
 __device__ __forceinline__ float op_relu(float a) { return a > 0.f ? a : 0.f; }
-__device__ __forceinline__ float op_max(float a, float b) {
-  if (a != a) return b;
-  if (b != b) return a;
-  if (a == 0.f && b == 0.f) return (signbit(a) && signbit(b)) ? -0.f : 0.f;
-  return a > b ? a : b;
-}
-__device__ __forceinline__ float op_min(float a, float b) {
-  if (a != a) return b;
-  if (b != b) return a;
-  if (a == 0.f && b == 0.f) return (signbit(a) || signbit(b)) ? -0.f : 0.f;
-  return a < b ? a : b;
-}
+// max/min: NaN operands ignored, max(-0,+0) = +0, min(-0,+0) = -0 (reading
+// R24).  B200's FMNMX implements exactly this (tools/probes/maxmin_probe.cu,
+// measured), so fmaxf/fminf are single instructions with the oracle's bits.
+__device__ __forceinline__ float op_max(float a, float b) { return fmaxf(a, b); }
+__device__ __forceinline__ float op_min(float a, float b) { return fminf(a, b); }
 // .ftz forms: MUFU.EX2/RCP without the subnormal pre/post scaling.  In GELU
 // the flushed cases are e < 2^-126 (1 + e == 1 either way) and results below
 // 2^-126 (below fp16/bf16 resolution by 2^-100).
@@ -450,6 +443,14 @@ __device__ __forceinline__ void round2(float a, float b, float& ra, float& rb) {
 }
 __device__ __forceinline__ float op_gelu_erf(float v) { return 0.5f * v * erfcf(-0.70710678118654752f * v); }
 __device__ __forceinline__ float op_sigmoid(float v) { return __frcp_rn(1.0f + expf(-v)); }
+
+// Fast forms, used only for statements whose result is rounded to fp16/bf16
+// (DESIGN.md §4): relative error before the final rounding ~|x|*2^-24 + 2^-22
+// for |x| < 100 — far below 2^-11, so the <= 1 ulp lemma holds.
+__device__ __forceinline__ float exp_fast(float x) { return ex2_approx(x * 1.4426950408889634f); }
+__device__ __forceinline__ float sigmoid_fast(float x) {
+  return rcp_approx(1.0f + ex2_approx(x * -1.4426950408889634f));
+}
 
 // ------------------------------------------------------------------ reductions
 __device__ __forceinline__ float warp_sum(float v) {

@@ -102,6 +102,8 @@ struct Launch {
   int coal_loop = -1;
   std::vector<int> order;         // launch loop order, innermost first (before collapse)
   std::vector<int> seq;           // EW read-modify-write: loops walked in order by each thread (outer first)
+  std::vector<std::pair<std::string, int>> knobs;   // geometry overrides of this variant (auto-tuning)
+  std::string name_suffix;        // kernel name suffix of a tuning variant
   std::vector<KLoop> kl;          // kernel loops (see geometry.cpp for the per-class layout)
   int nsplit = 0;                 // ROW: #reduction kloops; COL: #parallel kloops; TR: 2
   std::vector<int> load_cb;       // per load: vector chunk bytes (0 = not contiguous along d_v)
@@ -149,7 +151,15 @@ struct Plan {
   // lazily built narrow variants (misaligned pointers), guarded by mu
   std::mutex mu;
   std::vector<Launch> narrow;     // same indexing as launches (empty src = not built)
-  struct Loaded { void* ctx; std::vector<void*> mods, fns, nmods, nfns; };
+  // auto-tuning candidates per launch (entry 0 = the launch itself is implicit)
+  std::vector<std::vector<Launch>> variants;
+  bool tunable = false;           // re-running the plan is idempotent (no in-place statements)
+  struct Loaded {
+    void* ctx;
+    std::vector<void*> mods, fns, nmods, nfns;
+    std::vector<std::vector<void*>> vfns;   // per launch: functions of variants[i]
+    std::vector<int> choice;                // per launch: -1 untuned, 0 = default, k = variants[i][k-1]
+  };
   std::vector<Loaded> loaded;
 };
 
@@ -158,6 +168,8 @@ void validate(const fop_desc& d);
 // planner.cpp
 void plan_launches(Plan& p);
 void finalize_launch_geometry(const Plan& p, Launch& L);
+int geometry_knob(const Launch& L, const char* name, int dflt);
+std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Launch& L);
 // codegen.cpp
 std::string generate(const Plan& p, Launch& L, int launch_index);
 extern const char* kDeviceHeader;   // device/fop_device.cuh, embedded at build time

@@ -124,6 +124,50 @@ int64_t coef(const Launch& L, const Affine& a, int k) { return a.coef[L.kl[k].me
 
 }  // namespace
 
+// A geometry knob: the launch's variant overrides first (auto-tuning), then
+// the environment (manual sweeps, tools/sweep.py), then the default rule.
+int geometry_knob(const Launch& L, const char* name, int dflt) {
+  for (const auto& kv : L.knobs)
+    if (kv.first == name) return kv.second;
+  const char* e = std::getenv(name);
+  return e && *e ? std::atoi(e) : dflt;
+}
+
+// Candidate geometries the run-time auto-tuner times (the paper's tile sizes
+// come from auto-tuners too).  Entry 0 is the default rule.  Chosen
+// from the measured sweeps (profiles/sweep_r01_*.log): streaming kernels
+// prefer few threads with many vectors in flight, ALU-heavy ones more threads.
+std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Launch& L) {
+  typedef std::vector<std::pair<std::string, int>> K;
+  std::vector<K> v = {K{}};
+  switch (L.kclass) {
+    case FOP_CLASS_EW:
+      if (!L.seq.empty()) break;
+      v.push_back({{"FOP_EW_U", 4}, {"FOP_EW_MINB", 2}, {"FOP_SMEM_TABLES", 0}});
+      v.push_back({{"FOP_EW_U", 2}, {"FOP_EW_MINB", 4}, {"FOP_SMEM_TABLES", 0}});
+      v.push_back({{"FOP_EW_U", 2}, {"FOP_EW_MINB", 4}});
+      v.push_back({{"FOP_EW_U", 1}, {"FOP_EW_MINB", 8}});
+      v.push_back({{"FOP_EW_U", 4}, {"FOP_EW_MINB", 3}});
+      break;
+    case FOP_CLASS_TRANSPOSE:
+      if (L.tma) break;
+      v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 2}});
+      v.push_back({{"FOP_TR_U", 2}, {"FOP_TR_MINB", 2}});
+      v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 3}});
+      break;
+    case FOP_CLASS_ROW_REDUCE:
+      v.push_back({{"FOP_ROW_MINB", 2}});
+      v.push_back({{"FOP_ROW_MINB", 4}});
+      v.push_back({{"FOP_BLOCK", 128}, {"FOP_ROW_MINB", 6}});
+      break;
+    default:
+      v.push_back({{"FOP_COL_U", 4}, {"FOP_COL_MINB", 3}});
+      v.push_back({{"FOP_COL_U", 8}, {"FOP_COL_MINB", 2}, {"FOP_COL_SLAB_BYTES", 256}});
+      v.push_back({{"FOP_COL_U", 4}, {"FOP_COL_MINB", 4}});
+  }
+  return v;
+}
+
 void finalize_launch_geometry(const Plan& p, Launch& L) {
   const fop_desc& d = p.desc;
   const fop_plan_opts& o = p.opts;
@@ -242,10 +286,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   // FOP_<CLASS>_U / FOP_<CLASS>_MINB override the defaults (tuning sweeps).
   int64_t prod_rest = 1;
   L.ws_bytes = 0;
-  auto knob = [](const char* name, int dflt) {
-    const char* e = std::getenv(name);
-    return e && *e ? std::atoi(e) : dflt;
-  };
+  auto knob = [&](const char* name, int dflt) { return geometry_knob(L, name, dflt); };
   L.block = knob("FOP_BLOCK", 256);
   if (L.kclass == FOP_CLASS_EW) {
     for (size_t k = 1; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;

@@ -43,6 +43,12 @@ struct Cuda {
   CUresult (*d2h)(void*, CUdeviceptr, size_t, CUstream);
   CUresult (*errstr)(CUresult, const char**);
   CUresult (*func_attr)(CUfunction, int, int);
+  CUresult (*ev_create)(void**, unsigned);
+  CUresult (*ev_record)(void*, CUstream);
+  CUresult (*ev_sync)(void*);
+  CUresult (*ev_elapsed)(float*, void*, void*);
+  CUresult (*ev_destroy)(void*);
+  CUresult (*stream_capturing)(CUstream, int*);
   CUresult (*tmap_encode)(void*, int, unsigned, void*, const uint64_t*, const uint64_t*, const unsigned*,
                           const unsigned*, int, int, int, int);
 };
@@ -76,6 +82,12 @@ Cuda& cuda() {
     SYM(d2h, "cuMemcpyDtoHAsync_v2");
     SYM(errstr, "cuGetErrorString");
     SYM(func_attr, "cuFuncSetAttribute");
+    SYM(ev_create, "cuEventCreate");
+    SYM(ev_record, "cuEventRecord");
+    SYM(ev_sync, "cuEventSynchronize");
+    SYM(ev_elapsed, "cuEventElapsedTime");
+    SYM(ev_destroy, "cuEventDestroy_v2");
+    SYM(stream_capturing, "cuStreamIsCapturing");
     SYM(tmap_encode, "cuTensorMapEncodeTiled");
 #undef SYM
     if (c.init(0) != 0) {
@@ -117,22 +129,31 @@ int64_t span_bytes(const fop_tensor& t) {
   return n * esize(t.dtype);
 }
 
+CUfunction load_fn(const Launch& L, std::vector<void*>& mods) {
+  CUmodule m = nullptr;
+  CUfunction f = nullptr;
+  check(cuda().mod_load(&m, L.cubin.data()), "cuModuleLoadData");
+  check(cuda().mod_func(&f, m, L.name.c_str()), "cuModuleGetFunction");
+  if (L.tma && L.smem > 48 * 1024)
+    check(cuda().func_attr(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)L.smem), "cuFuncSetAttribute");
+  mods.push_back(m);
+  return f;
+}
+
 Plan::Loaded& loaded_for(Plan& p, CUcontext ctx) {
   for (auto& l : p.loaded)
     if (l.ctx == ctx) return l;
   Plan::Loaded l;
   l.ctx = ctx;
-  for (auto& L : p.launches) {
-    CUmodule m = nullptr;
-    CUfunction f = nullptr;
-    check(cuda().mod_load(&m, L.cubin.data()), "cuModuleLoadData");
-    check(cuda().mod_func(&f, m, L.name.c_str()), "cuModuleGetFunction");
-    if (L.tma && L.smem > 48 * 1024)
-      check(cuda().func_attr(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)L.smem), "cuFuncSetAttribute");
-    l.mods.push_back(m);
-    l.fns.push_back(f);
+  for (size_t i = 0; i < p.launches.size(); i++) {
+    l.fns.push_back(load_fn(p.launches[i], l.mods));
     l.nmods.push_back(nullptr);
     l.nfns.push_back(nullptr);
+    std::vector<void*> vf;
+    if (i < p.variants.size())
+      for (const Launch& V : p.variants[i]) vf.push_back(load_fn(V, l.mods));
+    l.vfns.push_back(vf);
+    l.choice.push_back(vf.empty() ? 0 : -1);
   }
   p.loaded.push_back(l);
   return p.loaded.back();
@@ -191,17 +212,7 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
 
   std::lock_guard<std::mutex> g(p.mu);
   Plan::Loaded& l = loaded_for(p, ctx);
-  for (size_t i = 0; i < p.launches.size(); i++) {
-    Launch& L = p.launches[i];
-    bool aligned = true;
-    for (int t = 0; t < d.ntensors; t++)
-      if (args.p[t] && ((uintptr_t)args.p[t] % (uintptr_t)L.align[t])) aligned = false;
-    CUfunction f = l.fns[i];
-    Launch* G = &L;
-    if (!aligned) {
-      f = narrow_fn(p, l, i);
-      G = &p.narrow[i];
-    }
+  auto launch_one = [&](Launch* G, CUfunction f) {
     if (G->tma) {  // tensor maps for this run's base addresses (cached for the last pair)
       const char* gin = args.p[G->tma_in_tensor] + G->tma_in_base * 2;
       const char* gout = args.p[G->tma_out_tensor] + G->tma_out_base * 2;
@@ -221,10 +232,66 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
       void* params[] = {&args, &G->tma_map_in, &G->tma_map_out};
       check(c.launch(f, (unsigned)G->grid, 1, 1, (unsigned)G->block, 1, 1, (unsigned)G->smem, st, params, nullptr),
             "cuLaunchKernel(tma)");
-      continue;
+      return;
     }
     void* params[] = {&args};
     check(c.launch(f, (unsigned)G->grid, 1, 1, (unsigned)G->block, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
+  };
+
+  // Auto-tuning (opts.autotune): the first run of a launch on this context
+  // times each candidate geometry (1 warm-up + 3 timed launches, CUDA events
+  // on the caller's stream) and keeps the fastest.  All candidates compute the
+  // same results (bit-identical for ASSIGN; reductions within R16), and the
+  // plan is idempotent, so the extra launches only cost time once.
+  auto tune = [&](size_t i) {
+    int capturing = 0;
+    if (c.stream_capturing(st, &capturing) != 0 || capturing) return -1;
+    void *e0 = nullptr, *e1 = nullptr;
+    check(c.ev_create(&e0, 0), "cuEventCreate");
+    check(c.ev_create(&e1, 0), "cuEventCreate");
+    int best = 0;
+    float best_ms = 0.f;
+    for (size_t k = 0; k <= l.vfns[i].size(); k++) {
+      Launch* G = k == 0 ? &p.launches[i] : &p.variants[i][k - 1];
+      CUfunction f = k == 0 ? l.fns[i] : l.vfns[i][k - 1];
+      launch_one(G, f);
+      check(c.ev_record(e0, st), "cuEventRecord");
+      for (int r = 0; r < 3; r++) launch_one(G, f);
+      check(c.ev_record(e1, st), "cuEventRecord");
+      check(c.ev_sync(e1), "cuEventSynchronize");
+      float ms = 0.f;
+      check(c.ev_elapsed(&ms, e0, e1), "cuEventElapsedTime");
+      if (k == 0 || ms < best_ms) {
+        best = (int)k;
+        best_ms = ms;
+      }
+    }
+    c.ev_destroy(e0);
+    c.ev_destroy(e1);
+    return best;
+  };
+
+  for (size_t i = 0; i < p.launches.size(); i++) {
+    Launch& L = p.launches[i];
+    bool aligned = true;
+    for (int t = 0; t < d.ntensors; t++)
+      if (args.p[t] && ((uintptr_t)args.p[t] % (uintptr_t)L.align[t])) aligned = false;
+    if (!aligned) {
+      launch_one(&p.narrow[i], narrow_fn(p, l, i));
+      continue;
+    }
+    int ch = l.choice[i];
+    if (ch < 0) {
+      int t = tune(i);
+      if (t >= 0) l.choice[i] = ch = t;
+      else ch = 0;   // capturing: default geometry, tune on a later eager run
+    }
+    bool var_aligned = true;
+    if (ch > 0)
+      for (int t = 0; t < d.ntensors; t++)
+        if (args.p[t] && ((uintptr_t)args.p[t] % (uintptr_t)p.variants[i][ch - 1].align[t])) var_aligned = false;
+    if (ch > 0 && var_aligned) launch_one(&p.variants[i][ch - 1], l.vfns[i][ch - 1]);
+    else launch_one(&L, l.fns[i]);
   }
 
   if (host_ptrs) {  // device -> host results

@@ -65,7 +65,8 @@ class Desc(C.Structure):
 class PlanOpts(C.Structure):
     _fields_ = [("w", C.c_double * 5), ("thread_limit", C.c_int32), ("max_scenarios", C.c_int32),
                 ("max_vec_bytes", C.c_int32), ("readings", C.c_int32), ("force_width", C.c_int32),
-                ("coalesce_order", C.c_int32), ("sm_count", C.c_int32), ("jit", C.c_int32)]
+                ("coalesce_order", C.c_int32), ("sm_count", C.c_int32), ("jit", C.c_int32),
+                ("autotune", C.c_int32)]
 
 
 class LaunchInfo(C.Structure):
@@ -244,8 +245,11 @@ class FusedOp:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
-            _lib.fop_plan_destroy(h)
+        if h is not None and h.value and _lib is not None:
+            try:
+                _lib.fop_plan_destroy(h)
+            except Exception:       # interpreter shutdown
+                pass
             self._h = None
 
     # ------------------------------------------------------------ planner view

@@ -1,0 +1,109 @@
+"""fused operators shaped like the other Table I networks.
+
+CPU: the oracle's evaluation of each new composition is pinned to torch
+(float64 reference of the same formula, a library routine sharing no code with
+the oracle).  GPU (marked): the CUDA path vs the oracle with the north_star
+tolerances."""
+import numpy as np
+import pytest
+import torch
+
+import workloads as W
+from oracle import oracle as O
+
+SMALL = {
+    "lstm_cell": dict(B=8, H=96),
+    "mobilenet_bn_relu6": dict(N=2, C=24, H=14, W=14),
+    "resnext_bn_add_relu": dict(N=2, C=32, H=7, W=8),
+    "vgg_bias_relu": dict(N=2, C=16, H=9, W=16),
+    "bert_layernorm": dict(B=2, S=16, H=768),
+    "bert_softmax": dict(B=1, NH=3, S=128),
+}
+
+
+def _ulp16(a, b):
+    from harness import ordered16
+    return np.abs(ordered16(a) - ordered16(b))
+
+
+# ---------------------------------------------------------------- oracle pins (CPU)
+def test_oracle_layernorm_vs_torch():
+    d = W.N4["bert_layernorm"](**SMALL["bert_layernorm"])
+    x = W.make_inputs(d)
+    y = O.run(d, x)["y"]
+    xt = torch.from_numpy(x["x"].astype(np.float64).reshape(2, 16, 768))
+    ref = torch.nn.functional.layer_norm(xt, (768,), torch.from_numpy(x["gamma"].astype(np.float64)),
+                                         torch.from_numpy(x["beta"].astype(np.float64)), eps=1e-12)
+    assert _ulp16(y, ref.numpy().astype(np.float16).reshape(-1)).max() <= 1
+
+
+def test_oracle_softmax_vs_torch():
+    d = W.N4["bert_softmax"](**SMALL["bert_softmax"])
+    x = W.make_inputs(d)
+    y = O.run(d, x)["y"]
+    ref = torch.softmax(torch.from_numpy(x["x"].astype(np.float64).reshape(1, 3, 128, 128)), -1)
+    assert _ulp16(y, ref.numpy().astype(np.float16).reshape(-1)).max() <= 1
+    assert np.allclose(y.astype(np.float64).reshape(-1, 128).sum(1), 1.0, atol=2e-2)
+
+
+def test_oracle_lstm_vs_torch():
+    B, H = 8, 96
+    d = W.N4["lstm_cell"](B, H)
+    x = W.make_inputs(d)
+    r = O.run(d, x)
+    g = torch.from_numpy(x["g"].astype(np.float64).reshape(B, 4 * H))
+    i, f, gg, o = g.split(H, dim=1)
+    c = torch.sigmoid(f) * torch.from_numpy(x["c_prev"].astype(np.float64).reshape(B, H)) + \
+        torch.sigmoid(i) * torch.tanh(gg)
+    h = torch.sigmoid(o) * torch.tanh(torch.from_numpy(r["c"].astype(np.float64).reshape(B, H)))
+    assert np.allclose(r["c"].reshape(B, H), c.numpy(), rtol=1e-6, atol=1e-6)
+    assert np.allclose(r["h_out"].reshape(B, H), h.numpy(), rtol=1e-6, atol=1e-6)
+
+
+def test_oracle_relu6_and_residual_vs_numpy():
+    d = W.N4["mobilenet_bn_relu6"](**SMALL["mobilenet_bn_relu6"])
+    x = W.make_inputs(d)
+    y = O.run(d, x)["y"]
+    sc = x["gamma"] / np.sqrt(x["var"] + np.float32(1e-5))
+    sh = x["beta"] - x["mean"] * sc
+    v = x["x"].astype(np.float32).reshape(2, 24, 14, 14) * sc[None, :, None, None] + sh[None, :, None, None]
+    ref = np.minimum(np.maximum(v, np.float32(0)), np.float32(6)).astype(np.float16).reshape(-1)
+    assert np.array_equal(y.view(np.uint16), (ref + np.float16(0)).view(np.uint16))
+    d = W.N4["resnext_bn_add_relu"](**SMALL["resnext_bn_add_relu"])
+    x = W.make_inputs(d)
+    y = O.run(d, x)["y"]
+    sc = x["gamma"] / np.sqrt(x["var"] + np.float32(1e-5))
+    sh = x["beta"] - x["mean"] * sc
+    v = (x["x"].astype(np.float32).reshape(2, 32, 7, 8) * sc[None, :, None, None] + sh[None, :, None, None]) + \
+        x["res"].astype(np.float32).reshape(2, 32, 7, 8)
+    ref = np.where(v > 0, v, np.float32(0)).astype(np.float16).reshape(-1)
+    assert np.array_equal(y.view(np.uint16), ref.view(np.uint16))
+
+
+# ---------------------------------------------------------------- GPU parity
+@pytest.mark.gpu
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("full", [False, True])
+def test_n4_gpu_vs_oracle(name, full):
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from harness import run_gpu, assert_bitexact, assert_ulp
+    d = W.N4[name]() if full else W.N4[name](**SMALL[name])
+    if full and name in ("mobilenet_bn_relu6", "resnext_bn_add_relu", "vgg_bias_relu", "bert_softmax", "bert_layernorm"):
+        loop = list(d["loops"])[0]
+        d["loops"][loop] = 2                     # full per-sample shape, 2 samples (oracle time)
+        for t in d["tensors"].values():
+            if t["shape"] and t["shape"][0] == W.N4[name]()["loops"][loop] and len(t["shape"]) > 1:
+                t["shape"][0] = 2
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert len(op.info()["launches"]) == 1
+    ref = O.run(d, x)
+    for n, v in got.items():
+        if name == "lstm_cell":
+            err = np.abs(v.astype(np.float64) - ref[n].astype(np.float64))
+            assert np.all(err <= 4e-6 * np.abs(ref[n].astype(np.float64)) + 4e-6), (n, err.max())
+        elif name in ("bert_layernorm", "bert_softmax"):
+            assert_ulp(v, ref[n], 1, n)
+        else:
+            assert_bitexact(v, ref[n], n)
