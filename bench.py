@@ -63,25 +63,32 @@ class ClockSampler:
         self.samples = []
         self.stop = threading.Event()
         self.t = threading.Thread(target=self.run, daemon=True)
-
-    def run(self):
-        # NVML (the library nvidia-smi reads) every 5 ms; nvidia-smi itself as a fallback
-        try:
+        self.nvml = None
+        try:  # NVML (the library nvidia-smi reads), initialised before the timed region
             import pynvml as N
             N.nvmlInit()
-            h = N.nvmlDeviceGetHandleByIndex(self.index)
-            mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
-            bits = [N.nvmlClocksThrottleReasonHwSlowdown, N.nvmlClocksThrottleReasonHwThermalSlowdown,
-                    N.nvmlClocksThrottleReasonSwThermalSlowdown, N.nvmlClocksThrottleReasonSwPowerCap]
-            while not self.stop.is_set():
-                sm = N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
-                r = N.nvmlDeviceGetCurrentClocksThrottleReasons(h)
-                self.samples.append([str(sm), str(mx), "0x%x" % r] +
-                                    ["Active" if r & b else "Not Active" for b in bits])
-                self.stop.wait(0.005)
-            return
+            self.nvml = (N, N.nvmlDeviceGetHandleByIndex(index))
         except Exception:
-            pass
+            self.nvml = None
+
+    def sample_nvml(self):
+        N, h = self.nvml
+        mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
+        bits = [N.nvmlClocksThrottleReasonHwSlowdown, N.nvmlClocksThrottleReasonHwThermalSlowdown,
+                N.nvmlClocksThrottleReasonSwThermalSlowdown, N.nvmlClocksThrottleReasonSwPowerCap]
+        sm = N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
+        r = N.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+        self.samples.append([str(sm), str(mx), "0x%x" % r] + ["Active" if r & b else "Not Active" for b in bits])
+
+    def run(self):
+        if self.nvml is not None:   # every 2 ms (one query ~55 us)
+            while not self.stop.is_set():
+                try:
+                    self.sample_nvml()
+                except Exception:
+                    break
+                self.stop.wait(0.002)
+            return
         while not self.stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
@@ -94,12 +101,22 @@ class ClockSampler:
             self.stop.wait(0.2)
 
     def __enter__(self):
+        # the launch loop holds the GIL between ctypes calls: let the sampler
+        # thread in every 0.2 ms instead of Python's default 5 ms
+        self.old_switch = sys.getswitchinterval()
+        sys.setswitchinterval(0.0002)
+        if self.nvml is not None:
+            try:
+                self.sample_nvml()
+            except Exception:
+                pass
         self.t.start()
         return self
 
     def __exit__(self, *a):
         self.stop.set()
         self.t.join(timeout=10)
+        sys.setswitchinterval(self.old_switch)
 
     def summary(self):
         if not self.samples:
@@ -225,21 +242,28 @@ def run_fop(args):
     torch.cuda.synchronize()
 
     # ---- timed region: K steps between barrier + sync, CUDA events on the launch stream
-    ev = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)] for _ in ops]
-          for _ in range(args.steps)]
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clk = ClockSampler(local)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    with ClockSampler(local) as clk:
+    with clk:
         start.record(stream)
         for k in range(args.steps):
-            step(ev[k])
+            step()
         end.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     ms = start.elapsed_time(end)
+    # ---- per-launch durations for the roofline: the same K steps again with
+    # CUDA events around every fused op (kept out of the headline region)
+    ev = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)] for _ in ops]
+          for _ in range(args.steps)]
+    torch.cuda.synchronize()
+    for k in range(args.steps):
+        step(ev[k])
+    torch.cuda.synchronize()
     per_op = [statistics.mean(ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(args.steps))
               for i in range(len(ops))]
     t = torch.tensor([ms] + per_op, dtype=torch.float64, device=dev)
@@ -280,12 +304,14 @@ def run_fop(args):
     if os.path.exists(tp):
         with open(tp) as f:
             traffic = json.load(f).get(ops[dom]["name"])
-    per_op_json = {o["name"]: {"class": o["cls"], "kernel": "fop_%s_k0" % o["cls"], "ms": per_op[i],
+    for o in ops:
+        o["selected"] = o["op"].selected(0)   # kernel the auto-tuner kept (name, grid, block)
+    per_op_json = {o["name"]: {"class": o["cls"], "kernel": o["selected"][0], "ms": per_op[i],
                                "alg_bytes": o["bytes"], "GB_s": o["bytes"] / (per_op[i] / 1e3) / 1e9,
                                "frac_of_measured_peak": o["bytes"] / (per_op[i] / 1e3) / 1e9 / peak,
                                "frac_of_8TBs": o["bytes"] / (per_op[i] / 1e3) / 1e9 / 8000.0,
                                "vec_loop": o["kernel"]["vec_loop"], "width": o["kernel"]["width"],
-                               "grid": o["kernel"]["grid"]}
+                               "grid": o["selected"][1], "block": o["selected"][2]}
                    for i, o in enumerate(ops)}
 
     cpu = None
@@ -308,10 +334,13 @@ def run_fop(args):
                 "parallelism": "dp%d (batch-sharded, NCCL all-reduce of cfg4b partials)" % world,
                 "l2": "no flush: every input is re-read once per step after >1 GB of other ops' traffic "
                       "(B200 L2 126 MB); cfg2/cfg3 inputs alone exceed L2",
+                "per_op_note": "per-op times come from a second pass of the same K steps with CUDA events "
+                               "around each op; an op also pays the write-back of dirty L2 lines the "
+                               "previous op left (e.g. cfg4b after cfg4a's 50 MB y)",
                 "per_op": per_op_json,
                 "peak_gbs": peak, "peak_source": peak_src,
             },
-            "roofline": {"bound": "hbm", "kernel": "fop_%s_k0" % ops[dom]["cls"], "op": ops[dom]["name"],
+            "roofline": {"bound": "hbm", "kernel": ops[dom]["selected"][0], "op": ops[dom]["name"],
                          "achieved": dom_gbs, "peak": peak, "unit": "GB/s", "frac": dom_gbs / peak,
                          "traffic": traffic, "alg_bytes_per_launch": ops[dom]["bytes"],
                          "peak_source": peak_src},

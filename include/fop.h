@@ -237,6 +237,12 @@ FOP_API fop_status  fop_run(const fop_plan_t* plan, void* const* dev_ptrs, int32
 FOP_API fop_status  fop_run_host(const fop_plan_t* plan, void* const* host_ptrs,
                          void* const* dev_ptrs, int32_t nptrs, void* workspace, void* stream);
 
+/* The kernel fop_run launches for `launch` on the current CUDA context (after
+ * auto-tuning; the default geometry before the first run): its name, grid and
+ * block.  Pointers stay owned by the plan. */
+FOP_API fop_status  fop_plan_selected(const fop_plan_t* plan, int32_t launch, const char** kernel_name,
+                                      int64_t* grid, int32_t* block);
+
 FOP_API void        fop_plan_destroy(fop_plan_t* plan);
 FOP_API const char* fop_status_str(fop_status s);
 FOP_API const char* fop_last_error(void);      /* thread-local detail of the last failure */

@@ -217,6 +217,22 @@ fop_status fop_run_host(const fop_plan_t* plan, void* const* host_ptrs, void* co
   });
 }
 
+fop_status fop_plan_selected(const fop_plan_t* plan, int32_t i, const char** name, int64_t* grid, int32_t* block) {
+  return guarded([&] {
+    if (!plan || !name || i < 0 || i >= (int)plan->p.launches.size()) fop::fail(FOP_E_INVALID, "bad launch index");
+    fop::Plan& p = const_cast<fop_plan_t*>(plan)->p;
+    std::lock_guard<std::mutex> g(p.mu);
+    const fop::Launch* L = &p.launches[i];
+    void* ctx = fop::current_context_or_null();
+    for (const auto& l : p.loaded)
+      if (l.ctx == ctx && l.choice[i] > 0) L = &p.variants[i][l.choice[i] - 1];
+    *name = L->name.c_str();
+    if (grid) *grid = L->grid;
+    if (block) *block = L->block;
+    return FOP_OK;
+  });
+}
+
 void fop_plan_destroy(fop_plan_t* plan) { delete plan; }
 
 const char* fop_status_str(fop_status s) {

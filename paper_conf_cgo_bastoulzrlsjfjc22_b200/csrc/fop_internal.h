@@ -179,5 +179,6 @@ bool jit_available();
 // runtime.cpp
 fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream,
                     void* const* host_ptrs);
+void* current_context_or_null();   // the calling thread's CUDA context (nullptr without a driver)
 
 }  // namespace fop

@@ -176,6 +176,14 @@ CUfunction narrow_fn(Plan& p, Plan::Loaded& l, size_t i) {
 }
 }  // namespace
 
+void* current_context_or_null() {
+  Cuda& c = cuda();
+  if (!c.ok) return nullptr;
+  CUcontext ctx = nullptr;
+  if (c.ctx_get(&ctx) != 0) return nullptr;
+  return ctx;
+}
+
 fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream, void* const* host_ptrs) {
   const fop_desc& d = p.desc;
   if (nptrs != d.ntensors) fail(FOP_E_INVALID, "nptrs must equal desc.ntensors");

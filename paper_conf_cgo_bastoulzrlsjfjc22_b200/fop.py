@@ -102,13 +102,16 @@ _lib.fop_run.restype = C.c_int
 _lib.fop_run_host.argtypes = [C.c_void_p, C.POINTER(C.c_void_p), C.POINTER(C.c_void_p), C.c_int32,
                               C.c_void_p, C.c_void_p]
 _lib.fop_run_host.restype = C.c_int
+_lib.fop_plan_selected.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_char_p), C.POINTER(C.c_int64),
+                                   C.POINTER(C.c_int32)]
+_lib.fop_plan_selected.restype = C.c_int
 _lib.fop_plan_destroy.argtypes = [C.c_void_p]
 _lib.fop_status_str.restype = C.c_char_p
 _lib.fop_last_error.restype = C.c_char_p
 
 ABI_SYMBOLS = ["fop_abi_version", "fop_plan_opts_default", "fop_plan", "fop_plan_info_get",
                "fop_plan_workspace_bytes", "fop_plan_source", "fop_plan_cubin", "fop_run",
-               "fop_run_host", "fop_plan_destroy", "fop_status_str", "fop_last_error"]
+               "fop_run_host", "fop_plan_selected", "fop_plan_destroy", "fop_status_str", "fop_last_error"]
 
 
 class FopError(RuntimeError):
@@ -288,6 +291,12 @@ class FusedOp:
         p, n = C.c_void_p(), C.c_size_t()
         _check(_lib.fop_plan_cubin(self._h, i, C.byref(p), C.byref(n)))
         return C.string_at(p, n.value)
+
+    def selected(self, i=0):
+        """(kernel name, grid, block) fop_run launches for launch i on the current context."""
+        nm, g, b = C.c_char_p(), C.c_int64(), C.c_int32()
+        _check(_lib.fop_plan_selected(self._h, i, C.byref(nm), C.byref(g), C.byref(b)))
+        return nm.value.decode(), g.value, b.value
 
     @property
     def workspace_bytes(self):
