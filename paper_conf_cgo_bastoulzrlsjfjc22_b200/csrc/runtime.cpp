@@ -257,18 +257,27 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
     void *e0 = nullptr, *e1 = nullptr;
     check(c.ev_create(&e0, 0), "cuEventCreate");
     check(c.ev_create(&e1, 0), "cuEventCreate");
-    int best = 0;
-    float best_ms = 0.f;
-    for (size_t k = 0; k <= l.vfns[i].size(); k++) {
+    // time `reps` back-to-back launches of candidate k (after one warm-up)
+    auto time_k = [&](size_t k, int reps) {
       Launch* G = k == 0 ? &p.launches[i] : &p.variants[i][k - 1];
       CUfunction f = k == 0 ? l.fns[i] : l.vfns[i][k - 1];
       launch_one(G, f);
       check(c.ev_record(e0, st), "cuEventRecord");
-      for (int r = 0; r < 3; r++) launch_one(G, f);
+      for (int r = 0; r < reps; r++) launch_one(G, f);
       check(c.ev_record(e1, st), "cuEventRecord");
       check(c.ev_sync(e1), "cuEventSynchronize");
       float ms = 0.f;
       check(c.ev_elapsed(&ms, e0, e1), "cuEventElapsedTime");
+      return ms / reps;
+    };
+    // enough repetitions that a batch lasts >= 0.25 ms (event resolution ~2 us)
+    float t0 = time_k(0, 3);
+    int reps = t0 > 0.f ? (int)(0.25f / t0) + 1 : 3;
+    reps = reps < 3 ? 3 : (reps > 40 ? 40 : reps);
+    int best = 0;
+    float best_ms = 0.f;
+    for (size_t k = 0; k <= l.vfns[i].size(); k++) {
+      float ms = time_k(k, reps);
       if (k == 0 || ms < best_ms) {
         best = (int)k;
         best_ms = ms;
