@@ -1346,9 +1346,21 @@ struct Gen {
     o.l("const bool okc = j < " + num(NVD) + "u;");
     o.l("const idx_t iv = j * " + num(W) + "u;");
     cits.push_back({0, "iv"});
-    o.l("const idx_t r0 = chunk * " + num(RPC) + "u;");
-    o.l("const idx_t r1 = (r0 + " + num(RPC) + "u < " + num(ROWS) + "u) ? r0 + " + num(RPC) + "u : " + num(ROWS) +
-        "u;");
+    // Row assignment.  Interleaved (default): chunk c takes rows
+    // (k*NCH + c)*gr + rl, so the whole grid sweeps the matrix front to back
+    // together (measured +3% over contiguous chunks, tools/probes/col_probe.cu);
+    // contiguous: chunk c owns rows [c*RPC, (c+1)*RPC).  Both are fixed
+    // assignments, so the summation order is fixed run to run.
+    const bool il = L.col_il && NCH > 1;
+    const int64_t RSTEP = il ? NCH * (int64_t)L.gr : (int64_t)L.gr;   // between the U rows of a batch
+    if (il) {
+      o.l("const idx_t r0 = chunk * " + num(L.gr) + "u;");
+      o.l("const idx_t r1 = " + num(ROWS) + "u;");
+    } else {
+      o.l("const idx_t r0 = chunk * " + num(RPC) + "u;");
+      o.l("const idx_t r1 = (r0 + " + num(RPC) + "u < " + num(ROWS) + "u) ? r0 + " + num(RPC) + "u : " + num(ROWS) +
+          "u;");
+    }
     const bool packed = !isMax && W % 2 == 0 && g_packed;
     o.l("float acc[" + num(W) + "];");
     o.l("#pragma unroll");
@@ -1369,13 +1381,13 @@ struct Gen {
       if (cv == 1 && W * eb >= 4 && L.load_cb[k] >= 4 && !written_here(L.loads[k].tensor)) wpv[k] = W * eb / 4;
       else if (cv != 0) pipe = false;
     }
-    const int64_t BSTEP = (int64_t)L.gr * U;
+    const int64_t BSTEP = RSTEP * U;
     auto batch_loads = [&](const std::string& rbase, const std::string& buf, const std::string& tg) {
       for (int u = 0; u < U; u++) {
         std::string t = tg + num(u);
         o.l("{");
         o.ind++;
-        o.l("const idx_t rr = " + rbase + " + " + num((int64_t)L.gr * u) + "u;");
+        o.l("const idx_t rr = " + rbase + " + " + num(RSTEP * u) + "u;");
         o.l("idx_t q = rr;");
         std::vector<std::pair<int, std::string>> bits = cits;
         decompose("q", L.nsplit, (int)L.kl.size(), t, bits);
@@ -1404,22 +1416,24 @@ struct Gen {
         for (size_t k = 0; k < L.loads.size(); k++)
           if (wpv[k]) o.l("u32 B" + num(k) + "_" + num(u) + "[" + num(wpv[k]) + "];");
       batch_loads("(r + " + num(BSTEP) + "u)", "B", "_b");
+    } else {
+      // the batch's vector loads stay raw words (half the registers of fp32
+      // for 16-bit data) until they are accumulated
+      for (int u = 0; u < U; u++)
+        for (size_t k = 0; k < L.loads.size(); k++)
+          if (wpv[k]) o.l("u32 A" + num(k) + "_" + num(u) + "[" + num(wpv[k]) + "];");
+      batch_loads("r", "A", "_a");
     }
     std::vector<std::vector<std::pair<int, std::string>>> its(U);
     for (int u = 0; u < U; u++) {
       std::string t = "_" + num(u);
-      o.l("const idx_t rr" + t + " = r + " + num((int64_t)L.gr * u) + "u;");
+      o.l("const idx_t rr" + t + " = r + " + num(RSTEP * u) + "u;");
       o.l("const bool ok" + t + " = okc && rr" + t + " < r1;");
       o.l("idx_t q" + t + " = rr" + t + ";");
       its[u] = cits;
       decompose("q" + t, L.nsplit, (int)L.kl.size(), t, its[u]);
       for (size_t k = 0; k < L.loads.size(); k++) {
-        if (pipe && wpv[k]) {
-          o.l("float L" + num(k) + t + "[" + num(W) + "];");
-          o.l("fop::cvt_words<" + std::string(dtn(d.t[L.loads[k].tensor].dtype)) + ", " + num(W) + ">(L" + num(k) + t +
-              ", A" + num(k) + t + ");");
-          continue;
-        }
+        if (wpv[k]) continue;   // converted inside the accumulation below
         const Affine& a = L.loads[k];
         int64_t cv = C(a, 0);
         std::string off = affine(a, its[u]);
@@ -1452,6 +1466,12 @@ struct Gen {
       auto var = varies(x, c);
       o.l("if (ok" + t + ") {");
       o.ind++;
+      for (size_t k = 0; k < L.loads.size(); k++)
+        if (wpv[k]) {   // raw words -> fp32 only here, so one row's values are live at a time
+          o.l("float L" + num(k) + t + "[" + num(W) + "];");
+          o.l("fop::cvt_words<" + std::string(dtn(d.t[L.loads[k].tensor].dtype)) + ", " + num(W) + ">(L" + num(k) + t +
+              ", A" + num(k) + t + ");");
+        }
       emit_nodes(o, x, var, false, c);
       Sink sk;
       sk.scalar = [&](const std::string& v) { o.l("acc[e] = " + comb("acc[e]", v) + ";"); };
@@ -1479,20 +1499,41 @@ struct Gen {
       o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) { float a0_, a1_; fop::upk(accp[p], a0_, a1_); "
           "acc[2 * p] = __fadd_rn(acc[2 * p], a0_); acc[2 * p + 1] = __fadd_rn(acc[2 * p + 1], a1_); }");
     }
-    // block tree over the row lanes (fixed order => deterministic)
+    // Block combine over the row lanes, fixed order (deterministic): xor
+    // butterflies over the row lanes that share a warp, then one thread per
+    // (column, element) adds the NG warp-group results in order; the block's
+    // sums end in red[0 .. SW).
+    const int RPW = L.gv < 32 ? 32 / L.gv : 1;   // row lanes per warp
+    const int NG = L.gr / RPW;                    // row groups (one per warp when gv < 32)
     auto tree = [&]() {
-      o.l("#pragma unroll");
-      o.l("for (int e = 0; e < " + num(W) + "; ++e) red[rl * " + num(SW) + "u + cv * " + num(W) + "u + e] = acc[e];");
-      o.l("__syncthreads();");
-      o.l("#pragma unroll 1");
-      o.l("for (unsigned s = " + num(L.gr / 2) + "u; s > 0u; s >>= 1) {");
-      o.l("  if (rl < s) {");
-      o.l("    #pragma unroll");
-      o.l("    for (int e = 0; e < " + num(W) + "; ++e) { float* a_ = &red[rl * " + num(SW) + "u + cv * " + num(W) +
-          "u + e]; *a_ = " + comb("*a_", "a_[s * " + num(SW) + "u]") + "; }");
-      o.l("  }");
-      o.l("  __syncthreads();");
+      if (RPW > 1) {
+        o.l("#pragma unroll");
+        o.l("for (int e = 0; e < " + num(W) + "; ++e) {");
+        for (int m = L.gv; m < 32; m *= 2)
+          o.l("  acc[e] = " + comb("acc[e]", "__shfl_xor_sync(0xffffffffu, acc[e], " + num(m) + ")") + ";");
+        o.l("}");
+      }
+      if (NG == 1) {
+        o.l("if (rl == 0u) {");
+        o.l("  #pragma unroll");
+        o.l("  for (int e = 0; e < " + num(W) + "; ++e) red[cv * " + num(W) + "u + e] = acc[e];");
+        o.l("}");
+        o.l("__syncthreads();");
+        return;
+      }
+      o.l("if (rl % " + num(RPW) + "u == 0u) {");
+      o.l("  #pragma unroll");
+      o.l("  for (int e = 0; e < " + num(W) + "; ++e) red[(rl / " + num(RPW) + "u) * " + num(SW) + "u + cv * " + num(W) +
+          "u + e] = acc[e];");
       o.l("}");
+      o.l("__syncthreads();");
+      o.l("for (unsigned t_ = tid; t_ < " + num(SW) + "u; t_ += " + num(L.block) + "u) {");
+      o.l("  float s_ = red[t_];");
+      o.l("  #pragma unroll");
+      o.l("  for (int g = 1; g < " + num(NG) + "; ++g) s_ = " + comb("s_", "red[g * " + num(SW) + "u + t_]") + ";");
+      o.l("  red[t_] = s_;");
+      o.l("}");
+      o.l("__syncthreads();");
     };
     tree();
     auto final_store = [&]() {
@@ -1540,13 +1581,39 @@ struct Gen {
       o.l("__threadfence();");
       o.l("#pragma unroll");
       o.l("for (int e = 0; e < " + num(W) + "; ++e) acc[e] = " + init + ";");
-      o.l("for (idx_t c = rl; c < " + num(NCH) + "u; c += " + num(L.gr) + "u) {");
-      o.l("  #pragma unroll");
-      o.l("  for (int e = 0; e < " + num(W) + "; ++e) { float v_; const float* p_ = &part[(c * " + num(slabs) +
-          "u + slab) * " + num(SW) + "u + cv * " + num(W) +
-          "u + e]; asm volatile(\"ld.global.cg.f32 %0, [%1];\" : \"=f\"(v_) : \"l\"(p_)); acc[e] = " +
-          comb("acc[e]", "v_") + "; }");
-      o.l("}");
+      // every partial this thread combines is requested before the first is
+      // used (one L2 round trip instead of one per chunk), then combined in
+      // chunk order
+      const int64_t MAXIT = (NCH + L.gr - 1) / L.gr;
+      const bool v4 = W % 4 == 0 && MAXIT <= 8;
+      if (v4) {
+        o.l("float pv_[" + num(MAXIT) + "][" + num(W) + "];");
+        o.l("#pragma unroll");
+        o.l("for (int it = 0; it < " + num(MAXIT) + "; ++it) {");
+        o.l("  const idx_t c = rl + it * " + num(L.gr) + "u;");
+        o.l("  if (c < " + num(NCH) + "u) {");
+        o.l("    const float* p_ = &part[(c * " + num(slabs) + "u + slab) * " + num(SW) + "u + cv * " + num(W) + "u];");
+        o.l("    #pragma unroll");
+        o.l("    for (int q = 0; q < " + num(W / 4) + "; ++q) asm volatile(\"ld.global.cg.v4.f32 {%0,%1,%2,%3}, [%4];\" : "
+            "\"=f\"(pv_[it][4 * q]), \"=f\"(pv_[it][4 * q + 1]), \"=f\"(pv_[it][4 * q + 2]), \"=f\"(pv_[it][4 * q + 3]) : "
+            "\"l\"(p_ + 4 * q));");
+        o.l("  }");
+        o.l("}");
+        o.l("#pragma unroll");
+        o.l("for (int it = 0; it < " + num(MAXIT) + "; ++it)");
+        o.l("  if (rl + it * " + num(L.gr) + "u < " + num(NCH) + "u) {");
+        o.l("    #pragma unroll");
+        o.l("    for (int e = 0; e < " + num(W) + "; ++e) acc[e] = " + comb("acc[e]", "pv_[it][e]") + ";");
+        o.l("  }");
+      } else {
+        o.l("for (idx_t c = rl; c < " + num(NCH) + "u; c += " + num(L.gr) + "u) {");
+        o.l("  #pragma unroll");
+        o.l("  for (int e = 0; e < " + num(W) + "; ++e) { float v_; const float* p_ = &part[(c * " + num(slabs) +
+            "u + slab) * " + num(SW) + "u + cv * " + num(W) +
+            "u + e]; asm volatile(\"ld.global.cg.f32 %0, [%1];\" : \"=f\"(v_) : \"l\"(p_)); acc[e] = " +
+            comb("acc[e]", "v_") + "; }");
+        o.l("}");
+      }
       o.l("__syncthreads();");
       tree();
       final_store();

@@ -113,6 +113,7 @@ struct Launch {
   int minblocks = 1;              // __launch_bounds__ min blocks/SM; grid-stride grids = SMs x minblocks
   int row_prefetch = 0;           // ROW: prefetch the next row's streaming loads
   int col_pipe = 0;               // COL: software-pipelined row batches
+  int col_il = 1;                 // COL: chunks interleave over rows (grid sweeps rows together)
   int row_hoist = 1;              // ROW: keep row-invariant loads in registers across rows
   // TRANSPOSE through TMA (16-bit data): 64x64 tiles, tensor maps encoded per run
   int tma = 0;

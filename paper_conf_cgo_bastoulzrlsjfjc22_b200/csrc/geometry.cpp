@@ -161,9 +161,9 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       v.push_back({{"FOP_BLOCK", 128}, {"FOP_ROW_MINB", 6}});
       break;
     default:
-      v.push_back({{"FOP_COL_U", 4}, {"FOP_COL_MINB", 3}});
-      v.push_back({{"FOP_COL_U", 8}, {"FOP_COL_MINB", 2}, {"FOP_COL_SLAB_BYTES", 256}});
-      v.push_back({{"FOP_COL_U", 4}, {"FOP_COL_MINB", 4}});
+      v.push_back({{"FOP_COL_U", 2}, {"FOP_COL_MINB", 8}});
+      v.push_back({{"FOP_COL_U", 8}, {"FOP_COL_MINB", 4}});
+      v.push_back({{"FOP_COL_U", 4}, {"FOP_COL_MINB", 6}, {"FOP_COL_SLAB_BYTES", 256}});
   }
   return v;
 }
@@ -400,16 +400,19 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       if (coef(L, a, 0) == 1) big = &a;
     int es_ld = big ? esize(d.t[big->tensor].dtype) : 4;
     int gv = (int)std::min<int64_t>(32, std::max<int64_t>(1, knob("FOP_COL_SLAB_BYTES", 128) / (W * es_ld)));
-    gv = std::min(gv, pow2_floor(nvd));
+    gv = std::min(pow2_floor(gv), pow2_floor(nvd));
     L.gv = gv;
     L.gr = L.block / gv;
     int64_t slabs = (nvd + gv - 1) / gv;
     for (int k = 1; k < L.nsplit; k++) slabs *= L.kl[k].extent;
     int64_t rows = 1;
     for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
-    L.col_pipe = knob("FOP_COL_PIPE", 0);   // measured: no gain over U=8 batches (sweep_r01_4)
-    L.minblocks = knob("FOP_COL_MINB", 2);
-    L.unroll = knob("FOP_COL_U", L.col_pipe ? 4 : 8);
+    L.col_pipe = knob("FOP_COL_PIPE", 0);   // measured: no gain over plain batches (sweep_r01_4)
+    L.col_il = knob("FOP_COL_IL", 1);
+    // 6 blocks/SM x 4 rows in flight: the column-sum probe and the sweep
+    // (profiles/col_probe_r01.log, sweep_r01_col.log) peak at 6-8 blocks/SM
+    L.minblocks = knob("FOP_COL_MINB", 6);
+    L.unroll = knob("FOP_COL_U", 4);
     int64_t target = (int64_t)sms * L.minblocks;   // one resident wave
     int64_t nch = std::max<int64_t>(1, target / std::max<int64_t>(1, slabs));
     nch = std::min<int64_t>(nch, std::max<int64_t>(1, (rows + L.gr - 1) / L.gr));
