@@ -49,7 +49,7 @@ extern "C" {
 #define FOP_API
 #endif
 
-#define FOP_ABI_VERSION 1
+#define FOP_ABI_VERSION 2
 
 #define FOP_MAX_RANK     8   /* tensor rank */
 #define FOP_MAX_LOOPS    8   /* loops of the fused operator */
@@ -60,6 +60,7 @@ extern "C" {
 #define FOP_MAX_FIN      8   /* finalize nodes per REDUCE statement */
 #define FOP_MAX_LAUNCH   8   /* kernel launches per plan */
 #define FOP_MAX_SCEN     8   /* scenarios kept per statement ("set to 8") */
+#define FOP_MAX_DEPS    16   /* dependence vectors reported per statement */
 
 typedef enum {
   FOP_OK = 0,
@@ -187,7 +188,13 @@ typedef struct {
   int32_t coal_loop;         /* next loop mapped to threads (scenario goal (ii)), -1 if none */
   int64_t grid;
   int32_t block;
-  int32_t _pad;
+  int32_t nseq;              /* loops each thread walks in order (read-modify-write / recurrence), 0 = none */
+  int32_t seq[FOP_MAX_LOOPS];/* their ids, outermost first */
+  int32_t scen_pick;         /* scenario whose innermost loop is d_v; -1 = none feasible (row N3) */
+  int32_t fallback;          /* row N3 influence-tree outcome: 0 scenario as ranked, 1 looser variant (vector
+                                constraint only), 2 no feasible scenario: uninfluenced schedule, no
+                                explicit vector type, 3 fully sequential (every loop carries a
+                                dependence) */
 } fop_launch_info;
 
 typedef struct {
@@ -199,6 +206,11 @@ typedef struct {
   int32_t nlaunch;
   fop_launch_info launch[FOP_MAX_LAUNCH];
   size_t  workspace_bytes;
+  /* validity: uniform self-dependences per statement — distance vectors by loop id,
+     lexicographically positive in the statement's loop order; anti = the read precedes the write */
+  int32_t ndeps[FOP_MAX_STMTS];
+  int64_t dep[FOP_MAX_STMTS][FOP_MAX_DEPS][FOP_MAX_LOOPS];
+  int32_t dep_anti[FOP_MAX_STMTS][FOP_MAX_DEPS];
 } fop_plan_info;
 
 typedef struct fop_plan fop_plan_t;   /* opaque, immutable after fop_plan */

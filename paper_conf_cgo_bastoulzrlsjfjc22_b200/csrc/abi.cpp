@@ -169,15 +169,26 @@ fop_status fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* o) {
       li.kernel_class = L.kclass;
       li.main_stmt = L.main_stmt;
       li.stmt_mask = L.mask;
-      li.vec_loop = L.vec_loop;
+      li.vec_loop = L.virt_vec ? -1 : L.vec_loop;
       li.width = L.width;
       li.read_loop = L.read_loop;
       li.read_width = L.read_width;
       li.coal_loop = L.coal_loop;
       li.grid = L.grid;
       li.block = L.block;
+      li.nseq = (int32_t)L.seq.size();
+      for (size_t q = 0; q < L.seq.size() && q < FOP_MAX_LOOPS; q++) li.seq[q] = L.seq[q];
+      li.scen_pick = L.scen_pick;
+      li.fallback = L.fallback;
     }
     o->workspace_bytes = p.ws_bytes;
+    for (int s = 0; s < p.desc.nstmts; s++) {
+      o->ndeps[s] = (int32_t)std::min<size_t>(p.deps[s].size(), FOP_MAX_DEPS);
+      for (int k = 0; k < o->ndeps[s]; k++) {
+        for (int l = 0; l < FOP_MAX_LOOPS; l++) o->dep[s][k][l] = p.deps[s][k].dist[l];
+        o->dep_anti[s][k] = p.deps[s][k].anti;
+      }
+    }
     return FOP_OK;
   });
 }

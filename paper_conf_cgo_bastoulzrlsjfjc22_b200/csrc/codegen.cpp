@@ -629,12 +629,19 @@ struct Gen {
     footer();
   }
 
-  // ------------------------------------------------------------ EW, read-modify-write
+  // ------------------------------------------------------------ EW, read-modify-write / recurrence
   // Fig. 2(c) of the paper: forall (parallel loops) / for (the
-  // loops the target ignores, in original order) / forvec (d_v).  Each thread
-  // owns W target elements, keeps their running values in registers across
-  // the sequential loops (rounded to the target dtype after every update, as
-  // the in-order program stores them) and stores once at the end.
+  // loops carrying the statement's dependences, in original order) / forvec
+  // (d_v).  Read-modify-write (the target ignores the sequential loops): each
+  // thread owns W target elements, keeps their running values in registers
+  // across the sequential loops (rounded to the target dtype after every
+  // update, as the in-order program stores them) and stores once at the end.
+  // Recurrence (row N3: the target depends on every sequential loop and is
+  // read back at a constant distance): each iteration stores its result; a
+  // read 1..4 iterations back along the innermost sequential loop comes from
+  // a register ring holding this thread's last stored values, any other read
+  // of the target from memory (coherent loads of this thread's own stores —
+  // the planner proved every dependence stays inside one thread).
   void gen_ew_seq() {
     const int W = L.width;
     const int64_t EV = L.kl[0].extent;
@@ -643,7 +650,9 @@ struct Gen {
     const int64_t STRIDE = L.grid * L.block;
     const XStmt& x = L.stmts[0];
     const fop_desc& dd = d;
-    header("EW read-modify-write (forall / for in order / forvec, Fig. 2(c))", 1);
+    const bool rec = L.rec;
+    header(rec ? "EW recurrence (forall / for in order / forvec, row N3)"
+               : "EW read-modify-write (forall / for in order / forvec, Fig. 2(c))", 1);
     o.l("const idx_t tid = (idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x;");
     o.l("#pragma unroll 1");
     o.l("for (idx_t g = tid; g < (idx_t)" + num(L.work) + "ull; g += (idx_t)" + num(STRIDE) + "ull) {");
@@ -667,39 +676,74 @@ struct Gen {
       }
       return s;
     };
-    // running values of the target, read once
     std::string dto = dtn(x.out_dtype);
     std::string woff = affine(x.write, its);
     int64_t cw = C(x.write, 0);
-    o.l("float ACC[" + num(W) + "];");
-    o.l("#pragma unroll");
-    o.l("for (int e = 0; e < " + num(W) + "; ++e) ACC[e] = 0.f;");
-    o.l("#pragma unroll");
-    o.l("for (int e = 0; e < " + num(W) + "; ++e) " + guard + "ACC[e] = fop::sload<" + dto +
-        ", fop::LD_COHERENT>(" + ptr(x.write.tensor, woff + " + e * " + num(cw)) + ");");
+    auto store_vals = [&](const std::string& off, const std::string& v) {
+      if (cw == 1 && !tail && L.store_cb[0])
+        o.l("fop::vstore<" + dto + ", " + num(W) + ", " + num(L.store_cb[0]) + ", fop::ST_DEFAULT>(" +
+            ptr(x.write.tensor, off) + ", " + v + ");");
+      else
+        o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) " + guard + "fop::sstore<" + dto + ">(" +
+            ptr(x.write.tensor, off + " + e * " + num(cw)) + ", " + v + "[e]);");
+    };
+    int maxd = 0;
+    if (rec)
+      for (int f : L.fwd_dist) maxd = std::max(maxd, f);
+    if (!rec) {  // running values of the target, read once
+      o.l("float ACC[" + num(W) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) ACC[e] = 0.f;");
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) " + guard + "ACC[e] = fop::sload<" + dto +
+          ", fop::LD_COHERENT>(" + ptr(x.write.tensor, woff + " + e * " + num(cw)) + ");");
+    }
+    // ring of this thread's last stored values.  Zero-initialised although
+    // never read before being written: left undefined on loop entry, ptxas
+    // 12.9 merged H2 with the new H1 (tools/probes/fibdbg.py, measured).
+    for (int q = 1; q <= maxd; q++) {
+      o.l("float H" + num(q) + "[" + num(W) + "];   // stored value " + num(q) + " iteration(s) back");
+      o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) H" + num(q) + "[e] = 0.f;");
+    }
     for (size_t q = 0; q < L.seq.size(); q++) {
       o.l("#pragma unroll 1");
       o.l("for (idx_t s" + num(q) + " = 0; s" + num(q) + " < " + num(dd.extent[L.seq[q]]) + "u; ++s" + num(q) + ") {");
       o.ind++;
     }
+    const std::string slast = "s" + num(L.seq.size() - 1);
     for (size_t k = 0; k < L.loads.size(); k++) {
       const Affine& a = L.loads[k];
       int64_t cv = C(a, 0);
       std::string off = "(" + affine(a, its) + seq_terms(a) + ")";
       std::string nm = "L" + num(k);
       std::string dt = dtn(dd.t[a.tensor].dtype);
+      int fd = rec && k < L.fwd_dist.size() ? L.fwd_dist[k] : 0;
       if (cv == 0) {
-        o.l("const float " + nm + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
-      } else if (cv == 1 && !tail && L.load_cb[k]) {
-        o.l("float " + nm + "[" + num(W) + "];");
+        std::string ld = "fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ")";
+        if (fd) o.l("const float " + nm + " = (" + slast + " >= " + num(fd) + "u) ? H" + num(fd) + "[0] : " + ld + ";");
+        else o.l("const float " + nm + " = " + ld + ";");
+        continue;
+      }
+      o.l("float " + nm + "[" + num(W) + "];");
+      if (fd) {
+        o.l("if (" + slast + " >= " + num(fd) + "u) {");
+        o.l("  #pragma unroll");
+        o.l("  for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = H" + num(fd) + "[e];");
+        o.l("} else {");
+        o.ind++;
+      }
+      if (cv == 1 && !tail && L.load_cb[k]) {
         o.l("fop::vload<" + dt + ", " + num(W) + ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + nm + ", " +
             ptr(a.tensor, off) + ");");
       } else {
-        o.l("float " + nm + "[" + num(W) + "];");
         o.l("#pragma unroll");
         o.l("for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = " + (tail ? "(iv + e < " + num(EV) + "u) ? " : "") +
             "fop::sload<" + dt + ", " + pol(a, false) + ">(" + ptr(a.tensor, off + " + e * " + num(cv)) + ")" +
             (tail ? " : 0.f" : "") + ";");
+      }
+      if (fd) {
+        o.ind--;
+        o.l("}");
       }
     }
     DagCtx c;
@@ -719,18 +763,21 @@ struct Gen {
       o.l("fop::upk(" + v + ", R[2 * " + p + "], R[2 * " + p + " + 1]);");
     };
     emit_elems(o, x, var, c, W, sk);
-    o.l("#pragma unroll");
-    o.l("for (int e = 0; e < " + num(W) + "; ++e) ACC[e] = fop::round_to<" + dto + ">(R[e]);   // the stored value");
+    if (rec) {
+      store_vals("(" + woff + seq_terms(x.write) + ")", "R");
+      for (int q = maxd; q >= 2; q--)
+        o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) H" + num(q) + "[e] = H" + num(q - 1) + "[e];");
+      if (maxd >= 1)
+        o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) H1[e] = fop::round_to<" + dto + ">(R[e]);   // the stored value");
+    } else {
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) ACC[e] = fop::round_to<" + dto + ">(R[e]);   // the stored value");
+    }
     for (size_t q = 0; q < L.seq.size(); q++) {
       o.ind--;
       o.l("}");
     }
-    if (cw == 1 && !tail && L.store_cb[0])
-      o.l("fop::vstore<" + dto + ", " + num(W) + ", " + num(L.store_cb[0]) + ", fop::ST_DEFAULT>(" +
-          ptr(x.write.tensor, woff) + ", ACC);");
-    else
-      o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) " + guard + "fop::sstore<" + dto + ">(" +
-          ptr(x.write.tensor, woff + " + e * " + num(cw)) + ", ACC[e]);");
+    if (!rec) store_vals(woff, "ACC");
     o.ind--;
     o.l("}");
     footer();

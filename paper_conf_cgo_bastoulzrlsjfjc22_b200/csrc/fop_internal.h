@@ -51,6 +51,23 @@ struct Scenarios {
 };
 Scenarios rank_scenarios(const fop_desc& d, int s, const fop_plan_opts& o);
 
+// ---------------------------------------------------------------- N3
+// A dependence of a statement on itself (validity): a distance
+// vector over global loop ids, lexicographically positive in the statement's
+// original loop order.  Statements here have uniform dependences only: a
+// read of the target at a constant offset from the write (a recurrence), or
+// the write-write pairs of a read-modify-write over the loops the target
+// ignores (Fig. 2's Y over k).
+struct Dep {
+  int64_t dist[FOP_MAX_LOOPS] = {0};
+  bool anti = false;   // the read happens before the write (else flow / output)
+};
+std::vector<Dep> self_dependences(const fop_desc& d, int s);
+// Permutation-only legality of the schedule "parallel loops (threads) /
+// seq loops in the given order (each thread) / vector loop" for deps.
+bool schedule_legal(const std::vector<Dep>& deps, const std::vector<int>& seq, int vec_loop, int nloops,
+                    const int* loops);
+
 // ---------------------------------------------------------------- a5/a7
 enum XOp {  // expanded DAG node kinds (fop_opcode values + internal ones)
   X_FWD = 100,     // value of an earlier ASSIGN statement of the same launch (registers)
@@ -101,7 +118,13 @@ struct Launch {
   int trans_load = -1;            // TRANSPOSE: index into loads of the transposed access
   int coal_loop = -1;
   std::vector<int> order;         // launch loop order, innermost first (before collapse)
-  std::vector<int> seq;           // EW read-modify-write: loops walked in order by each thread (outer first)
+  std::vector<int> seq;           // EW read-modify-write / recurrence: loops walked in order by each thread (outer first)
+  bool rec = false;               // recurrence: the target depends on every seq loop (stored every iteration)
+  bool force_w1 = false;          // no influence scenario feasible: no explicit vector type (width 1)
+  std::vector<int> fwd_dist;      // recurrence: per load, iterations back along the last seq loop (0 = memory)
+  bool virt_vec = false;          // no dependence-free loop: vec_loop is a placeholder of extent 1
+  int scen_pick = 0;              // N3: scenario whose innermost loop carries the vector type (-1: none feasible)
+  int fallback = 0;               // N3: 0 scenario as ranked, 1 looser (vector constraint only), 2 no influence, 3 fully sequential
   std::vector<std::pair<std::string, int>> knobs;   // geometry overrides of this variant (auto-tuning)
   std::string name_suffix;        // kernel name suffix of a tuning variant
   std::vector<KLoop> kl;          // kernel loops (see geometry.cpp for the per-class layout)
@@ -146,6 +169,7 @@ struct Plan {
   fop_desc desc;
   fop_plan_opts opts;
   Scenarios scen[FOP_MAX_STMTS];
+  std::vector<Dep> deps[FOP_MAX_STMTS];
   std::vector<Launch> launches;
   std::vector<int64_t> temp_off;  // per tensor: workspace byte offset (-1 = not materialised)
   size_t ws_bytes = 0;

@@ -193,6 +193,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     if (L.kclass == FOP_CLASS_EW) {
       L.kl.clear();
       collapse_into(p, acc, ord, L.kl);
+      if (L.virt_vec) L.kl[0].extent = 1;   // fully sequential statement (row N3)
     } else {
       collapse_into(p, acc, seg1, L.kl);
     }
@@ -228,7 +229,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     }
   int W = any_vec ? std::max(1, o.max_vec_bytes / min_es) : 1;
   if (o.force_width > 0) W = std::min(W, pow2_floor(o.force_width));
-  if (L.scalar_variant) W = 1;
+  if (L.scalar_variant || L.force_w1) W = 1;
   int64_t EV = L.kl[0].extent;
   bool tail_ok = L.kclass == FOP_CLASS_EW && L.kl.size() == 1;
   if (tail_ok) {

@@ -222,7 +222,10 @@ struct Group {
   int kclass = FOP_CLASS_EW;
   int vec = -1;
   bool has_reduce = false;
-  bool closed = false;   // a read-modify-write launch: nothing joins it
+  bool closed = false;   // a read-modify-write / recurrence launch: nothing joins it
+  std::vector<int> seq;  // closed: loops carrying the statement's dependences, outer first
+  bool rec = false;
+  int scen_pick = 0, fallback = 0, coal = -1;
 };
 
 // read-modify-write ASSIGN (Fig. 2's Y): some loop of extent > 1 leaves the target index unchanged
@@ -245,6 +248,99 @@ uint32_t red_loops(const fop_desc& d, int s) {
 }
 
 }  // namespace
+
+// ======================================================================== N3
+
+std::vector<Dep> self_dependences(const fop_desc& d, int s) {
+  const fop_stmt& st = d.s[s];
+  std::vector<Dep> out;
+  if (st.kind != FOP_ASSIGN) return out;
+  auto lex_positive = [&](const Dep& D) {
+    for (int k = 0; k < st.nloops; k++)
+      if (D.dist[st.loop[k]] != 0) return D.dist[st.loop[k]] > 0;
+    return false;
+  };
+  auto push = [&](Dep D) {
+    for (const Dep& e : out)
+      if (std::memcmp(e.dist, D.dist, sizeof D.dist) == 0 && e.anti == D.anti) return;
+    out.push_back(D);
+  };
+  const fop_access& w = st.acc[0];
+  if (is_rmw(d, s)) {
+    // Fig. 2's Y: the target element is rewritten at every iteration of the
+    // loops it ignores, so every lexicographically positive vector over those
+    // loops is a dependence; e_i (carried by ignored loop i) and e_i - e_j
+    // (i before j) represent them for a permutation test.
+    Affine wa = affine_of(d, w);
+    std::vector<int> ign;
+    for (int k = 0; k < st.nloops; k++)
+      if (wa.coef[st.loop[k]] == 0 && d.extent[st.loop[k]] > 1) ign.push_back(st.loop[k]);
+    for (size_t i = 0; i < ign.size(); i++) {
+      Dep D;
+      D.dist[ign[i]] = 1;
+      push(D);
+    }
+    for (size_t i = 0; i < ign.size(); i++)
+      for (size_t j = i + 1; j < ign.size(); j++) {
+        Dep D;
+        D.dist[ign[i]] = 1;
+        D.dist[ign[j]] = -1;
+        push(D);
+      }
+    return out;
+  }
+  const fop_tensor& t = d.t[w.tensor];
+  for (int a = 1; a < st.nacc; a++) {
+    const fop_access& r = st.acc[a];
+    if (r.tensor != w.tensor) continue;
+    // written at iteration I, read at J: J_l = I_l + (w.offset - r.offset) on
+    // the loop of every tensor dim (validate() guarantees the same loop map)
+    Dep D;
+    bool meets = true;
+    for (int q = 0; q < t.rank; q++) {
+      if (w.loop[q] < 0) {
+        if (w.offset[q] != r.offset[q]) meets = false;   // constant dims never coincide
+        continue;
+      }
+      D.dist[w.loop[q]] = w.offset[q] - r.offset[q];
+    }
+    bool zero = true;
+    for (int l = 0; l < FOP_MAX_LOOPS; l++)
+      if (D.dist[l] != 0) {
+        zero = false;
+        if (D.dist[l] >= d.extent[l] || -D.dist[l] >= d.extent[l]) meets = false;  // no pair inside the domain
+      }
+    if (!meets || zero) continue;
+    if (!lex_positive(D)) {   // the read comes first: anti dependence from the read to the write
+      for (int l = 0; l < FOP_MAX_LOOPS; l++) D.dist[l] = -D.dist[l];
+      D.anti = true;
+    }
+    push(D);
+  }
+  return out;
+}
+
+bool schedule_legal(const std::vector<Dep>& deps, const std::vector<int>& seq, int vec_loop, int nloops,
+                    const int* loops) {
+  for (const Dep& D : deps) {
+    // parallel loops (threads, and the vector lanes) must not carry anything
+    for (int k = 0; k < nloops; k++) {
+      int l = loops[k];
+      bool in_seq = std::find(seq.begin(), seq.end(), l) != seq.end();
+      if (!in_seq && D.dist[l] != 0) return false;
+    }
+    (void)vec_loop;
+    // and each thread's sequential order must keep the source first
+    int first = 0;
+    for (int l : seq)
+      if (D.dist[l] != 0) {
+        first = D.dist[l] > 0 ? 1 : -1;
+        break;
+      }
+    if (first <= 0) return false;
+  }
+  return true;
+}
 
 // Expand statement s's DAG for a launch: inlined producers are substituted,
 // values of earlier statements in the same launch are forwarded.
@@ -317,26 +413,79 @@ void plan_launches(Plan& p) {
     bool is_red = st.kind == FOP_REDUCE;
     bool row = is_red && (red_loops(d, s) >> v & 1u);
     bool joined = false;
-    bool rmw = is_rmw(d, s);
-    if (rmw) {
-      // the vector loop must be one the target depends on (each thread owns W
-      // target elements); take the best-ranked scenario whose innermost loop
-      // is such a loop — the fallback order of the scenario list
-      Affine w = affine_of(d, st.acc[0]);
-      const Scenarios& sc = p.scen[s];
-      int pick = -1;
-      for (int k = 0; k < sc.nscen && pick < 0; k++) {
-        int l = sc.loops[k][sc.len[k] - 1];
-        if (w.coef[l] != 0) pick = l;
-      }
-      if (pick < 0)
-        for (int k = st.nloops - 1; k >= 0 && pick < 0; k--)
-          if (w.coef[st.loop[k]] != 0) pick = st.loop[k];
+    p.deps[s] = self_dependences(d, s);
+    if (!p.deps[s].empty()) {
+      // Row N3: the influence tree restricted to permutation
+      // schedules whose loop nest, seen from one thread, is
+      //     [parallel loops (threads; the coalescing loop innermost),
+      //      dependence-carrying loops in a legal order, d_v (vector lanes)].
+      // Siblings are the ranked scenarios.  Depth 0 of a scenario is
+      // the vector loop: feasible when it carries no dependence (a parallel
+      // dimension has zero dependence distance).  Deeper levels
+      // must be the innermost sequential loops (any order the permutation
+      // test accepts), then parallel loops; a scenario failing there keeps
+      // only its vector constraint (the lower-priority looser variant).
+      // With no feasible scenario the schedule is the uninfluenced one (P:202,
+      // P:289): original order, no explicit vector type.
+      const std::vector<Dep>& deps = p.deps[s];
+      uint32_t carried = 0;
+      for (const Dep& D : deps)
+        for (int l = 0; l < FOP_MAX_LOOPS; l++)
+          if (D.dist[l] != 0) carried |= 1u << l;
       Group g;
       g.stmts.push_back(s);
-      g.vec = pick;
       g.kclass = FOP_CLASS_EW;
       g.closed = true;
+      g.rec = !is_rmw(d, s);
+      std::vector<int> seq0;   // carrying loops, original order (always legal)
+      for (int k = 0; k < st.nloops; k++)
+        if (carried >> st.loop[k] & 1u) seq0.push_back(st.loop[k]);
+      const Scenarios& sc = p.scen[s];
+      g.scen_pick = -1;
+      for (int k = 0; k < sc.nscen && g.scen_pick < 0; k++) {
+        const int m = sc.len[k];
+        int vl = sc.loops[k][m - 1];
+        if (carried >> vl & 1u) continue;                 // depth 0 infeasible: next sibling
+        std::vector<int> inner;                           // scenario-fixed sequential loops, innermost first
+        bool full = true;
+        int coal = -1;
+        for (int q = m - 2; q >= 0 && full; q--) {
+          int l = sc.loops[k][q];
+          bool cl = carried >> l & 1u;
+          if (inner.size() < seq0.size()) {
+            if (cl) inner.push_back(l);
+            else full = false;                            // a parallel loop cannot sit inside a sequential one
+          } else if (cl) {
+            full = false;
+          } else if (coal < 0) {
+            coal = l;
+          }
+        }
+        std::vector<int> order;
+        for (int l : seq0)
+          if (std::find(inner.begin(), inner.end(), l) == inner.end()) order.push_back(l);
+        for (auto it = inner.rbegin(); it != inner.rend(); ++it) order.push_back(*it);
+        if (!full || !schedule_legal(deps, order, vl, st.nloops, st.loop)) {
+          full = false;                                   // looser variant: vector constraint only
+          order = seq0;
+          coal = -1;
+          for (int q = m - 2; q >= 0 && coal < 0; q--)
+            if (!(carried >> sc.loops[k][q] & 1u)) coal = sc.loops[k][q];
+        }
+        if (!schedule_legal(deps, order, vl, st.nloops, st.loop)) continue;
+        g.vec = vl;
+        g.seq = order;
+        g.coal = coal;
+        g.scen_pick = k;
+        g.fallback = full ? 0 : 1;
+      }
+      if (g.scen_pick < 0) {
+        g.seq = seq0;
+        g.vec = -1;
+        for (int k = st.nloops - 1; k >= 0 && g.vec < 0; k--)
+          if (!(carried >> st.loop[k] & 1u)) g.vec = st.loop[k];
+        g.fallback = g.vec >= 0 ? 2 : 3;
+      }
       groups.push_back(g);
       continue;
     }
@@ -459,16 +608,52 @@ void plan_launches(Plan& p) {
     // coalescing loop: next loop of the main scenario (goal (ii))
     const Scenarios& sc = p.scen[L.main_stmt];
     L.coal_loop = sc.len[0] >= 2 ? sc.loops[0][sc.len[0] - 2] : -1;
-    if (g.closed) {  // read-modify-write: loops the target ignores run in order inside each thread
+    if (g.closed) {  // read-modify-write / recurrence: dependence-carrying loops run in order inside each thread
       L.kclass = FOP_CLASS_EW;
       L.read_loop = -1;
       L.trans_load = -1;
+      L.seq = g.seq;
+      L.rec = g.rec;
+      L.scen_pick = g.scen_pick;
+      L.fallback = g.fallback;
+      L.force_w1 = g.fallback >= 2;
+      L.coal_loop = g.coal;
       const fop_stmt& st = d.s[L.main_stmt];
-      for (int k = 0; k < st.nloops; k++)
-        if (L.stmts[0].write.coef[st.loop[k]] == 0) L.seq.push_back(st.loop[k]);
-      L.coal_loop = -1;
-      for (int q = sc.len[0] - 2; q >= 0 && L.coal_loop < 0; q--)
-        if (L.stmts[0].write.coef[sc.loops[0][q]] != 0) L.coal_loop = sc.loops[0][q];
+      if (g.vec < 0) {
+        // fully sequential: a placeholder vector loop of extent 1 (an id the
+        // statement does not use, so every access has coefficient 0 on it)
+        for (int id = 0; id < FOP_MAX_LOOPS && L.vec_loop < 0; id++) {
+          bool used = false;
+          for (int k = 0; k < st.nloops; k++) used |= st.loop[k] == id;
+          if (!used) L.vec_loop = id;
+        }
+        if (L.vec_loop < 0) fail(FOP_E_UNSUPPORTED, "fully sequential statement over 8 loops");
+        L.virt_vec = true;
+      }
+      if (L.rec) {
+        // reads of the target 1..4 iterations back along the innermost
+        // sequential loop come from registers (this thread's last stores)
+        L.fwd_dist.assign(L.loads.size(), 0);
+        const fop_access& w = st.acc[0];
+        const fop_tensor& t = d.t[w.tensor];
+        int sl = g.seq.back();
+        for (int a = 1; a < st.nacc; a++) {
+          const fop_access& r = st.acc[a];
+          if (r.tensor != w.tensor) continue;
+          int64_t dist[FOP_MAX_LOOPS] = {0};
+          bool ok = true;
+          for (int q = 0; q < t.rank; q++) {
+            if (w.loop[q] < 0) ok = ok && w.offset[q] == r.offset[q];
+            else dist[w.loop[q]] = w.offset[q] - r.offset[q];
+          }
+          for (int l = 0; l < FOP_MAX_LOOPS; l++)
+            if (l != sl && dist[l] != 0) ok = false;
+          if (!ok || dist[sl] < 1 || dist[sl] > 4) continue;
+          Affine f = affine_of(d, r);
+          for (size_t k = 0; k < L.loads.size(); k++)
+            if (L.loads[k].same(f)) L.fwd_dist[k] = (int)dist[sl];
+        }
+      }
     }
     p.launches.push_back(L);
   }

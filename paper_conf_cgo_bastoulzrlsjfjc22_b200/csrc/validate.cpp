@@ -159,6 +159,18 @@ void validate(const fop_desc& d) {
           fail(FOP_E_UNSUPPORTED, where(s) + "read-modify-write statement reads its target at another index");
       if (wt.dtype == FOP_I32) fail(FOP_E_UNSUPPORTED, where(s) + "i32 read-modify-write");
     }
+    if (st.kind == FOP_ASSIGN && injective) {
+      // A read of the target at another index makes the statement a
+      // recurrence (row N3): supported when the dependence is uniform — the
+      // read maps every tensor dim to the same loop as the write, so the
+      // distance vector is the constant offset difference.
+      for (int a = 1; a < st.nacc; a++) {
+        if (st.acc[a].tensor != st.acc[0].tensor) continue;
+        for (int r = 0; r < wt.rank; r++)
+          if (st.acc[a].loop[r] != st.acc[0].loop[r])
+            fail(FOP_E_UNSUPPORTED, where(s) + "reads its target through another index map (non-uniform dependence)");
+      }
+    }
     if (st.kind == FOP_REDUCE && !has_red)
       fail(FOP_E_UNSUPPORTED, where(s) + "REDUCE statement without a reduction loop (use ASSIGN)");
 

@@ -21,7 +21,7 @@ if not os.path.exists(LIB_PATH):
 _lib = C.CDLL(LIB_PATH)
 
 MAX_RANK, MAX_LOOPS, MAX_TENSORS, MAX_STMTS = 8, 8, 16, 8
-MAX_ACC, MAX_NODES, MAX_FIN, MAX_LAUNCH, MAX_SCEN = 8, 48, 8, 8, 8
+MAX_ACC, MAX_NODES, MAX_FIN, MAX_LAUNCH, MAX_SCEN, MAX_DEPS = 8, 48, 8, 8, 8, 16
 
 DTYPE = {"f32": 0, "f16": 1, "bf16": 2, "i32": 3}
 ROLE = {"in": 1, "out": 2, "inout": 3, "temp": 4}
@@ -73,7 +73,8 @@ class LaunchInfo(C.Structure):
     _fields_ = [("kernel_class", C.c_int32), ("main_stmt", C.c_int32), ("stmt_mask", C.c_uint32),
                 ("vec_loop", C.c_int32), ("width", C.c_int32), ("read_loop", C.c_int32),
                 ("read_width", C.c_int32), ("coal_loop", C.c_int32), ("grid", C.c_int64),
-                ("block", C.c_int32), ("_pad", C.c_int32)]
+                ("block", C.c_int32), ("nseq", C.c_int32), ("seq", C.c_int32 * MAX_LOOPS),
+                ("scen_pick", C.c_int32), ("fallback", C.c_int32)]
 
 
 class PlanInfo(C.Structure):
@@ -82,10 +83,16 @@ class PlanInfo(C.Structure):
                 ("scenario", ((C.c_int32 * 3) * MAX_SCEN) * MAX_STMTS),
                 ("inner_score", (C.c_double * MAX_LOOPS) * MAX_STMTS),
                 ("nlaunch", C.c_int32), ("launch", LaunchInfo * MAX_LAUNCH),
-                ("workspace_bytes", C.c_size_t)]
+                ("workspace_bytes", C.c_size_t), ("ndeps", C.c_int32 * MAX_STMTS),
+                ("dep", ((C.c_int64 * MAX_LOOPS) * MAX_DEPS) * MAX_STMTS),
+                ("dep_anti", (C.c_int32 * MAX_DEPS) * MAX_STMTS)]
 
 
 _lib.fop_abi_version.restype = C.c_int
+ABI_VERSION = 2   # the struct layouts above mirror include/fop.h at this version
+if _lib.fop_abi_version() != ABI_VERSION:
+    raise ImportError(f"{LIB_PATH}: ABI version {_lib.fop_abi_version()} != binding {ABI_VERSION}; rebuild "
+                      "with python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build")
 _lib.fop_plan_opts_default.argtypes = [C.POINTER(PlanOpts)]
 _lib.fop_plan.argtypes = [C.POINTER(Desc), C.POINTER(PlanOpts), C.POINTER(C.c_void_p)]
 _lib.fop_plan.restype = C.c_int
@@ -267,6 +274,10 @@ class FusedOp:
                 "scenarios": [[ln(pi.scenario[s][k][q]) for q in range(pi.scen_len[s][k])]
                               for k in range(pi.nscen[s])],
                 "inner_score": {sl[k]: pi.inner_score[s][k] for k in range(len(sl))},
+                # uniform self-dependences (distance by loop name, lexicographically positive)
+                "deps": [{"dist": {self.loops[l]: pi.dep[s][k][l] for l in range(len(self.loops))
+                                   if pi.dep[s][k][l] != 0},
+                          "anti": bool(pi.dep_anti[s][k])} for k in range(pi.ndeps[s])],
             })
         launches = []
         for i in range(pi.nlaunch):
@@ -275,7 +286,9 @@ class FusedOp:
                              "stmts": [s for s in range(8) if li.stmt_mask >> s & 1],
                              "vec_loop": ln(li.vec_loop), "width": li.width,
                              "read_loop": ln(li.read_loop), "read_width": li.read_width,
-                             "coal_loop": ln(li.coal_loop), "grid": li.grid, "block": li.block})
+                             "coal_loop": ln(li.coal_loop), "grid": li.grid, "block": li.block,
+                             "seq": [ln(li.seq[q]) for q in range(li.nseq)],
+                             "scen_pick": li.scen_pick, "fallback": li.fallback})
         return {"stmts": stmts, "launches": launches, "workspace_bytes": pi.workspace_bytes}
 
     @property
