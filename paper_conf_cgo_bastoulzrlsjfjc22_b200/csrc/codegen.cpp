@@ -705,20 +705,130 @@ struct Gen {
       o.l("float H" + num(q) + "[" + num(W) + "];   // stored value " + num(q) + " iteration(s) back");
       o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) H" + num(q) + "[e] = 0.f;");
     }
-    for (size_t q = 0; q < L.seq.size(); q++) {
+    const size_t nseq = L.seq.size();
+    const int sl = L.seq.back();
+    const int64_t EL = dd.extent[sl];
+    const std::string slast = "s" + num(nseq - 1);
+    // Loads that vary along the innermost sequential loop and do not touch the
+    // target are prefetched P iterations ahead into a per-slot register
+    // buffer (the loop is unrolled by P, so slots are static registers): a
+    // thread's sequential chain otherwise exposes one HBM round trip per
+    // iteration.  Raw words when the vector is word-granular.
+    const int P = L.seq_prefetch;
+    std::vector<int> pf(L.loads.size(), 0);   // 0: no, 1: float buffer, 2: raw words
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      const Affine& a = L.loads[k];
+      if (P <= 1 || a.tensor == x.write.tensor || a.coef[sl] == 0) continue;
+      int64_t cv = C(a, 0);
+      int eb = es(a.tensor);
+      pf[k] = (cv == 1 && !tail && L.load_cb[k] >= 4 && W * eb >= 4) ? 2 : 1;
+    }
+    auto words = [&](size_t k) { return W * es(L.loads[k].tensor) / 4; };
+    // the memory load of load k at the current iteration values into float dst[W] (or a scalar)
+    auto emit_load = [&](size_t k, const std::string& dst, const std::string& sexpr, bool decl) {
+      const Affine& a = L.loads[k];
+      int64_t cv = C(a, 0);
+      std::string off = "(" + affine(a, its) + seq_terms(a) + ")";
+      if (!sexpr.empty()) {   // the innermost sequential index replaced by sexpr
+        int64_t cs = a.coef[sl];
+        off = "(" + off + " + (" + sexpr + " - " + slast + ")" + (cs == 1 ? "" : " * " + num(cs)) + ")";
+      }
+      std::string dt = dtn(dd.t[a.tensor].dtype);
+      if (cv == 0) {
+        o.l(std::string(decl ? "float " : "") + dst + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" +
+            ptr(a.tensor, off) + ");");
+        return;
+      }
+      if (decl) o.l("float " + dst + "[" + num(W) + "];");
+      if (cv == 1 && !tail && L.load_cb[k]) {
+        o.l("fop::vload<" + dt + ", " + num(W) + ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + dst + ", " +
+            ptr(a.tensor, off) + ");");
+      } else {
+        o.l("#pragma unroll");
+        o.l("for (int e = 0; e < " + num(W) + "; ++e) " + dst + "[e] = " + (tail ? "(iv + e < " + num(EV) + "u) ? " : "") +
+            "fop::sload<" + dt + ", " + pol(a, false) + ">(" + ptr(a.tensor, off + " + e * " + num(cv)) + ")" +
+            (tail ? " : 0.f" : "") + ";");
+      }
+    };
+    auto emit_fill = [&](size_t k, const std::string& slot, const std::string& sexpr) {
+      const Affine& a = L.loads[k];
+      if (pf[k] == 2) {
+        std::string off = "(" + affine(a, its) + seq_terms(a) + ")";
+        int64_t cs = a.coef[sl];
+        off = "(" + off + " + (" + sexpr + " - " + slast + ")" + (cs == 1 ? "" : " * " + num(cs)) + ")";
+        o.l("fop::vload_words<" + std::string(dtn(dd.t[a.tensor].dtype)) + ", " + num(W) + ", " + num(L.load_cb[k]) +
+            ", " + pol(a, false) + ">(PB" + num(k) + "[" + slot + "], " + ptr(a.tensor, off) + ");");
+      } else {
+        emit_load(k, "PB" + num(k) + "[" + slot + "]", sexpr, false);
+      }
+    };
+    for (size_t q = 0; q + 1 < nseq; q++) {
       o.l("#pragma unroll 1");
       o.l("for (idx_t s" + num(q) + " = 0; s" + num(q) + " < " + num(dd.extent[L.seq[q]]) + "u; ++s" + num(q) + ") {");
       o.ind++;
     }
-    const std::string slast = "s" + num(L.seq.size() - 1);
+    bool any_pf = false;
+    for (int f : pf) any_pf |= f != 0;
+    if (any_pf) {
+      o.l("const idx_t " + slast + " = 0;   // prologue: iterations 0..P-1 of the innermost sequential loop");
+      for (size_t k = 0; k < L.loads.size(); k++) {
+        if (!pf[k]) continue;
+        bool sc = C(L.loads[k], 0) == 0;
+        if (pf[k] == 2) o.l("u32 PB" + num(k) + "[" + num(P) + "][" + num(words(k)) + "];");
+        else o.l("float PB" + num(k) + "[" + num(P) + "]" + (sc ? "" : "[" + num(W) + "]") + ";");
+      }
+      o.l("#pragma unroll");
+      o.l("for (int u = 0; u < " + num(P) + "; ++u) {");
+      o.ind++;
+      o.l("if ((idx_t)u < " + num(EL) + "u) {");
+      o.ind++;
+      for (size_t k = 0; k < L.loads.size(); k++)
+        if (pf[k]) emit_fill(k, "u", "(idx_t)u");
+      o.ind--;
+      o.l("}");
+      o.ind--;
+      o.l("}");
+      o.l("#pragma unroll 1");
+      o.l("for (idx_t sb_ = 0; sb_ < " + num(EL) + "u; sb_ += " + num(P) + "u) {");
+      o.ind++;
+      o.l("#pragma unroll");
+      o.l("for (int u = 0; u < " + num(P) + "; ++u) {");
+      o.ind++;
+      o.l("const idx_t " + slast + "_ = sb_ + (idx_t)u;");
+      o.l("if (" + slast + "_ >= " + num(EL) + "u) break;");
+      o.l("{");
+      o.ind++;
+      o.l("const idx_t " + slast + " = " + slast + "_;");
+    } else {
+      o.l("#pragma unroll 1");
+      o.l("for (idx_t " + slast + " = 0; " + slast + " < " + num(EL) + "u; ++" + slast + ") {");
+      o.ind++;
+    }
     for (size_t k = 0; k < L.loads.size(); k++) {
       const Affine& a = L.loads[k];
       int64_t cv = C(a, 0);
-      std::string off = "(" + affine(a, its) + seq_terms(a) + ")";
       std::string nm = "L" + num(k);
       std::string dt = dtn(dd.t[a.tensor].dtype);
       int fd = rec && k < L.fwd_dist.size() ? L.fwd_dist[k] : 0;
+      if (pf[k]) {   // take the prefetched slot, refill it P iterations ahead
+        if (pf[k] == 2) {
+          o.l("float " + nm + "[" + num(W) + "];");
+          o.l("fop::cvt_words<" + dt + ", " + num(W) + ">(" + nm + ", PB" + num(k) + "[u]);");
+        } else if (cv == 0) {
+          o.l("const float " + nm + " = PB" + num(k) + "[u];");
+        } else {
+          o.l("float " + nm + "[" + num(W) + "];");
+          o.l("#pragma unroll\nfor (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = PB" + num(k) + "[u][e];");
+        }
+        o.l("if (" + slast + " + " + num(P) + "u < " + num(EL) + "u) {");
+        o.ind++;
+        emit_fill(k, "u", slast + " + " + num(P) + "u");
+        o.ind--;
+        o.l("}");
+        continue;
+      }
       if (cv == 0) {
+        std::string off = "(" + affine(a, its) + seq_terms(a) + ")";
         std::string ld = "fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ")";
         if (fd) o.l("const float " + nm + " = (" + slast + " >= " + num(fd) + "u) ? H" + num(fd) + "[0] : " + ld + ";");
         else o.l("const float " + nm + " = " + ld + ";");
@@ -732,15 +842,7 @@ struct Gen {
         o.l("} else {");
         o.ind++;
       }
-      if (cv == 1 && !tail && L.load_cb[k]) {
-        o.l("fop::vload<" + dt + ", " + num(W) + ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + nm + ", " +
-            ptr(a.tensor, off) + ");");
-      } else {
-        o.l("#pragma unroll");
-        o.l("for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = " + (tail ? "(iv + e < " + num(EV) + "u) ? " : "") +
-            "fop::sload<" + dt + ", " + pol(a, false) + ">(" + ptr(a.tensor, off + " + e * " + num(cv)) + ")" +
-            (tail ? " : 0.f" : "") + ";");
-      }
+      emit_load(k, nm, "", false);
       if (fd) {
         o.ind--;
         o.l("}");
@@ -773,7 +875,16 @@ struct Gen {
       o.l("#pragma unroll");
       o.l("for (int e = 0; e < " + num(W) + "; ++e) ACC[e] = fop::round_to<" + dto + ">(R[e]);   // the stored value");
     }
-    for (size_t q = 0; q < L.seq.size(); q++) {
+    if (any_pf) {   // the unrolled block, the slot loop and the block loop
+      for (int q = 0; q < 3; q++) {
+        o.ind--;
+        o.l("}");
+      }
+    } else {
+      o.ind--;
+      o.l("}");
+    }
+    for (size_t q = 0; q + 1 < nseq; q++) {
       o.ind--;
       o.l("}");
     }

@@ -120,6 +120,7 @@ struct Launch {
   std::vector<int> order;         // launch loop order, innermost first (before collapse)
   std::vector<int> seq;           // EW read-modify-write / recurrence: loops walked in order by each thread (outer first)
   bool rec = false;               // recurrence: the target depends on every seq loop (stored every iteration)
+  int seq_prefetch = 1;           // sequential launches: iterations of target-independent loads kept in flight
   bool force_w1 = false;          // no influence scenario feasible: no explicit vector type (width 1)
   std::vector<int> fwd_dist;      // recurrence: per load, iterations back along the last seq loop (0 = memory)
   bool virt_vec = false;          // no dependence-free loop: vec_loop is a placeholder of extent 1

@@ -168,6 +168,8 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
   return v;
 }
 
+static int knob_w_cap(const Launch& L) { return geometry_knob(L, "FOP_SEQ_W", 1 << 20); }
+
 void finalize_launch_geometry(const Plan& p, Launch& L) {
   const fop_desc& d = p.desc;
   const fop_plan_opts& o = p.opts;
@@ -230,6 +232,15 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   int W = any_vec ? std::max(1, o.max_vec_bytes / min_es) : 1;
   if (o.force_width > 0) W = std::min(W, pow2_floor(o.force_width));
   if (L.scalar_variant || L.force_w1) W = 1;
+  if (!L.seq.empty() && any_vec) {
+    // sequential launches get one thread per W lanes and nothing else to hide
+    // latency with: narrow the vectors (down to 4-byte accesses) until the
+    // lanes cover ~128 threads per SM
+    int64_t lanes = 1;
+    for (const auto& k : L.kl) lanes *= k.extent;
+    while (W > 1 && W * min_es > 4 && lanes / W < (int64_t)sms * 128) W /= 2;
+    W = std::min(W, knob_w_cap(L));
+  }
   int64_t EV = L.kl[0].extent;
   bool tail_ok = L.kclass == FOP_CLASS_EW && L.kl.size() == 1;
   if (tail_ok) {
@@ -301,8 +312,27 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     int u = bytes > 0 ? std::max(1, std::min(8, pow2_floor(std::max(1, 128 / bytes)))) : 4;
     L.unroll = L.seq.empty() ? knob("FOP_EW_U", u) : 1;   // RMW: one target vector per thread
     L.minblocks = knob("FOP_EW_MINB", L.unroll >= 4 ? 2 : 3);
-    int64_t need = (L.work + (int64_t)L.block * L.unroll - 1) / ((int64_t)L.block * L.unroll);
-    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
+    if (!L.seq.empty()) {
+      // one pass over the lanes (a second grid-stride pass would double the
+      // sequential chain); small blocks spread the lanes over every SM; the
+      // target-independent loads of the innermost sequential loop are kept
+      // P iterations ahead (512 B per thread, <= 128 registers; measured on a
+      // [64,512,768] f16 time scan: P=16 3.3 TB/s, 64 4.8 TB/s, 128 5.2 TB/s)
+      int pbytes = 0;
+      const int sl = L.seq.back();
+      for (const auto& a : L.loads)
+        if (a.tensor != L.stmts[0].write.tensor && a.coef[sl] != 0)
+          pbytes += (coef(L, a, 0) != 0 ? W : 1) * esize(d.t[a.tensor].dtype);
+      int P = pbytes ? std::max(2, std::min(128, pow2_floor(std::max(1, 512 / pbytes)))) : 1;
+      L.seq_prefetch = knob("FOP_SEQ_P", P);
+      L.block = knob("FOP_BLOCK", L.work >= (int64_t)sms * 256 ? 256 : (L.work >= (int64_t)sms * 128 ? 128 : 64));
+      int64_t need = (L.work + L.block - 1) / L.block;
+      L.minblocks = knob("FOP_EW_MINB", (int)std::max<int64_t>(1, std::min<int64_t>(8, (need + sms - 1) / sms)));
+      L.grid = std::max<int64_t>(1, need);
+    } else {
+      int64_t need = (L.work + (int64_t)L.block * L.unroll - 1) / ((int64_t)L.block * L.unroll);
+      L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
+    }
   } else if (L.kclass == FOP_CLASS_TRANSPOSE) {
     for (size_t k = 2; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
     int64_t ntv = EV / W, ntr = L.kl[1].extent / L.read_width;

@@ -65,7 +65,7 @@ def test_fig2_plan_is_fig2c():
     li = op.info()["launches"]
     assert len(li) == 1 and li[0]["stmts"] == [1] and li[0]["vec_loop"] == "j"
     src = op.source(0)
-    assert "for (idx_t s0 = 0; s0 < 64u; ++s0)" in src      # the in-order k loop
+    assert "for (idx_t sb_ = 0; sb_ < 64u; sb_ += " in src   # the in-order k loop (blocks of prefetched iterations)
     # a read of the RMW target at another index is not supported (would need a dependence test)
     d = W.fig2_running_example(16)
     d["stmts"][1]["reads"][0] = ("C", ["j", "i"])

@@ -275,5 +275,6 @@ def test_scan_time_bert_size_f16():
     x = W.make_inputs(d)
     got, op = run_gpu(d, x)
     li = op.info()["launches"][0]
-    assert li["vec_loop"] == "h" and li["width"] == 8 and li["seq"] == ["t"]
+    # 49152 lanes: vectors narrowed to 4 bytes so the lanes cover the SMs
+    assert li["vec_loop"] == "h" and li["width"] == 2 and li["seq"] == ["t"]
     assert_bitexact(got["Y"], O.run(d, x)["Y"], "Y")
