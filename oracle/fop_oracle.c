@@ -212,6 +212,8 @@ static int check_ref(const orc_ref *r, const orc_statement *st, int narrays, con
                      const long long *ext, int s, char *err, int errlen) {
   if (r->array < 0 || r->array >= narrays) return fail(err, errlen, "bad array index", s);
   const orc_array *a = &arrays[r->array];
+  for (int k = 0; k < st->nloops; k++)
+    if (ext[st->loops[k]] == 0) return 0; /* empty domain: the access never happens */
   for (int d = 0; d < a->rank; d++) {
     long long lo = r->off[d], hi = r->off[d];
     if (r->iter[d] >= 0) {
@@ -332,7 +334,7 @@ int orc_run(int nloops, const long long *extents, int narrays, orc_array *arrays
             int nstatements, const orc_statement *statements, char *err, int errlen) {
   if (nloops < 0 || nloops > ORC_LOOPS) return fail(err, errlen, "bad loop count", -1);
   for (int l = 0; l < nloops; l++)
-    if (extents[l] < 1) return fail(err, errlen, "loop extent < 1", -1);
+    if (extents[l] < 0) return fail(err, errlen, "loop extent < 0", -1);  /* 0: empty box domain */
   for (int s = 0; s < nstatements; s++) {
     const orc_statement *st = &statements[s];
     if (st->nloops < 1 || st->nloops > ORC_LOOPS) return fail(err, errlen, "bad statement loop count", s);

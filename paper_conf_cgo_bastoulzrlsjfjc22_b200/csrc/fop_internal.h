@@ -191,6 +191,7 @@ struct Plan {
 
 // validate.cpp
 void validate(const fop_desc& d);
+bool empty_domain(const fop_desc& d, const fop_stmt& st);   // some loop of the statement has extent 0
 // planner.cpp
 void plan_launches(Plan& p);
 void finalize_launch_geometry(const Plan& p, Launch& L);

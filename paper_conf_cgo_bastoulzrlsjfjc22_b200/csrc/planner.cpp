@@ -407,7 +407,7 @@ void plan_launches(Plan& p) {
   // ---- grouping (statement order; a group = one launch)
   std::vector<Group> groups;
   for (int s = 0; s < d.nstmts; s++) {
-    if (inl[s]) continue;
+    if (inl[s] || empty_domain(d, d.s[s])) continue;   // an empty domain executes nothing
     const fop_stmt& st = d.s[s];
     int v = innermost(p, s);
     bool is_red = st.kind == FOP_REDUCE;

@@ -125,7 +125,10 @@ CUcontext current_context(void* const* ptrs, int n) {
 
 int64_t span_bytes(const fop_tensor& t) {
   int64_t n = 1;
-  for (int r = 0; r < t.rank; r++) n += (t.shape[r] - 1) * t.stride[r];
+  for (int r = 0; r < t.rank; r++) {
+    if (t.shape[r] == 0) return 0;   // empty tensor
+    n += (t.shape[r] - 1) * t.stride[r];
+  }
   return n * esize(t.dtype);
 }
 
@@ -193,16 +196,20 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
   if (!c.ok) fail(FOP_E_CUDA, c.why);
   if (p.ws_bytes && !ws) fail(FOP_E_INVALID, "this plan needs a workspace of fop_plan_workspace_bytes() bytes");
   for (int t = 0; t < d.ntensors; t++) {
-    if (!ptrs[t] && d.t[t].role != FOP_TEMP) fail(FOP_E_INVALID, "NULL pointer for tensor " + std::to_string(t));
+    if (!ptrs[t] && d.t[t].role != FOP_TEMP && span_bytes(d.t[t]) > 0)
+      fail(FOP_E_INVALID, "NULL pointer for tensor " + std::to_string(t));
     if (ptrs[t] && ((uintptr_t)ptrs[t] % esize(d.t[t].dtype)))
       fail(FOP_E_ALIGN, "tensor " + std::to_string(t) + " is not aligned to its element size");
   }
+  bool any_copy = false;
+  for (int t = 0; t < d.ntensors && host_ptrs; t++) any_copy |= host_ptrs[t] && span_bytes(d.t[t]) > 0;
+  if (p.launches.empty() && !any_copy) return FOP_OK;   // every statement has an empty domain
   CUcontext ctx = current_context(ptrs, nptrs);
   CUstream st = (CUstream)stream;
 
   if (host_ptrs) {  // end-to-end: inputs host -> device
     for (int t = 0; t < d.ntensors; t++)
-      if ((d.t[t].role == FOP_IN || d.t[t].role == FOP_INOUT) && host_ptrs[t])
+      if ((d.t[t].role == FOP_IN || d.t[t].role == FOP_INOUT) && host_ptrs[t] && span_bytes(d.t[t]) > 0)
         check(c.h2d((CUdeviceptr)ptrs[t], host_ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyHtoDAsync");
   }
 
@@ -313,7 +320,7 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
 
   if (host_ptrs) {  // device -> host results
     for (int t = 0; t < d.ntensors; t++)
-      if ((d.t[t].role == FOP_OUT || d.t[t].role == FOP_INOUT) && host_ptrs[t])
+      if ((d.t[t].role == FOP_OUT || d.t[t].role == FOP_INOUT) && host_ptrs[t] && span_bytes(d.t[t]) > 0)
         check(c.d2h(host_ptrs[t], (CUdeviceptr)ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyDtoHAsync");
   }
   return FOP_OK;

@@ -32,9 +32,16 @@ static bool in_stmt(const fop_stmt& st, int loop) {
   return false;
 }
 
+bool empty_domain(const fop_desc& d, const fop_stmt& st) {
+  for (int k = 0; k < st.nloops; k++)
+    if (st.loop[k] >= 0 && st.loop[k] < FOP_MAX_LOOPS && d.extent[st.loop[k]] == 0) return true;
+  return false;
+}
+
 static void check_access(const fop_desc& d, const fop_stmt& st, const fop_access& a, int s) {
   if (a.tensor < 0 || a.tensor >= d.ntensors) fail(FOP_E_INVALID, where(s) + "access tensor out of range");
   const fop_tensor& t = d.t[a.tensor];
+  const bool empty = empty_domain(d, st);   // an empty box domain accesses nothing
   for (int r = 0; r < t.rank; r++) {
     int64_t lo = a.offset[r], hi = a.offset[r];
     if (a.loop[r] >= 0) {
@@ -44,7 +51,7 @@ static void check_access(const fop_desc& d, const fop_stmt& st, const fop_access
     } else if (a.loop[r] != -1) {
       fail(FOP_E_INVALID, where(s) + "access loop id must be >= 0 or -1");
     }
-    if (lo < 0 || hi >= t.shape[r])
+    if (!empty && (lo < 0 || hi >= t.shape[r]))
       fail(FOP_E_INVALID, where(s) + "access index range leaves the tensor (dim " + std::to_string(r) + ")");
   }
   for (int r = t.rank; r < FOP_MAX_RANK; r++)
@@ -83,7 +90,7 @@ static void check_dag(const fop_node* n, int nn, int nacc, bool fin, int s) {
 void validate(const fop_desc& d) {
   if (d.nloops < 1 || d.nloops > FOP_MAX_LOOPS) fail(FOP_E_INVALID, "nloops must be 1..8");
   for (int l = 0; l < d.nloops; l++)
-    if (d.extent[l] < 1) fail(FOP_E_INVALID, "loop " + std::to_string(l) + " has extent < 1");
+    if (d.extent[l] < 0) fail(FOP_E_INVALID, "loop " + std::to_string(l) + " has extent < 0");
   if (d.ntensors < 1 || d.ntensors > FOP_MAX_TENSORS) fail(FOP_E_INVALID, "ntensors must be 1..16");
   for (int i = 0; i < d.ntensors; i++) {
     const fop_tensor& t = d.t[i];
@@ -92,7 +99,7 @@ void validate(const fop_desc& d) {
     if (t.dtype < FOP_F32 || t.dtype > FOP_I32) fail(FOP_E_INVALID, w + "unknown dtype");
     if (t.role < FOP_IN || t.role > FOP_TEMP) fail(FOP_E_INVALID, w + "unknown role");
     for (int r = 0; r < t.rank; r++) {
-      if (t.shape[r] < 1) fail(FOP_E_INVALID, w + "shape must be >= 1");
+      if (t.shape[r] < 0) fail(FOP_E_INVALID, w + "shape must be >= 0");
       if (t.stride[r] < 0) fail(FOP_E_UNSUPPORTED, w + "negative strides are not supported");
     }
   }
@@ -126,7 +133,7 @@ void validate(const fop_desc& d) {
 
     // Write-injectivity of the target over the domain (a write-write
     // pair is a dependence; within one ASSIGN that is a read-modify-write
-    // over the missing loops, Fig. 2's Y — row N2, not built yet).
+    // over the missing loops, Fig. 2's Y — row N2).
     Affine w = affine_of(d, st.acc[0]);
     bool injective = true;   // no loop of extent > 1 leaves the target index unchanged
     bool has_red = false;    // some loop does not appear in the target index

@@ -143,6 +143,8 @@ def _strides(t):
 
 
 def span_elems(t):
+    if any(s == 0 for s in t["shape"]):
+        return 0
     return 1 + sum((s - 1) * k for s, k in zip(t["shape"], _strides(t)))
 
 
