@@ -249,6 +249,24 @@ FOP_API fop_status  fop_run(const fop_plan_t* plan, void* const* dev_ptrs, int32
 FOP_API fop_status  fop_run_host(const fop_plan_t* plan, void* const* host_ptrs,
                          void* const* dev_ptrs, int32_t nptrs, void* workspace, void* stream);
 
+/* End to end for n INDEPENDENT plans (no plan reads what another writes):
+ * plan k takes host_ptrs[k] / dev_ptrs[k] (nptrs[k] entries each, as in
+ * fop_run_host; a NULL host pointer skips that tensor's copy) and
+ * workspaces[k] (workspaces may be NULL when no plan needs one).  The copies
+ * are pipelined: inputs host->device in order on an internal copy stream,
+ * plan k runs on `stream` once its inputs are in, its outputs go
+ * device->host on a second internal copy stream while later inputs are still
+ * arriving (PCIe is full duplex).  Being independent, the plans run in the
+ * order that minimises the two-direction copy makespan (Johnson's rule for
+ * a two-machine flow shop; ties keep the given order).  The first copies wait for work already on
+ * `stream`; `stream` waits for the last copy, so the call is ordered like one
+ * fop_run_host on `stream`.  Asynchronous; the caller synchronises `stream`
+ * before reading host buffers.  Host buffers should be pinned.  The internal
+ * streams are created once per context and live for the process. */
+FOP_API fop_status  fop_run_host_many(const fop_plan_t* const* plans, void* const* const* host_ptrs,
+                                      void* const* const* dev_ptrs, const int32_t* nptrs,
+                                      void* const* workspaces, int32_t n, void* stream);
+
 /* The kernel fop_run launches for `launch` on the current CUDA context (after
  * auto-tuning; the default geometry before the first run): its name, grid and
  * block.  Pointers stay owned by the plan. */

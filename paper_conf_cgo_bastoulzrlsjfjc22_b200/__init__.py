@@ -9,7 +9,8 @@ The binding (and libfop.so) is loaded on first use of an exported name, so
 ``python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build`` works before the
 library exists.
 """
-_EXPORTS = ("FusedOp", "FopError", "abi_version", "marshal", "default_opts", "ABI_SYMBOLS", "LIB_PATH")
+_EXPORTS = ("FusedOp", "FopError", "abi_version", "marshal", "default_opts", "ABI_SYMBOLS", "LIB_PATH",
+            "run_host_many")
 
 __all__ = list(_EXPORTS)
 

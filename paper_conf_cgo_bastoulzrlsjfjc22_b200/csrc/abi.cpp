@@ -228,6 +228,20 @@ fop_status fop_run_host(const fop_plan_t* plan, void* const* host_ptrs, void* co
   });
 }
 
+fop_status fop_run_host_many(const fop_plan_t* const* plans, void* const* const* host_ptrs,
+                             void* const* const* dev_ptrs, const int32_t* nptrs, void* const* workspaces,
+                             int32_t n, void* stream) {
+  return guarded([&] {
+    if (n > 0 && (!plans || !host_ptrs || !dev_ptrs || !nptrs)) fop::fail(FOP_E_INVALID, "NULL argument");
+    std::vector<fop::Plan*> ps((size_t)std::max(0, n));
+    for (int k = 0; k < n; k++) {
+      if (!plans[k]) fop::fail(FOP_E_INVALID, "NULL plan at " + std::to_string(k));
+      ps[k] = &const_cast<fop_plan_t*>(plans[k])->p;
+    }
+    return fop::run_host_many(ps.data(), host_ptrs, dev_ptrs, nptrs, workspaces, n, stream);
+  });
+}
+
 fop_status fop_plan_selected(const fop_plan_t* plan, int32_t i, const char** name, int64_t* grid, int32_t* block) {
   return guarded([&] {
     if (!plan || !name || i < 0 || i >= (int)plan->p.launches.size()) fop::fail(FOP_E_INVALID, "bad launch index");

@@ -204,6 +204,8 @@ extern const char* kDeviceHeader;   // device/fop_device.cuh, embedded at build 
 void jit_compile(Launch& L);
 bool jit_available();
 // runtime.cpp
+fop_status run_host_many(Plan* const* plans, void* const* const* host_ptrs, void* const* const* dev_ptrs,
+                         const int32_t* nptrs, void* const* ws, int n, void* stream);
 fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream,
                     void* const* host_ptrs);
 void* current_context_or_null();   // the calling thread's CUDA context (nullptr without a driver)

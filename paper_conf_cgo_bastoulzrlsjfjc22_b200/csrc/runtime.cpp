@@ -7,6 +7,8 @@
 // stream; fop_run only enqueues: one kernel per launch of the plan.
 #include <dlfcn.h>
 
+#include <algorithm>
+
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -49,6 +51,8 @@ struct Cuda {
   CUresult (*ev_elapsed)(float*, void*, void*);
   CUresult (*ev_destroy)(void*);
   CUresult (*stream_capturing)(CUstream, int*);
+  CUresult (*stream_create)(CUstream*, unsigned);
+  CUresult (*stream_wait)(CUstream, void*, unsigned);
   CUresult (*tmap_encode)(void*, int, unsigned, void*, const uint64_t*, const uint64_t*, const unsigned*,
                           const unsigned*, int, int, int, int);
 };
@@ -88,6 +92,8 @@ Cuda& cuda() {
     SYM(ev_elapsed, "cuEventElapsedTime");
     SYM(ev_destroy, "cuEventDestroy_v2");
     SYM(stream_capturing, "cuStreamIsCapturing");
+    SYM(stream_create, "cuStreamCreate");
+    SYM(stream_wait, "cuStreamWaitEvent");
     SYM(tmap_encode, "cuTensorMapEncodeTiled");
 #undef SYM
     if (c.init(0) != 0) {
@@ -323,6 +329,117 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
       if ((d.t[t].role == FOP_OUT || d.t[t].role == FOP_INOUT) && host_ptrs[t] && span_bytes(d.t[t]) > 0)
         check(c.d2h(host_ptrs[t], (CUdeviceptr)ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyDtoHAsync");
   }
+  return FOP_OK;
+}
+
+// ---------------------------------------------------------------- host pipeline
+// fop_run_host_many: independent plans end to end from host buffers with the
+// copies pipelined over two internal streams per context (created once, kept
+// for the process): all inputs host->device in order on the first, each
+// plan's kernels on the caller's stream once its inputs are in, its outputs
+// device->host on the second while later inputs are still arriving.  The
+// first copies wait for prior work on the caller's stream (which may still
+// read the same device buffers) and the caller's stream waits for the last
+// copy, so calls stay ordered with everything else on that stream.
+namespace {
+struct CopyStreams {
+  CUcontext ctx = nullptr;
+  CUstream h2d = nullptr, d2h = nullptr;
+  std::vector<void*> ev;   // reusable (a wait captures the event's state when it is enqueued)
+};
+std::mutex g_cs_mu;
+std::vector<CopyStreams> g_cs;
+
+void* pool_event(CopyStreams& cs, size_t i) {
+  Cuda& c = cuda();
+  while (cs.ev.size() <= i) {
+    void* e = nullptr;
+    check(c.ev_create(&e, 2 /* CU_EVENT_DISABLE_TIMING */), "cuEventCreate");
+    cs.ev.push_back(e);
+  }
+  return cs.ev[i];
+}
+
+int64_t copy_bytes(const Plan& p, void* const* host_ptrs, bool inputs) {
+  int64_t b = 0;
+  for (int t = 0; t < p.desc.ntensors; t++) {
+    int r = p.desc.t[t].role;
+    bool sel = inputs ? (r == FOP_IN || r == FOP_INOUT) : (r == FOP_OUT || r == FOP_INOUT);
+    if (sel && host_ptrs[t]) b += span_bytes(p.desc.t[t]);
+  }
+  return b;
+}
+
+void copy_tensors(const Plan& p, void* const* ptrs, void* const* host_ptrs, CUstream st, bool inputs) {
+  Cuda& c = cuda();
+  const fop_desc& d = p.desc;
+  for (int t = 0; t < d.ntensors; t++) {
+    bool in = d.t[t].role == FOP_IN || d.t[t].role == FOP_INOUT;
+    bool out = d.t[t].role == FOP_OUT || d.t[t].role == FOP_INOUT;
+    if (!host_ptrs[t] || span_bytes(d.t[t]) == 0 || (inputs ? !in : !out)) continue;
+    if (inputs) check(c.h2d((CUdeviceptr)ptrs[t], host_ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyHtoDAsync");
+    else check(c.d2h(host_ptrs[t], (CUdeviceptr)ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyDtoHAsync");
+  }
+}
+}  // namespace
+
+fop_status run_host_many(Plan* const* plans, void* const* const* host_ptrs, void* const* const* dev_ptrs,
+                         const int32_t* nptrs, void* const* ws, int n, void* stream) {
+  Cuda& c = cuda();
+  if (!c.ok) fail(FOP_E_CUDA, c.why);
+  if (n <= 0) return FOP_OK;
+  for (int k = 0; k < n; k++)
+    if (!plans[k] || !host_ptrs[k] || !dev_ptrs[k]) fail(FOP_E_INVALID, "NULL plan or pointer table at " + std::to_string(k));
+  CUcontext ctx = current_context(dev_ptrs[0], nptrs[0]);
+  CUstream st = (CUstream)stream;
+  std::lock_guard<std::mutex> g(g_cs_mu);
+  CopyStreams* cs = nullptr;
+  for (auto& x : g_cs)
+    if (x.ctx == ctx) cs = &x;
+  if (!cs) {
+    CopyStreams x;
+    x.ctx = ctx;
+    check(c.stream_create(&x.h2d, 1 /* CU_STREAM_NON_BLOCKING */), "cuStreamCreate");
+    check(c.stream_create(&x.d2h, 1), "cuStreamCreate");
+    g_cs.push_back(x);
+    cs = &g_cs.back();
+  }
+  // Order: the plans are independent and the two copy directions are a
+  // two-machine flow shop, so Johnson's rule gives the shortest makespan:
+  // plans with fewer input than output bytes first (by input bytes,
+  // ascending), then the rest (by output bytes, descending); ties keep the
+  // caller's order.
+  std::vector<int> ord(n);
+  std::vector<int64_t> hin(n), hout(n);
+  for (int k = 0; k < n; k++) {
+    ord[k] = k;
+    hin[k] = copy_bytes(*plans[k], host_ptrs[k], true);
+    hout[k] = copy_bytes(*plans[k], host_ptrs[k], false);
+  }
+  std::stable_sort(ord.begin(), ord.end(), [&](int a, int b) {
+    bool fa = hin[a] < hout[a], fb = hin[b] < hout[b];
+    if (fa != fb) return fa;
+    return fa ? hin[a] < hin[b] : hout[a] > hout[b];
+  });
+  size_t ei = 0;
+  void* e0 = pool_event(*cs, ei++);
+  check(c.ev_record(e0, st), "cuEventRecord");
+  check(c.stream_wait(cs->h2d, e0, 0), "cuStreamWaitEvent");
+  check(c.stream_wait(cs->d2h, e0, 0), "cuStreamWaitEvent");
+  for (int k : ord) {
+    copy_tensors(*plans[k], dev_ptrs[k], host_ptrs[k], cs->h2d, true);
+    void* ein = pool_event(*cs, ei++);
+    check(c.ev_record(ein, cs->h2d), "cuEventRecord");
+    check(c.stream_wait(st, ein, 0), "cuStreamWaitEvent");
+    run_plan(*plans[k], dev_ptrs[k], nptrs[k], ws ? ws[k] : nullptr, stream, nullptr);
+    void* ek = pool_event(*cs, ei++);
+    check(c.ev_record(ek, st), "cuEventRecord");
+    check(c.stream_wait(cs->d2h, ek, 0), "cuStreamWaitEvent");
+    copy_tensors(*plans[k], dev_ptrs[k], host_ptrs[k], cs->d2h, false);
+  }
+  void* eout = pool_event(*cs, ei++);
+  check(c.ev_record(eout, cs->d2h), "cuEventRecord");
+  check(c.stream_wait(st, eout, 0), "cuStreamWaitEvent");
   return FOP_OK;
 }
 

@@ -109,6 +109,10 @@ _lib.fop_run.restype = C.c_int
 _lib.fop_run_host.argtypes = [C.c_void_p, C.POINTER(C.c_void_p), C.POINTER(C.c_void_p), C.c_int32,
                               C.c_void_p, C.c_void_p]
 _lib.fop_run_host.restype = C.c_int
+_lib.fop_run_host_many.argtypes = [C.POINTER(C.c_void_p), C.POINTER(C.POINTER(C.c_void_p)),
+                                   C.POINTER(C.POINTER(C.c_void_p)), C.POINTER(C.c_int32), C.POINTER(C.c_void_p),
+                                   C.c_int32, C.c_void_p]
+_lib.fop_run_host_many.restype = C.c_int
 _lib.fop_plan_selected.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_char_p), C.POINTER(C.c_int64),
                                    C.POINTER(C.c_int32)]
 _lib.fop_plan_selected.restype = C.c_int
@@ -118,7 +122,7 @@ _lib.fop_last_error.restype = C.c_char_p
 
 ABI_SYMBOLS = ["fop_abi_version", "fop_plan_opts_default", "fop_plan", "fop_plan_info_get",
                "fop_plan_workspace_bytes", "fop_plan_source", "fop_plan_cubin", "fop_run",
-               "fop_run_host", "fop_plan_selected", "fop_plan_destroy", "fop_status_str", "fop_last_error"]
+               "fop_run_host", "fop_run_host_many", "fop_plan_selected", "fop_plan_destroy", "fop_status_str", "fop_last_error"]
 
 
 class FopError(RuntimeError):
@@ -365,6 +369,43 @@ class FusedOp:
             stream = torch.cuda.current_stream(dev)
         _check(_lib.fop_run_host(self._h, harr, arr, len(self.names),
                                  None if ws is None else ws.data_ptr(), stream.cuda_stream))
+
+    def _host_ptrs(self, host):
+        harr = (C.c_void_p * len(self.names))()
+        for i, n in enumerate(self.names):
+            h = host.get(n)
+            harr[i] = None if h is None else h.data_ptr()
+        return harr
+
+
+def run_host_many(items, stream=None):
+    """End to end for independent operators with pipelined copies
+    (fop_run_host_many): `items` is a list of (FusedOp, host tensors,
+    device tensors[, workspace]); a tensor missing from `host` is not copied."""
+    import torch
+    n = len(items)
+    plans = (C.c_void_p * n)()
+    hp = (C.POINTER(C.c_void_p) * n)()
+    dp = (C.POINTER(C.c_void_p) * n)()
+    np_ = (C.c_int32 * n)()
+    ws = (C.c_void_p * n)()
+    keep = []
+    dev = None
+    for k, it in enumerate(items):
+        op, host, devt = it[0], it[1], it[2]
+        arr, d = op._ptrs(devt)
+        dev = dev or d
+        harr = op._host_ptrs(host)
+        w = it[3] if len(it) > 3 and it[3] is not None else op._workspace(d)
+        keep += [arr, harr]
+        plans[k] = op._h
+        hp[k] = C.cast(harr, C.POINTER(C.c_void_p))
+        dp[k] = C.cast(arr, C.POINTER(C.c_void_p))
+        np_[k] = len(op.names)
+        ws[k] = None if w is None else w.data_ptr()
+    if stream is None:
+        stream = torch.cuda.current_stream(dev)
+    _check(_lib.fop_run_host_many(plans, hp, dp, np_, ws, n, stream.cuda_stream))
 
 
 def abi_version():

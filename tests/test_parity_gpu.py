@@ -356,3 +356,38 @@ def test_run_host_end_to_end():
     op.run_host(host, dev)
     torch.cuda.synchronize()
     assert_bitexact(host["y"].numpy(), O.run(d, x)["y"], "y")
+
+
+def _host_dev(d, x):
+    """Pinned host buffers (inputs from x, outputs NaN-filled) + empty device buffers."""
+    outs = W.alloc_outputs(d)
+    host, dev = {}, {}
+    for n, t in d["tensors"].items():
+        if t["role"] == "temp":
+            continue
+        buf = x[n] if t["role"] in ("in", "inout") else outs[n]
+        host[n] = torch.from_numpy(np.ascontiguousarray(buf)).pin_memory()
+        dev[n] = torch.empty_like(host[n], device="cuda")
+    return host, dev
+
+
+def test_run_host_many_pipelined():
+    """fop_run_host_many: independent plans, copies pipelined over two internal
+    streams and reordered (Johnson's rule); every result equals the oracle's,
+    and a second call on fresh inputs in the same buffers sees only them."""
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp, run_host_many
+    descs = [W.cfg2(2, 8, 16, 16), W.cfg3(2, 16, 8, 8), W.cfg1(3, 5, 7), W.cfg4b(300, 64)]
+    ops = [FusedOp(d) for d in descs]
+    for seed_offset in (0, 7):
+        xs = [W.make_inputs(d, seed_offset=seed_offset) for d in descs]
+        hd = [_host_dev(d, x) for d, x in zip(descs, xs)]
+        run_host_many([(op, h, dv) for op, (h, dv) in zip(ops, hd)])
+        torch.cuda.synchronize()
+        for d, x, (h, _) in zip(descs, xs, hd):
+            ref = O.run(d, x)
+            for n in _outs(d):
+                if d["stmts"][-1]["kind"] == "reduce":
+                    scale = O.run(abs_terms_desc(d, 0), x)[n]
+                    assert_normwise(h[n].numpy(), ref[n], scale, 1e-5, n)
+                else:
+                    assert_bitexact(h[n].numpy(), ref[n], f"{d['name']} {n}")
