@@ -1207,12 +1207,18 @@ struct Gen {
   void gen_row() {
     const int W = L.width;
     const int64_t NVD = L.kl[0].extent / W;
-    const int K = (int)((NVD + 31) / 32);
-    const bool jguard = NVD % 32 != 0;
+    // G warps per row (few long rows): LN lanes across the row's vectors, the
+    // G warp partials of a reduction combined in a fixed order through shared
+    // memory, the row loop uniform across the block (it synchronises)
+    const int G = std::max(1, L.row_g);
+    const int64_t LN = 32 * (int64_t)G;
+    const int64_t GPB = L.block / LN;
+    const int K = (int)((NVD + LN - 1) / LN);
+    const bool jguard = NVD % LN != 0 || G > 1;
     int64_t NRO = 1;
     for (int k = 1; k < L.nsplit; k++) NRO *= L.kl[k].extent;
     int64_t rows = L.work;
-    const int64_t WSTRIDE = L.grid * L.block / 32;
+    const int64_t WSTRIDE = L.grid * L.block / LN;
     // forwarded rows live in registers when they fit (<= 64 values per lane);
     // longer rows are re-read by the lane that stored them (same thread, same
     // address: program order makes the store visible; L2 serves the re-read)
@@ -1251,10 +1257,16 @@ struct Gen {
       return its;
     };
     auto lane_guard = [&](int kk) {
-      return jguard ? "if (lane + " + num(32 * kk) + "u < " + num(NVD) + "u) " : std::string("");
+      return NVD % LN != 0 ? "if (lane + " + num(LN * kk) + "u < " + num(NVD) + "u) " : std::string("");
     };
-    header("ROW_REDUCE (one warp per row, lanes across d_v vectors, butterfly)", 1);
-    o.l("const idx_t lane = threadIdx.x & 31u;");
+    header(G == 1 ? "ROW_REDUCE (one warp per row, lanes across d_v vectors, butterfly)"
+                  : "ROW_REDUCE (" + std::to_string(G) + " warps per row, butterfly + fixed-order shared-memory combine)", 1);
+    o.l("const idx_t lane = threadIdx.x % " + num(LN) + "u;");
+    if (G > 1) {
+      o.l("const idx_t grp = threadIdx.x / " + num(LN) + "u;");
+      for (auto& x : L.stmts)
+        if (x.kind == FOP_REDUCE) o.l("__shared__ float RS" + num(x.stmt) + "[" + num(L.block / 32) + "];");
+    }
     // hoisted row-invariant loads
     for (size_t k = 0; k < L.loads.size(); k++) {
       if (mode[k] != 'H') continue;
@@ -1265,7 +1277,7 @@ struct Gen {
       for (int64_t ro = 0; ro < NRO; ro++)
         for (int kk = 0; kk < K; kk++) {
           auto its = ro_its(ro, {});
-          its.push_back({0, "((lane + " + num(32 * kk) + "u) * " + num(W) + "u)"});
+          its.push_back({0, "((lane + " + num(LN * kk) + "u) * " + num(W) + "u)"});
           std::string off = affine(a, its);
           std::string dst = "H" + num(k) + "[" + num(ro * K + kk) + "]";
           if (vec)
@@ -1292,7 +1304,7 @@ struct Gen {
         for (int64_t ro = 0; ro < NRO; ro++)
           for (int kk = 0; kk < K; kk++) {
             auto its = ro_its(ro, pits);
-            its.push_back({0, "((lane + " + num(32 * kk) + "u) * " + num(W) + "u)"});
+            its.push_back({0, "((lane + " + num(LN * kk) + "u) * " + num(W) + "u)"});
             o.l(lane_guard(kk) + "fop::vload_words<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + num(W) +
                 ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(&P" + num(k) + "[" +
                 num((ro * K + kk) * wpv) + "], " + ptr(a.tensor, affine(a, its)) + ");");
@@ -1303,11 +1315,18 @@ struct Gen {
     };
     for (size_t k = 0; k < L.loads.size(); k++)
       if (mode[k] == 'P') o.l("u32 P" + num(k) + "[" + num(NP * W * es(L.loads[k].tensor) / 4) + "];");
-    o.l("idx_t row = ((idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x) >> 5;");
+    o.l("idx_t row = ((idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x) / " + num(LN) + "u;");
     emit_prefetch("row", "_p");
     o.l("#pragma unroll 1");
-    o.l("for (; row < (idx_t)" + num(rows) + "ull; row += (idx_t)" + num(WSTRIDE) + "ull) {");
-    o.ind++;
+    if (G > 1) {   // block-uniform trip count: every group reaches the barriers
+      o.l("for (idx_t rb_ = (idx_t)blockIdx.x * " + num(GPB) + "u; rb_ < (idx_t)" + num(rows) + "ull; rb_ += (idx_t)" +
+          num(WSTRIDE) + "ull, row += (idx_t)" + num(WSTRIDE) + "ull) {");
+      o.ind++;
+      o.l("const bool rv = row < (idx_t)" + num(rows) + "ull;");
+    } else {
+      o.l("for (; row < (idx_t)" + num(rows) + "ull; row += (idx_t)" + num(WSTRIDE) + "ull) {");
+      o.ind++;
+    }
     for (size_t k = 0; k < L.loads.size(); k++)
       if (mode[k] == 'P') {
         int n = NP * W * es(L.loads[k].tensor) / 4;
@@ -1342,8 +1361,8 @@ struct Gen {
           std::string t = "_" + num(si) + "_" + num(ro) + "_" + num(kk);
           o.l("{");
           o.ind++;
-          o.l("const idx_t iv = (lane + " + num(32 * kk) + "u) * " + num(W) + "u;");
-          if (jguard) o.l("if (lane + " + num(32 * kk) + "u < " + num(NVD) + "u) {");
+          o.l("const idx_t iv = (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
+          if (jguard) o.l(std::string("if (") + (G > 1 ? "rv && " : "") + "lane + " + num(LN * kk) + "u < " + num(NVD) + "u) {");
           auto its2 = its;
           its2.push_back({0, "iv"});
           // loads used by this statement
@@ -1462,10 +1481,20 @@ struct Gen {
         if (x.redop == FOP_RED_SUM)
           o.l(a + " = __fadd_rn(" + a + ", __fadd_rn(fop::lo(" + a + "p), fop::hi(" + a + "p)));");
         o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::warp_max(" : "fop::warp_sum(") + a + ");");
+        if (G > 1) {   // the row's G warp partials, combined in warp order
+          std::string rs = "RS" + num(x.stmt);
+          o.l("if ((threadIdx.x & 31u) == 0u) " + rs + "[threadIdx.x >> 5] = " + a + ";");
+          o.l("__syncthreads();");
+          o.l(a + " = " + rs + "[grp * " + num(G) + "u];");
+          o.l("#pragma unroll");
+          o.l("for (int g_ = 1; g_ < " + num(G) + "; ++g_) " + a + " = " +
+              (x.redop == FOP_RED_MAX ? "fop::op_max(" : "__fadd_rn(") + a + ", " + rs + "[grp * " + num(G) + "u + g_]);");
+          o.l("__syncthreads();");
+        }
         std::string res = fin_expr(o, x, a, "");
         if (x.fwd) o.l("const float S" + num(x.stmt) + " = fop::round_to<" + dtn(x.out_dtype) + ">(" + res + ");");
         if (x.store)
-          o.l("if (lane == 0) fop::sstore<" + std::string(dtn(x.out_dtype)) + ">(" +
+          o.l(std::string(G > 1 ? "if (rv && lane == 0) " : "if (lane == 0) ") + "fop::sstore<" + std::string(dtn(x.out_dtype)) + ">(" +
               ptr(x.write.tensor, affine(x.write, rits)) + ", " + res + ");");
       }
     }

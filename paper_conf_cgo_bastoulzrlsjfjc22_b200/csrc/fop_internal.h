@@ -139,6 +139,7 @@ struct Launch {
   int col_pipe = 0;               // COL: software-pipelined row batches
   int col_il = 1;                 // COL: chunks interleave over rows (grid sweeps rows together)
   int row_hoist = 1;              // ROW: keep row-invariant loads in registers across rows
+  int row_g = 1;                  // ROW: warps per row (> 1 for few long rows)
   // TRANSPOSE through TMA (16-bit data): 64x64 tiles, tensor maps encoded per run
   int tma = 0;
   int tma_rank = 0, tma_stages = 4;

@@ -156,6 +156,11 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 3}});
       break;
     case FOP_CLASS_ROW_REDUCE:
+      if (L.row_g > 1) {   // few long rows: neighbouring warps-per-row counts
+        v.push_back({{"FOP_ROW_G", L.row_g / 2}});
+        if (L.row_g < 32) v.push_back({{"FOP_ROW_G", L.row_g * 2}});
+        break;
+      }
       v.push_back({{"FOP_ROW_MINB", 2}});
       v.push_back({{"FOP_ROW_MINB", 4}});
       v.push_back({{"FOP_BLOCK", 128}, {"FOP_ROW_MINB", 6}});
@@ -417,11 +422,21 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   } else if (L.kclass == FOP_CLASS_ROW_REDUCE) {
     int64_t rows = 1;
     for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
-    L.work = rows;  // one warp per row
-    L.minblocks = knob("FOP_ROW_MINB", 3);
+    L.work = rows;
+    // one warp per row while the rows fill the GPU; few long rows get G warps
+    // each (up to 32), until ~16 warps per SM are busy and every lane still
+    // has >= 2 vectors of the row
+    int64_t nvd = EV / W;
+    int G = 1;
+    while (G < 32 && rows * G < (int64_t)sms * 16 && 64 * (int64_t)G <= nvd) G *= 2;
+    G = std::max(1, pow2_floor(knob("FOP_ROW_G", G)));
+    L.row_g = G;
+    if (G > 1) L.block = std::max(L.block, 32 * G);
+    L.minblocks = knob("FOP_ROW_MINB", L.block >= 1024 ? 1 : (L.block >= 512 ? 2 : 3));
     L.row_prefetch = knob("FOP_ROW_PREFETCH", 1);
     L.row_hoist = knob("FOP_ROW_HOIST", 1);
-    int64_t need = (rows + L.block / 32 - 1) / (L.block / 32);
+    int64_t gpb = L.block / (32 * G);
+    int64_t need = (rows + gpb - 1) / gpb;
     L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
     L.unroll = 1;
   } else {  // COL_REDUCE

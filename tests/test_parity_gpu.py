@@ -391,3 +391,44 @@ def test_run_host_many_pipelined():
                     assert_normwise(h[n].numpy(), ref[n], scale, 1e-5, n)
                 else:
                     assert_bitexact(h[n].numpy(), ref[n], f"{d['name']} {n}")
+
+
+@pytest.mark.parametrize("warm", [True, False])
+def test_cuda_graph_capture_and_replay(warm):
+    """fop_run inside torch.cuda.graph capture: replays follow the buffers'
+    current contents.  warm=False: the plan's first run (module load, no
+    auto-tuning while capturing) happens inside the capture."""
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    descs = [W.cfg2(2, 8, 16, 16), W.cfg3(2, 16, 8, 8), W.cfg4a(1, 7, 200), W.cfg4b(300, 64)]
+    ops = [FusedOp(d) for d in descs]
+    xs = [W.make_inputs(d) for d in descs]
+    devs = [device_tensors(d, x) for d, x in zip(descs, xs)]
+    wss = [op._workspace(torch.device("cuda")) for op in ops]
+    if warm:
+        for op, dv, ws in zip(ops, devs, wss):
+            op.run(dv, workspace=ws)
+        torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for op, dv, ws in zip(ops, devs, wss):
+            op.run(dv, workspace=ws)
+    for seed_offset in (3, 11):
+        xs = [W.make_inputs(d, seed_offset=seed_offset) for d in descs]
+        for d, x, dv in zip(descs, xs, devs):
+            for n, t in d["tensors"].items():
+                if t["role"] in ("in", "inout"):
+                    dv[n].copy_(device_tensors(d, x)[n])
+        g.replay()
+        torch.cuda.synchronize()
+        for d, x, dv in zip(descs, xs, devs):
+            ref = O.run(d, x)
+            for n in _outs(d):
+                got = to_host(dv[n], d["tensors"][n]["dtype"])
+                if d["name"].startswith("cfg4a"):
+                    if n == "y":
+                        assert_ulp(got, ref[n], 1, n)
+                elif d["stmts"][-1]["kind"] == "reduce":
+                    scale = O.run(abs_terms_desc(d, 0), x)[n]
+                    assert_normwise(got, ref[n], scale, 1e-5, n)
+                else:
+                    assert_bitexact(got, ref[n], f"{d['name']} {n}")
