@@ -330,9 +330,9 @@ struct Gen {
                  std::vector<std::pair<int, std::string>>& its) {
     for (int k = k0; k < k1; k++) {
       std::string nm = "i" + num(k) + tag;
-      if (k == k1 - 1) o.l("const idx_t " + nm + " = " + var + ";");
+      if (k == k1 - 1) o.l("[[maybe_unused]] const idx_t " + nm + " = " + var + ";");
       else {
-        o.l("const idx_t " + nm + " = " + var + " % " + num(L.kl[k].extent) + "u;");
+        o.l("[[maybe_unused]] const idx_t " + nm + " = " + var + " % " + num(L.kl[k].extent) + "u;");
         o.l(var + " /= " + num(L.kl[k].extent) + "u;");
       }
       its.push_back({k, nm});
@@ -1361,7 +1361,7 @@ struct Gen {
           std::string t = "_" + num(si) + "_" + num(ro) + "_" + num(kk);
           o.l("{");
           o.ind++;
-          o.l("const idx_t iv = (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
+          o.l("[[maybe_unused]] const idx_t iv = (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
           if (jguard) o.l(std::string("if (") + (G > 1 ? "rv && " : "") + "lane + " + num(LN * kk) + "u < " + num(NVD) + "u) {");
           auto its2 = its;
           its2.push_back({0, "iv"});

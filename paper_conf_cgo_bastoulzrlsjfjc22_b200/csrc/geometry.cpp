@@ -424,11 +424,12 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
     L.work = rows;
     // one warp per row while the rows fill the GPU; few long rows get G warps
-    // each (up to 32), until ~16 warps per SM are busy and every lane still
-    // has >= 2 vectors of the row
+    // each (up to 32), until ~16 warps per SM are busy or a lane would hold
+    // fewer than 4 vectors of the row (measured: G=16 beats 32 at 2-4
+    // vectors per lane, profiles/sweep_r01_rowg.log)
     int64_t nvd = EV / W;
     int G = 1;
-    while (G < 32 && rows * G < (int64_t)sms * 16 && 64 * (int64_t)G <= nvd) G *= 2;
+    while (G < 32 && rows * G < (int64_t)sms * 16 && 256 * (int64_t)G <= nvd) G *= 2;
     G = std::max(1, pow2_floor(knob("FOP_ROW_G", G)));
     L.row_g = G;
     if (G > 1) L.block = std::max(L.block, 32 * G);
