@@ -586,7 +586,8 @@ struct Gen {
         for (const Table& tb : tables)
           if (tb.si == (int)si)
             for (auto& kv : its[u])
-              if (kv.first == tb.k) ov[tb.node] = tb.name + "[" + kv.second + "]";
+              if (kv.first == tb.k)   // slots past the end (ok false) still evaluate: keep the index in the table
+                ov[tb.node] = tb.name + "[ok" + t + " ? " + kv.second + " : 0u]";
         g_over = &ov;
         auto var = varies(x, c);
         emit_nodes(o, x, var, false, c);
@@ -1226,8 +1227,12 @@ struct Gen {
     for (auto& x : L.stmts)
       if (x.kind == FOP_ASSIGN && x.fwd && !regmode && !x.store)
         fail(FOP_E_UNSUPPORTED, "ROW_REDUCE: a long forwarded row must be stored to be re-read");
-    if (NRO > 64) fail(FOP_E_UNSUPPORTED, "ROW_REDUCE: too many outer reduction iterations");
-    const int NP = (int)(NRO * K);   // vectors per lane per row
+    // outer reduction iterations: unrolled at compile time while the row can
+    // stay in registers, a runtime loop otherwise (no per-vector register
+    // arrays are indexed then: no hoisting, prefetch or register forwarding)
+    const bool rt_ro = NRO > 64;
+    const int64_t NRO_E = rt_ro ? 1 : NRO;
+    const int NP = (int)(NRO_E * K);   // vectors per lane per row held in registers
     // per-load treatment: hoisted (independent of the row: e.g. a bias, loaded
     // once per warp), prefetched (streaming vector of the first phase, loaded
     // one row ahead so the reductions overlap the next row's HBM latency), or
@@ -1242,6 +1247,7 @@ struct Gen {
       for (size_t q = L.nsplit; q < L.kl.size(); q++) row_inv &= C(a, (int)q) == 0;
       int64_t cv = C(a, 0);
       int es_k = es(a.tensor);
+      if (rt_ro) continue;
       if (L.row_hoist && row_inv && regmode && (cv == 0 || cv == 1) && !written_here(a.tensor)) mode[k] = 'H';
       else if (L.row_prefetch && used0[k] && cv == 1 && W * es_k >= 4 && L.load_cb[k] >= 4 &&
                NP * W * es_k / 4 <= 32 && !written_here(a.tensor))
@@ -1349,13 +1355,24 @@ struct Gen {
         if (x.redop == FOP_RED_SUM) o.l("u64 acc" + num(x.stmt) + "p = fop::pk1(0.f);");
       }
       if (x.kind == FOP_ASSIGN && x.fwd && regmode) o.l("float F" + num(x.stmt) + "[" + num(NRO * K * W) + "];");
-      for (int64_t ro = 0; ro < NRO; ro++) {
-        // compile-time decomposition of ro over the outer reduction kloops
+      if (rt_ro) {
+        o.l("#pragma unroll 1");
+        o.l("for (idx_t ro_ = 0; ro_ < " + num(NRO) + "u; ++ro_) {");
+        o.ind++;
+        o.l("idx_t rq_ = ro_;");
+      }
+      for (int64_t ro = 0; ro < NRO_E; ro++) {
+        // decomposition of ro over the outer reduction kloops (compile time,
+        // or at run time for the runtime loop)
         std::vector<std::pair<int, std::string>> its = rits;
-        int64_t rem = ro;
-        for (int k = 1; k < L.nsplit; k++) {
-          its.push_back({k, num(rem % L.kl[k].extent) + "u"});
-          rem /= L.kl[k].extent;
+        if (rt_ro) {
+          decompose("rq_", 1, L.nsplit, "_r" + num(si), its);
+        } else {
+          int64_t rem = ro;
+          for (int k = 1; k < L.nsplit; k++) {
+            its.push_back({k, num(rem % L.kl[k].extent) + "u"});
+            rem /= L.kl[k].extent;
+          }
         }
         for (int kk = 0; kk < K; kk++) {
           std::string t = "_" + num(si) + "_" + num(ro) + "_" + num(kk);
@@ -1475,6 +1492,10 @@ struct Gen {
           o.ind--;
           o.l("}");
         }
+      }
+      if (rt_ro) {
+        o.ind--;
+        o.l("}");
       }
       if (red) {
         std::string a = "acc" + num(x.stmt);

@@ -60,16 +60,19 @@ def ordered32(f):
     return np.where(i < 0, -(i & 0x7FFFFFFF), i)
 
 
+def _isnan(a):
+    """NaN mask; uint16 arrays hold raw bf16 bit patterns."""
+    if a.dtype == np.uint16:
+        return ((a & 0x7F80) == 0x7F80) & ((a & 0x007F) != 0)
+    return np.isnan(a.astype(np.float32))
+
+
 def assert_bitexact(got, ref, name=""):
     got, ref = np.asarray(got), np.asarray(ref)
     assert got.shape == ref.shape, (name, got.shape, ref.shape)
     if got.dtype.kind == "f" or got.dtype == np.uint16:
-        wide = got.astype(np.float32) if got.dtype != np.uint16 else got.astype(np.uint32)
-        nan_g = np.isnan(got.astype(np.float32)) if got.dtype != np.uint16 else np.zeros(got.shape, bool)
-        nan_r = np.isnan(ref.astype(np.float32)) if ref.dtype != np.uint16 else np.zeros(ref.shape, bool)
         view = np.uint16 if got.itemsize == 2 else np.uint32
-        same = (got.view(view) == ref.view(view)) | (nan_g & nan_r)
-        del wide
+        same = (got.view(view) == ref.view(view)) | (_isnan(got) & _isnan(ref))
     else:
         same = got == ref
     bad = np.flatnonzero(~same)
@@ -78,13 +81,13 @@ def assert_bitexact(got, ref, name=""):
 
 
 def assert_ulp(got, ref, max_ulp, name=""):
-    """fp16/fp32 outputs within max_ulp (NaN == NaN)."""
+    """fp16/bf16/fp32 outputs within max_ulp (NaN == NaN)."""
     got, ref = np.asarray(got), np.asarray(ref)
-    if got.dtype == np.float16:
+    if got.dtype in (np.float16, np.uint16):   # f16, or raw bf16 bit patterns (same ordering)
         d = np.abs(ordered16(got) - ordered16(ref))
     else:
         d = np.abs(ordered32(got.astype(np.float32)) - ordered32(ref.astype(np.float32)))
-    nan = np.isnan(got.astype(np.float32)) & np.isnan(ref.astype(np.float32))
+    nan = _isnan(got) & _isnan(ref)
     d = np.where(nan, 0, d)
     assert d.max(initial=0) <= max_ulp, f"{name}: max {d.max()} ulp at {np.argmax(d)} " \
                                         f"(got {got.reshape(-1)[np.argmax(d)]}, ref {ref.reshape(-1)[np.argmax(d)]})"

@@ -1,0 +1,100 @@
+"""Randomised operators (tests/fuzz_gen.py) through the whole path.
+
+CPU: every random operator validates, plans and compiles for sm_100a (NVRTC).
+GPU: every random operator matches the oracle — ASSIGN outputs bit for bit
+(IEEE-exact ops; <= 1 ulp for 16-bit outputs of a DAG with a division, which
+may use the correctly-rounded reciprocal of a loop-invariant divisor, DESIGN
+§4), max reductions bit for bit, sums normwise (R16).
+"""
+import numpy as np
+import pytest
+
+import workloads as W
+from oracle import oracle as O
+
+from fuzz_gen import random_op
+
+N_CPU, N_GPU = 80, 160
+
+
+def _ops(n, seed):
+    rng = np.random.default_rng(seed)
+    return [random_op(rng) for _ in range(n)]
+
+
+def test_random_ops_plan_and_compile():
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    classes = set()
+    for d in _ops(N_CPU, 2026):
+        op = FusedOp(d, autotune=0)
+        for li in op.info()["launches"]:
+            classes.add(li["class"])
+            assert li["grid"] >= 1 and li["block"] >= 32
+    assert classes >= {"ew", "row_reduce", "col_reduce"}
+
+
+@pytest.mark.gpu
+def test_random_ops_match_oracle():
+    from harness import run_gpu, assert_bitexact, assert_ulp, assert_normwise, abs_terms_desc
+    for i, d in enumerate(_ops(N_GPU, 4242)):
+        x = W.make_inputs(d)
+        got, op = run_gpu(d, x)
+        ref = O.run(d, x, outputs=W.alloc_outputs(d))
+        for si, st in enumerate(d["stmts"]):
+            n = st["write"][0]
+            t = d["tensors"][n]
+            if t["role"] != "out":
+                continue
+            tag = f"case {i} ({d['name']}) {n}"
+            # reads a statistic produced by a sum reduction: inherits its error
+            from_sum = any(q["kind"] == "reduce" and q.get("op", "sum") == "sum" and
+                           any(r[0] == q["write"][0] for r in st["reads"]) for q in d["stmts"][:si])
+            if st["kind"] == "reduce" and st.get("op", "sum") == "sum":
+                scale = O.run(abs_terms_desc(d, si), x)[n]
+                assert_normwise(got[n], ref[n], scale, 1e-5, tag)
+            elif from_sum and t["dtype"] == "f32":
+                g, r = got[n].astype(np.float64), ref[n].astype(np.float64)
+                assert np.all((np.abs(g - r) <= 1e-5 * np.abs(r) + 1e-30) | (np.isnan(g) & np.isnan(r))), tag
+            elif t["dtype"] != "f32" and (from_sum or any(e[0] == "div" for e in st["expr"])):
+                assert_ulp(got[n], ref[n], 1, tag)
+            else:
+                assert_bitexact(got[n], ref[n], tag)
+
+
+def _table_tail_case():
+    """Found by the fuzz campaign: a per-l0 shared-memory table (x1[l0] / x1[l0]
+    is costly and invariant along l1) read by unroll slots past the end of the
+    work — their index left the table (illegal address)."""
+    return {"name": "table_tail", "loops": {"l0": 100, "l1": 7},
+            "tensors": {"x0": {"shape": [7], "dtype": "f32", "role": "in", "init": ("normal", 0.0, 1.0, 1)},
+                        "x1": {"shape": [100], "dtype": "f16", "role": "in", "init": ("normal", 0.0, 1.0, 2)},
+                        "x2": {"shape": [7], "dtype": "f32", "role": "in", "init": ("normal", 0.0, 1.0, 3)},
+                        "out": {"shape": [100, 7], "dtype": "f16", "role": "out", "strides": [8, 1]}},
+            "stmts": [{"kind": "assign", "loops": ["l0", "l1"], "write": ("out", ["l0", "l1"]),
+                       "reads": [("x0", ["l1"]), ("x1", ["l0"]), ("x2", ["l1"])],
+                       "expr": [("load", 0), ("load", 1), ("load", 2), ("div", 1, 1), ("add", 3, 0),
+                                ("add", 4, 2), ("cast", 5, "bf16")]}]}
+
+
+def _long_outer_reduction_case():
+    """Found by the fuzz campaign: a row reduction over two loops whose outer
+    one has > 64 iterations was rejected (now a runtime loop)."""
+    return {"name": "outer_red", "loops": {"a": 6, "b": 100, "c": 40},
+            "tensors": {"x": {"shape": [6, 100, 40], "dtype": "f16", "role": "in", "init": ("normal", 0.0, 1.0, 4)},
+                        "s": {"shape": [6], "dtype": "f32", "role": "out"}},
+            "stmts": [{"kind": "reduce", "op": "sum", "loops": ["a", "b", "c"], "write": ("s", ["a"]),
+                       "reads": [("x", ["a", "b", "c"])], "expr": [("load", 0)]}]}
+
+
+@pytest.mark.gpu
+def test_fuzz_regressions():
+    from harness import run_gpu, assert_ulp, assert_normwise, abs_terms_desc
+    d = _table_tail_case()
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    assert_ulp(got["out"], O.run(d, x, outputs=W.alloc_outputs(d))["out"], 1, "out")
+    d = _long_outer_reduction_case()
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.info()["launches"][0]["class"] == "row_reduce"
+    assert_normwise(got["s"], O.run(d, x)["s"], O.run(abs_terms_desc(d, 0), x)["s"], 1e-5, "s")
