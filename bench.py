@@ -14,10 +14,13 @@ value = algorithmic bytes of all ranks / device time (max over ranks).
 Multi-GPU (torchrun, one process per GPU, NCCL): weak scaling — every rank
 runs the same per-GPU batch (the global batch is N x; N = 4 is
 BASELINE.json's cfg5 "4x the above batch").  cfg4b's reduced axis (rows) is
-the sharded axis: its [1024] fp32 partial sums are all-reduced (SUM) over
-NCCL inside the timed step.  Nothing else communicates.
+the sharded axis: its [1024] fp32 partial sums are combined across the GPUs
+INSIDE the column-reduction kernel (--exchange peer, default: each rank's
+kernel pushes its partials into every rank's exchange buffer over NVLink peer
+memory and sums all ranks' contributions in rank order), or all-reduced over
+NCCL after it (--exchange nccl, the baseline).  Nothing else communicates.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl fop|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl fop|reference] [--exchange peer|nccl]
 """
 import argparse
 import json
@@ -193,18 +196,29 @@ def run_fop(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # FOP_BENCH_ONE_GPU=1 (test hook): every rank on cuda:0 over gloo, to run
+    # the N > 1 path (CUDA IPC exchange buffers included) on a 1-GPU box
+    one_gpu = os.environ.get("FOP_BENCH_ONE_GPU") == "1"
+    if one_gpu:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
-    from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc, allreduce_partials
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc, allreduce_partials, PeerExchange
+    peer = world > 1 and args.exchange == "peer"
     ops = []
     for name, mk, cls in OPS:
         gmk, loop = GLOBAL[name]
-        d, shard_info = shard_desc(gmk(world), loop, rank, world)   # == mk() per rank
+        d, shard_info = shard_desc(gmk(world), loop, rank, world, fused=peer)   # == mk() per rank
+        popts = {"peer_world": world, "peer_loop": loop} if peer and shard_info["partials"] else {}
         op = FusedOp(d, **({"max_vec_bytes": args.vec_bytes} if args.vec_bytes else {}),
-                     **({"coalesce_order": args.order} if args.order else {}))
+                     **({"coalesce_order": args.order} if args.order else {}), **popts)
+        px = PeerExchange(op.peer_bytes) if op.peer_bytes else None
         x = W.make_inputs(d, seed_offset=rank * 1000)
         outs = W.alloc_outputs(d, fill_nan=False)
         tens, host = {}, {}
@@ -218,22 +232,29 @@ def run_fop(args):
                   if t["role"] in ("in", "inout"))
         d2h = sum(host[n].numel() * host[n].element_size() for n, t in d["tensors"].items()
                   if t["role"] in ("out", "inout"))
-        ops.append({"name": name, "cls": cls, "desc": d, "op": op, "dev": tens, "host": host, "shard": shard_info,
+        ops.append({"name": name, "cls": cls, "desc": d, "op": op, "px": px, "dev": tens, "host": host,
+                    "shard": shard_info,
                     "bytes": W.algorithmic_bytes(d), "h2d": h2d, "d2h": d2h,
                     "launches": len(op.info()["launches"]), "kernel": op.info()["launches"][0]})
         del x, outs
     stream = torch.cuda.current_stream(dev)
 
     def allreduce(o):   # only cfg4b has partials: its rows are the sharded (reduced) axis
-        if world > 1:
+        if world > 1 and o["px"] is None:
             allreduce_partials(o["dev"], o["shard"])
+
+    def run_op(o):
+        if o["px"] is not None:   # partials combined inside the kernel over NVLink (fop_run_peer)
+            o["op"].run(o["dev"], stream=stream, peers=o["px"].peers)
+        else:
+            o["op"].run(o["dev"], stream=stream)
+            allreduce(o)
 
     def step(events=None):
         for i, o in enumerate(ops):
             if events is not None:
                 events[i][0].record(stream)
-            o["op"].run(o["dev"], stream=stream)
-            allreduce(o)
+            run_op(o)
             if events is not None:
                 events[i][1].record(stream)
 
@@ -281,13 +302,22 @@ def run_fop(args):
     def e2e_step():
         items = []
         for o in ops:
+            if o["px"] is not None:
+                continue
             host = o["host"]
             if world > 1 and o["shard"].get("partials"):
                 host = {n: h for n, h in host.items() if n not in dict(o["shard"]["partials"])}
             items.append((o["op"], host, o["dev"]))
         run_host_many(items, stream=stream)
         for o in ops:
-            if world > 1 and o["shard"].get("partials"):
+            if o["px"] is not None:     # inputs in, kernel with the in-kernel combine, result out
+                for n, t in o["desc"]["tensors"].items():
+                    if t["role"] in ("in", "inout"):
+                        o["dev"][n].copy_(o["host"][n], non_blocking=True)
+                run_op(o)
+                for n, _ in o["shard"]["partials"]:
+                    o["host"][n].copy_(o["dev"][n], non_blocking=True)
+            elif world > 1 and o["shard"].get("partials"):
                 allreduce(o)
                 for n, _ in o["shard"]["partials"]:
                     o["host"][n].copy_(o["dev"][n], non_blocking=True)
@@ -347,7 +377,10 @@ def run_fop(args):
                             "[256,256,56,56] f16, cfg4a bias+GELU+row mean/var [64,512,768] f16, cfg4b colsum "
                             "[65536,1024] f16->f32 (BASELINE.json configs[1..3]) per GPU",
                 "global_batch_scale": world,
-                "parallelism": "dp%d (batch-sharded, NCCL all-reduce of cfg4b partials)" % world,
+                "parallelism": ("dp%d (batch-sharded; " % world) + (
+                    "no exchange)" if world == 1 else
+                    "cfg4b partials combined inside the column-reduction kernel over NVLink peer memory)"
+                    if peer else "cfg4b partials all-reduced over NCCL)"),
                 "l2": "no flush: every input is re-read once per step after >1 GB of other ops' traffic "
                       "(B200 L2 126 MB); cfg2/cfg3 inputs alone exceed L2",
                 "per_op_note": "per-op times come from a second pass of the same K steps with CUDA events "
@@ -369,6 +402,10 @@ def run_fop(args):
             "gpu_launches": args.steps * sum(o["launches"] for o in ops),
         }
         print(json.dumps(line), flush=True)
+    torch.cuda.synchronize()
+    for o in ops:
+        if o["px"] is not None:
+            o["px"].close()
     if world > 1:
         dist.destroy_process_group()
     return 0
@@ -383,6 +420,8 @@ def main():
     ap.add_argument("--vec-bytes", type=int, default=0, help="16 or 32 (default: planner default 16)")
     ap.add_argument("--order", choices=["paper", "memory"], default=None)
     ap.add_argument("--no-cpu", action="store_true", help="skip the oracle cpu_baseline leg")
+    ap.add_argument("--exchange", choices=["peer", "nccl"], default="peer",
+                    help="N > 1: combine cfg4b's partial sums inside the kernel over NVLink (peer) or NCCL after it")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

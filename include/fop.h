@@ -49,7 +49,7 @@ extern "C" {
 #define FOP_API
 #endif
 
-#define FOP_ABI_VERSION 2
+#define FOP_ABI_VERSION 3
 
 #define FOP_MAX_RANK     8   /* tensor rank */
 #define FOP_MAX_LOOPS    8   /* loops of the fused operator */
@@ -61,6 +61,7 @@ extern "C" {
 #define FOP_MAX_LAUNCH   8   /* kernel launches per plan */
 #define FOP_MAX_SCEN     8   /* scenarios kept per statement ("set to 8") */
 #define FOP_MAX_DEPS    16   /* dependence vectors reported per statement */
+#define FOP_MAX_PEERS    8   /* GPUs of one peer group (one NVLink/NVSwitch node) */
 
 typedef enum {
   FOP_OK = 0,
@@ -168,6 +169,19 @@ typedef struct {
                                     keeps the fastest (tile sizes are auto-tuned in the paper too).
                                     Skipped for plans that are not idempotent (in-place / read-modify-write)
                                     and while the stream is being captured into a CUDA graph. */
+  /* Multi-GPU (BASELINE.json north_star (4)).  peer_world >= 1: the operator is ONE
+     shard of a larger one whose loop `peer_loop` is split into peer_world contiguous blocks, one per
+     GPU (every rank plans the same shard descriptor).  Each REDUCE statement whose reduction loops
+     include peer_loop then combines the partial results of all ranks INSIDE its kernel: the
+     COL_REDUCE epilogue pushes the rank's per-slab sums into every rank's exchange buffer over
+     NVLink peer memory, waits for the others' pushes, and adds the world contributions in rank
+     order (identical bits on every rank), then finalizes and stores.  Run with fop_run_peer.
+     0 = no exchange (the default). */
+  int32_t peer_world;
+  int32_t peer_loop;             /* loop id split across the peer group (peer_world >= 1) */
+  int32_t peer_timeout_ms;       /* bound on a kernel's wait for its peers; 0 = 10000.  On timeout the
+                                    run's exchanged outputs are NaN and the exchange buffer's error word
+                                    is set (fop_peer_group) */
 } fop_plan_opts;
 
 typedef enum {
@@ -195,6 +209,7 @@ typedef struct {
                                 constraint only), 2 no feasible scenario: uninfluenced schedule, no
                                 explicit vector type, 3 fully sequential (every loop carries a
                                 dependence) */
+  int32_t peer_exchange;     /* 1: this launch combines partial results across the peer group */
 } fop_launch_info;
 
 typedef struct {
@@ -266,6 +281,48 @@ FOP_API fop_status  fop_run_host(const fop_plan_t* plan, void* const* host_ptrs,
 FOP_API fop_status  fop_run_host_many(const fop_plan_t* const* plans, void* const* const* host_ptrs,
                                       void* const* const* dev_ptrs, const int32_t* nptrs,
                                       void* const* workspaces, int32_t n, void* stream);
+
+/* ---------------------------------------------------------------- peer groups (multi-GPU)
+ * Cross-GPU reductions fused into the reducing kernel (plans with
+ * opts.peer_world >= 1, see fop_plan_opts).  Every rank owns one EXCHANGE
+ * BUFFER of fop_plan_peer_bytes() bytes, zero-filled before first use, and maps
+ * every other rank's buffer into its address space (fop_peer_alloc on the
+ * owner, the 64-byte handle sent to the others by any means, fop_peer_open
+ * there; CUDA IPC, so peers are GPUs of one node reached over NVLink /
+ * NVSwitch).  Layout of a buffer, per exchanging launch: [2 parities][world
+ * senders][slabs][slab columns] fp32 partial sums, then [slabs][world] arrival
+ * epochs (written by the senders, release at system scope), then [slabs] local
+ * run counters; the LAST 16 bytes hold an error word (nonzero = a wait timed
+ * out).  The kernels keep the buffer consistent across runs: the buffer must
+ * not be touched between runs, and every rank must run the plan the same
+ * number of times, in the same order relative to the plan's other runs. */
+typedef struct { unsigned char bytes[64]; } fop_ipc_handle;
+typedef struct {
+  int32_t rank;                      /* this GPU's index in the group, 0 <= rank < world */
+  int32_t world;                     /* must equal the plan's opts.peer_world */
+  void* buf[FOP_MAX_PEERS];          /* every rank's exchange buffer as addressed from THIS process;
+                                        buf[rank] = the local one */
+} fop_peer_group;
+
+/* Size of the exchange buffer (0 for plans without peer exchange). */
+FOP_API size_t      fop_plan_peer_bytes(const fop_plan_t* plan);
+/* fop_run for plans with a peer exchange: every rank of the group calls it
+ * (typically on its own GPU, one process per GPU) and each launch waits, on
+ * the device, for the other ranks' matching launch.  Tuning is disabled for
+ * exchanging launches (all ranks must run the same geometry) and a
+ * misaligned tensor pointer returns FOP_E_ALIGN before anything is launched.
+ * Plans without exchange accept group = NULL (then it is fop_run). */
+FOP_API fop_status  fop_run_peer(const fop_plan_t* plan, void* const* dev_ptrs, int32_t nptrs,
+                                 void* workspace, const fop_peer_group* group, void* stream);
+/* Exchange buffers: device memory on the current context's GPU, zero-filled,
+ * owned by libfop until fop_peer_free; `handle` lets other processes map it. */
+FOP_API fop_status  fop_peer_alloc(size_t bytes, void** dev_ptr, fop_ipc_handle* handle);
+FOP_API fop_status  fop_peer_free(void* dev_ptr);
+/* Map another process's exchange buffer (peer access over NVLink is enabled
+ * lazily); unmap with fop_peer_close.  A handle of this same process's buffer
+ * is rejected by CUDA: use the pointer itself. */
+FOP_API fop_status  fop_peer_open(const fop_ipc_handle* handle, void** dev_ptr);
+FOP_API fop_status  fop_peer_close(void* dev_ptr);
 
 /* The kernel fop_run launches for `launch` on the current CUDA context (after
  * auto-tuning; the default geometry before the first run): its name, grid and

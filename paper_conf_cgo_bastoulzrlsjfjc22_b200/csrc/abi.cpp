@@ -75,6 +75,7 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
       if (p.opts.max_vec_bytes != 4 && p.opts.max_vec_bytes != 8 && p.opts.max_vec_bytes != 16 &&
           p.opts.max_vec_bytes != 32)
         fop::fail(FOP_E_INVALID, "max_vec_bytes must be 4, 8, 16 or 32");
+      if (p.opts.peer_world < 0 || p.opts.peer_timeout_ms < 0) fop::fail(FOP_E_INVALID, "negative peer option");
       fop::validate(p.desc);
       fop::plan_launches(p);
       // narrow (scalar) variants for misaligned base pointers: geometry now,
@@ -112,6 +113,7 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
       p.variants.assign(p.launches.size(), {});
       if (p.opts.autotune && p.opts.jit && p.tunable) {
         for (size_t i = 0; i < p.launches.size(); i++) {
+          if (p.launches[i].peer) continue;   // every rank must run the same geometry (fop_run_peer)
           auto vs = fop::tuning_variants(p.launches[i]);
           std::vector<std::string> seen = {p.launches[i].src};
           for (size_t k = 1; k < vs.size(); k++) {
@@ -180,6 +182,7 @@ fop_status fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* o) {
       for (size_t q = 0; q < L.seq.size() && q < FOP_MAX_LOOPS; q++) li.seq[q] = L.seq[q];
       li.scen_pick = L.scen_pick;
       li.fallback = L.fallback;
+      li.peer_exchange = L.peer ? 1 : 0;
     }
     o->workspace_bytes = p.ws_bytes;
     for (int s = 0; s < p.desc.nstmts; s++) {
@@ -239,6 +242,41 @@ fop_status fop_run_host_many(const fop_plan_t* const* plans, void* const* const*
       ps[k] = &const_cast<fop_plan_t*>(plans[k])->p;
     }
     return fop::run_host_many(ps.data(), host_ptrs, dev_ptrs, nptrs, workspaces, n, stream);
+  });
+}
+
+size_t fop_plan_peer_bytes(const fop_plan_t* plan) { return plan ? plan->p.peer_bytes : 0; }
+
+fop_status fop_run_peer(const fop_plan_t* plan, void* const* dev_ptrs, int32_t nptrs, void* workspace,
+                        const fop_peer_group* group, void* stream) {
+  return guarded([&] {
+    if (!plan || !dev_ptrs) fop::fail(FOP_E_INVALID, "NULL plan or pointer table");
+    return fop::run_plan(const_cast<fop_plan_t*>(plan)->p, dev_ptrs, nptrs, workspace, stream, nullptr, group);
+  });
+}
+
+fop_status fop_peer_alloc(size_t bytes, void** dev_ptr, fop_ipc_handle* handle) {
+  return guarded([&] {
+    fop::peer_alloc(bytes, dev_ptr, handle);
+    return FOP_OK;
+  });
+}
+fop_status fop_peer_free(void* dev_ptr) {
+  return guarded([&] {
+    fop::peer_free(dev_ptr);
+    return FOP_OK;
+  });
+}
+fop_status fop_peer_open(const fop_ipc_handle* handle, void** dev_ptr) {
+  return guarded([&] {
+    fop::peer_open(handle, dev_ptr);
+    return FOP_OK;
+  });
+}
+fop_status fop_peer_close(void* dev_ptr) {
+  return guarded([&] {
+    fop::peer_close(dev_ptr);
+    return FOP_OK;
   });
 }
 

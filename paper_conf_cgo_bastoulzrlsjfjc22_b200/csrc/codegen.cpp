@@ -1744,6 +1744,67 @@ struct Gen {
       o.l("__syncthreads();");
     };
     tree();
+    // Cross-GPU combine (opts.peer_world >= 1, fop.h peer groups; SURVEY
+    // §8(e)): the block holding this rank's slab sums in red[0 .. SW) pushes
+    // them into slot [parity][rank][slab] of every rank's exchange buffer
+    // (NVLink stores), publishes one epoch flag per receiver (release, system
+    // scope), waits for every rank's flag in its own buffer (acquire), and
+    // sums the world contributions in rank order — the same order on every
+    // rank, so all ranks store identical bits.  The epoch is a per-slab run
+    // counter kept in the local buffer; the two parities let a rank run ahead
+    // by one run without overwriting data a slower rank has not read yet (it
+    // cannot get further: its next wait needs that rank's next push).
+    auto exchange = [&]() {
+      if (!L.peer) return;
+      const int PW = p.opts.peer_world;
+      const PeerLayout pl = peer_layout(L, PW);
+      const int64_t S = L.peer_slabs;
+      const unsigned long long lim =
+          (unsigned long long)(p.opts.peer_timeout_ms > 0 ? p.opts.peer_timeout_ms : 10000) * 1000000ull;
+      const std::string base = num((int64_t)L.peer_off);
+      o.l("{");
+      o.ind++;
+      o.l("__shared__ unsigned xep_, xok_;");
+      o.l("char* const xb_ = args.peer[args.rank] + " + base + "ull;");
+      o.l("if (tid == 0u) {");
+      o.l("  volatile unsigned* c_ = (volatile unsigned*)(xb_ + " + num((int64_t)pl.epoch) + "ull) + slab;");
+      o.l("  xep_ = *c_ + 1u;");
+      o.l("  *c_ = xep_;");
+      o.l("  xok_ = 1u;");
+      o.l("}");
+      o.l("__syncthreads();");
+      o.l("const unsigned xe_ = xep_, xp_ = xe_ & 1u;");
+      o.l("for (unsigned i_ = tid; i_ < " + num(PW * SW) + "u; i_ += " + num(L.block) + "u) {");
+      o.l("  const unsigned q_ = i_ / " + num(SW) + "u, e_ = i_ % " + num(SW) + "u;");
+      o.l("  float* d_ = (float*)(args.peer[q_] + " + base + "ull) + ((xp_ * " + num(PW) + "u + args.rank) * " + num(S) +
+          "ull + slab) * " + num(SW) + "u + e_;");
+      o.l("  *d_ = red[e_];");
+      o.l("}");
+      o.l("__syncthreads();");
+      o.l("if (tid < " + num(PW) + "u) {");
+      o.l("  __threadfence_system();");
+      o.l("  fop::st_release_sys((unsigned*)(args.peer[tid] + " + base + "ull + " + num((int64_t)pl.flags) + "ull) + slab * " +
+          num(PW) + "u + args.rank, xe_);");
+      o.l("  if (!fop::wait_epoch((const unsigned*)(xb_ + " + num((int64_t)pl.flags) + "ull) + slab * " + num(PW) +
+          "u + tid, xe_, " + std::to_string(lim) + "ull)) {");
+      o.l("    xok_ = 0u;");
+      o.l("    atomicExch((unsigned*)(args.peer[args.rank] + " + num((int64_t)(p.peer_bytes - 16)) + "ull), 1u);");
+      o.l("  }");
+      o.l("}");
+      o.l("__syncthreads();");
+      o.l("if (rl == 0u) {");
+      o.l("  #pragma unroll");
+      o.l("  for (int e = 0; e < " + num(W) + "; ++e) {");
+      o.l("    float s_ = " + init + ";");
+      o.l("    for (unsigned q_ = 0; q_ < " + num(PW) + "u; ++q_)");
+      o.l("      s_ = " + comb("s_", "fop::ld_relaxed_sys((const float*)xb_ + ((xp_ * " + num(PW) + "u + q_) * " + num(S) +
+                                  "ull + slab) * " + num(SW) + "u + cv * " + num(W) + "u + e)") + ";");
+      o.l("    red[cv * " + num(W) + "u + e] = xok_ ? s_ : __int_as_float(0x7fc00000);");
+      o.l("  }");
+      o.l("}");
+      o.ind--;
+      o.l("}");
+    };
     auto final_store = [&]() {
       o.l("if (rl == 0u && okc) {");
       o.ind++;
@@ -1769,6 +1830,7 @@ struct Gen {
       o.l("}");
     };
     if (NCH == 1) {
+      exchange();
       final_store();
     } else {
       size_t part = (size_t)NCH * (size_t)slabs * (size_t)SW * sizeof(float);
@@ -1824,6 +1886,7 @@ struct Gen {
       }
       o.l("__syncthreads();");
       tree();
+      exchange();
       final_store();
       o.l("if (tid == 0u) cnt[slab] = 0u;");
       o.ind--;

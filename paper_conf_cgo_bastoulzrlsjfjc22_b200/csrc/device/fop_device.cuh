@@ -539,9 +539,48 @@ __device__ __forceinline__ void sts128(u32 addr, u32 a, u32 b, u32 c, u32 d) {
   asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
 }
 
+// ---------------------------------------------------------------- peer exchange (multi-GPU)
+// Cross-GPU reduction in a COL_REDUCE epilogue (fop.h, peer groups): plain
+// stores of the partial sums into every rank's exchange buffer (NVLink peer
+// memory), then per receiver one epoch flag stored with release semantics at
+// system scope; receivers poll their own flags with acquire loads.  The
+// block-wide barrier between the data stores and the flag store makes the
+// other threads' stores part of what the release publishes (the same pattern
+// as a grid barrier, at system scope).
+__device__ __forceinline__ void st_release_sys(unsigned* p, unsigned v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ float ld_relaxed_sys(const float* p) {
+  float v;
+  asm volatile("ld.relaxed.sys.global.f32 %0, [%1];" : "=f"(v) : "l"(p) : "memory");
+  return v;
+}
+// Wait until *flag has reached epoch `ep` (wrap-safe); false after ~limit_ns.
+__device__ __forceinline__ bool wait_epoch(const unsigned* flag, unsigned ep, unsigned long long limit_ns) {
+  unsigned long long t0 = 0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  unsigned ns = 32;
+  while ((int)(ld_acquire_sys(flag) - ep) < 0) {
+    unsigned long long t = 0;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > limit_ns) return false;
+    __nanosleep(ns);
+    if (ns < 1024) ns *= 2;
+  }
+  return true;
+}
+
 }  // namespace fop
 
 struct FopArgs {
   char* p[16];
   char* ws;
+  char* peer[8];     // exchange buffers of the peer group as seen from this GPU (fop_peer_group)
+  unsigned rank;     // this GPU's index in the peer group
+  unsigned world;
 };

@@ -165,7 +165,30 @@ struct Launch {
   size_t ws_off = 0, ws_bytes = 0;  // COL_REDUCE partials + counters
   std::vector<int> align;         // per tensor: byte alignment the vector variant assumes
   bool scalar_variant = false;    // this launch is the narrow (W=1) variant
+  // multi-GPU (opts.peer_world >= 1): COL_REDUCE partials combined across the
+  // peer group in the kernel's epilogue (fop.h, peer groups)
+  bool peer = false;
+  size_t peer_off = 0;            // this launch's region in the exchange buffer
+  int64_t peer_slabs = 0;         // slabs (= exchange units) of the launch
 };
+
+// Exchange-buffer region of a peer-exchanging COL_REDUCE launch (fop.h, peer
+// groups): [2 parities][world][slabs][SW] fp32 | [slabs][world] u32 epochs
+// written by the senders | [slabs] u32 local run counters.  Offsets relative
+// to Launch::peer_off.
+struct PeerLayout {
+  size_t data = 0, flags = 0, epoch = 0, total = 0;
+};
+inline PeerLayout peer_layout(const Launch& L, int world) {
+  auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
+  PeerLayout r;
+  const size_t sw = (size_t)L.gv * (size_t)L.width;
+  r.data = 0;
+  r.flags = al(2 * (size_t)world * (size_t)L.peer_slabs * sw * sizeof(float));
+  r.epoch = r.flags + al((size_t)L.peer_slabs * (size_t)world * sizeof(unsigned));
+  r.total = r.epoch + al((size_t)L.peer_slabs * sizeof(unsigned));
+  return r;
+}
 
 struct Plan {
   fop_desc desc;
@@ -175,6 +198,7 @@ struct Plan {
   std::vector<Launch> launches;
   std::vector<int64_t> temp_off;  // per tensor: workspace byte offset (-1 = not materialised)
   size_t ws_bytes = 0;
+  size_t peer_bytes = 0;          // exchange buffer (fop_plan_peer_bytes); 0 = no peer exchange
   // lazily built narrow variants (misaligned pointers), guarded by mu
   std::mutex mu;
   std::vector<Launch> narrow;     // same indexing as launches (empty src = not built)
@@ -208,7 +232,11 @@ bool jit_available();
 fop_status run_host_many(Plan* const* plans, void* const* const* host_ptrs, void* const* const* dev_ptrs,
                          const int32_t* nptrs, void* const* ws, int n, void* stream);
 fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream,
-                    void* const* host_ptrs);
+                    void* const* host_ptrs, const fop_peer_group* peers = nullptr);
+void peer_alloc(size_t bytes, void** dev_ptr, fop_ipc_handle* handle);
+void peer_free(void* dev_ptr);
+void peer_open(const fop_ipc_handle* handle, void** dev_ptr);
+void peer_close(void* dev_ptr);
 void* current_context_or_null();   // the calling thread's CUDA context (nullptr without a driver)
 
 }  // namespace fop

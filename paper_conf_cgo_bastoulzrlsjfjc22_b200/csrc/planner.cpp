@@ -681,6 +681,50 @@ void plan_launches(Plan& p) {
     }
   }
   p.ws_bytes = ws;
+
+  // ---- multi-GPU (opts.peer_world >= 1; fop.h): a REDUCE
+  // statement whose reduction loops include the loop split across the peer
+  // group combines the ranks' partial results in its COL_REDUCE epilogue.
+  // Only the final result may be exchanged: a statement that consumes it in
+  // the same operator would read a partial value.
+  p.peer_bytes = 0;
+  if (p.opts.peer_world >= 1) {
+    const int PW = p.opts.peer_world, PL = p.opts.peer_loop;
+    if (PW > FOP_MAX_PEERS) fail(FOP_E_INVALID, "peer_world exceeds FOP_MAX_PEERS");
+    if (PL < 0 || PL >= d.nloops) fail(FOP_E_INVALID, "peer_loop is not a loop of the operator");
+    for (int s = 0; s < d.nstmts; s++) {
+      bool iterates = false;
+      for (int k = 0; k < d.s[s].nloops; k++) iterates |= d.s[s].loop[k] == PL;
+      if (!iterates || empty_domain(d, d.s[s])) continue;
+      const int T = d.s[s].acc[0].tensor;
+      if (d.s[s].kind != FOP_REDUCE || !(red_loops(d, s) >> PL & 1u)) continue;
+      if (inl[s])
+        fail(FOP_E_UNSUPPORTED, "statement " + std::to_string(s) + " reduces over the peer loop but is fused into a consumer");
+      for (int q = s + 1; q < d.nstmts; q++)
+        for (int a = 1; a < d.s[q].nacc; a++)
+          if (d.s[q].acc[a].tensor == T)
+            fail(FOP_E_UNSUPPORTED, "statement " + std::to_string(q) + " consumes the cross-GPU reduction of statement " +
+                                        std::to_string(s) + " inside the same operator");
+      Launch* X = nullptr;
+      for (auto& L : p.launches)
+        if (L.main_stmt == s) X = &L;
+      if (!X || X->kclass != FOP_CLASS_COL_REDUCE || X->stmts.size() != 1)
+        fail(FOP_E_UNSUPPORTED, "statement " + std::to_string(s) +
+                                    ": a reduction over the peer loop must be a COL_REDUCE launch of its own (the "
+                                    "vector loop parallel)");
+      X->peer = true;
+    }
+    size_t off = 0;
+    for (auto& L : p.launches) {
+      if (!L.peer) continue;
+      int64_t svn = (L.kl[0].extent / L.width + L.gv - 1) / L.gv;
+      for (int k = 1; k < L.nsplit; k++) svn *= L.kl[k].extent;
+      L.peer_slabs = svn;
+      L.peer_off = off;
+      off += peer_layout(L, PW).total;
+    }
+    p.peer_bytes = off ? off + 16 : 0;   // + error word; no exchanging launch: no buffer
+  }
 }
 
 }  // namespace fop

@@ -53,6 +53,13 @@ struct Cuda {
   CUresult (*stream_capturing)(CUstream, int*);
   CUresult (*stream_create)(CUstream*, unsigned);
   CUresult (*stream_wait)(CUstream, void*, unsigned);
+  CUresult (*mem_alloc)(CUdeviceptr*, size_t);
+  CUresult (*mem_free)(CUdeviceptr);
+  CUresult (*memset8)(CUdeviceptr, unsigned char, size_t);
+  CUresult (*ctx_sync)();
+  CUresult (*ipc_get)(fop_ipc_handle*, CUdeviceptr);
+  CUresult (*ipc_open)(CUdeviceptr*, fop_ipc_handle, unsigned);
+  CUresult (*ipc_close)(CUdeviceptr);
   CUresult (*tmap_encode)(void*, int, unsigned, void*, const uint64_t*, const uint64_t*, const unsigned*,
                           const unsigned*, int, int, int, int);
 };
@@ -95,6 +102,13 @@ Cuda& cuda() {
     SYM(stream_create, "cuStreamCreate");
     SYM(stream_wait, "cuStreamWaitEvent");
     SYM(tmap_encode, "cuTensorMapEncodeTiled");
+    SYM(mem_alloc, "cuMemAlloc_v2");
+    SYM(mem_free, "cuMemFree_v2");
+    SYM(memset8, "cuMemsetD8_v2");
+    SYM(ctx_sync, "cuCtxSynchronize");
+    SYM(ipc_get, "cuIpcGetMemHandle");
+    SYM(ipc_open, "cuIpcOpenMemHandle_v2");
+    SYM(ipc_close, "cuIpcCloseMemHandle");
 #undef SYM
     if (c.init(0) != 0) {
       c.why = "cuInit failed";
@@ -193,9 +207,25 @@ void* current_context_or_null() {
   return ctx;
 }
 
-fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream, void* const* host_ptrs) {
+fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream, void* const* host_ptrs,
+                    const fop_peer_group* peers) {
   const fop_desc& d = p.desc;
   if (nptrs != d.ntensors) fail(FOP_E_INVALID, "nptrs must equal desc.ntensors");
+  if (p.peer_bytes) {   // every argument error is caught before any launch (the peers would wait)
+    if (!peers) fail(FOP_E_INVALID, "this plan exchanges partial results across a peer group: run it with fop_run_peer");
+    if (peers->world != p.opts.peer_world)
+      fail(FOP_E_INVALID, "peer group world " + std::to_string(peers->world) + " != plan peer_world " +
+                              std::to_string(p.opts.peer_world));
+    if (peers->rank < 0 || peers->rank >= peers->world) fail(FOP_E_INVALID, "peer rank out of range");
+    for (int q = 0; q < peers->world; q++)
+      if (!peers->buf[q] || ((uintptr_t)peers->buf[q] % 256))
+        fail(FOP_E_INVALID, "exchange buffer of rank " + std::to_string(q) + " is NULL or not 256-byte aligned");
+    for (const auto& L : p.launches)
+      for (int t = 0; t < d.ntensors; t++)
+        if (L.peer && ptrs[t] && ((uintptr_t)ptrs[t] % (uintptr_t)L.align[t]))
+          fail(FOP_E_ALIGN, "tensor " + std::to_string(t) + " is not aligned for the planned vector width (peer "
+                            "exchanges need the same kernel on every rank)");
+  }
   for (auto& L : p.launches)
     if (L.cubin.empty()) fail(FOP_E_INVALID, "plan was built with opts.jit = 0: nothing to run");
   Cuda& c = cuda();
@@ -223,8 +253,15 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
 
     char* p[16];
     char* ws;
+    char* peer[8];
+    unsigned rank, world;
   } args;
   std::memset(&args, 0, sizeof args);
+  if (peers && p.peer_bytes) {
+    for (int q = 0; q < peers->world; q++) args.peer[q] = (char*)peers->buf[q];
+    args.rank = (unsigned)peers->rank;
+    args.world = (unsigned)peers->world;
+  }
   for (int t = 0; t < d.ntensors; t++) {
     args.p[t] = (char*)ptrs[t];
     if (d.t[t].role == FOP_TEMP && p.temp_off[t] >= 0) args.p[t] = (char*)ws + p.temp_off[t];
@@ -330,6 +367,47 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
         check(c.d2h(host_ptrs[t], (CUdeviceptr)ptrs[t], (size_t)span_bytes(d.t[t]), st), "cuMemcpyDtoHAsync");
   }
   return FOP_OK;
+}
+
+// ---------------------------------------------------------------- peer buffers (CUDA IPC)
+void peer_alloc(size_t bytes, void** dev_ptr, fop_ipc_handle* handle) {
+  Cuda& c = cuda();
+  if (!c.ok) fail(FOP_E_CUDA, c.why);
+  if (!dev_ptr || !handle || !bytes) fail(FOP_E_INVALID, "NULL argument or zero size");
+  CUcontext ctx = nullptr;
+  check(c.ctx_get(&ctx), "cuCtxGetCurrent");
+  if (!ctx) fail(FOP_E_CUDA, "no current CUDA context (select and initialise the device first)");
+  CUdeviceptr p = 0;
+  check(c.mem_alloc(&p, bytes), "cuMemAlloc");
+  CUresult r = c.memset8(p, 0, bytes);
+  if (r == 0) r = c.ctx_sync();
+  if (r == 0) r = c.ipc_get(handle, p);
+  if (r != 0) {
+    c.mem_free(p);
+    check(r, "exchange buffer (memset / cuIpcGetMemHandle)");
+  }
+  *dev_ptr = (void*)p;
+}
+void peer_free(void* dev_ptr) {
+  Cuda& c = cuda();
+  if (!c.ok) fail(FOP_E_CUDA, c.why);
+  if (dev_ptr) check(c.mem_free((CUdeviceptr)dev_ptr), "cuMemFree");
+}
+void peer_open(const fop_ipc_handle* handle, void** dev_ptr) {
+  Cuda& c = cuda();
+  if (!c.ok) fail(FOP_E_CUDA, c.why);
+  if (!dev_ptr || !handle) fail(FOP_E_INVALID, "NULL argument");
+  CUcontext ctx = nullptr;
+  check(c.ctx_get(&ctx), "cuCtxGetCurrent");
+  if (!ctx) fail(FOP_E_CUDA, "no current CUDA context (select and initialise the device first)");
+  CUdeviceptr p = 0;
+  check(c.ipc_open(&p, *handle, 1 /* CU_IPC_MEM_LAZY_ENABLE_PEER_ACCESS */), "cuIpcOpenMemHandle");
+  *dev_ptr = (void*)p;
+}
+void peer_close(void* dev_ptr) {
+  Cuda& c = cuda();
+  if (!c.ok) fail(FOP_E_CUDA, c.why);
+  if (dev_ptr) check(c.ipc_close((CUdeviceptr)dev_ptr), "cuIpcCloseMemHandle");
 }
 
 // ---------------------------------------------------------------- host pipeline

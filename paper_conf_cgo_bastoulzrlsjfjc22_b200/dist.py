@@ -14,6 +14,14 @@ finalize step (finalize(a+b) != finalize(a)+finalize(b) in general).
 
     sh = shard_desc(desc, "r", rank, world)       # the rank's sub-operator
     op = ShardedFusedOp(desc, "r", group=pg)      # plan + run + all-reduce
+
+Two ways to combine partial results:
+  exchange="peer" (default on GPUs): the reduction kernel itself pushes its
+      partial sums into every rank's exchange buffer over NVLink peer memory
+      and adds all ranks' contributions in rank order (fop_run_peer; one
+      kernel per rank, no separate collective; identical bits on all ranks;
+      a finalize step is then legal because it runs after the combine);
+  exchange="nccl": fop_run, then one NCCL all-reduce per partial tensor.
 """
 import copy
 
@@ -37,7 +45,7 @@ def _index_loops(index):
     return out
 
 
-def shard_desc(desc, loop, rank, world):
+def shard_desc(desc, loop, rank, world, fused=False):
     """Sub-operator of `rank` when `loop` is split in `world` contiguous blocks.
 
     Returns (shard, info): `shard` is a description whose tensors are the
@@ -50,7 +58,7 @@ def shard_desc(desc, loop, rank, world):
     blk = E // world
     sh = copy.deepcopy(desc)
     sh["loops"][loop] = blk
-    info = {"partials": [], "slices": {}}
+    info = {"partials": [], "slices": {}, "loop": loop}
     # every tensor dim indexed by `loop` is cut to the rank's block
     dims = {}
     for s in desc["stmts"]:
@@ -80,8 +88,9 @@ def shard_desc(desc, loop, rank, world):
             continue
         if s["kind"] != "reduce":
             raise ShardError(f"statement {i} writes {s['write'][0]} repeatedly along {loop!r}")
-        if s.get("finalize"):
-            raise ShardError(f"statement {i}: a finalize step cannot be applied to partial results")
+        if s.get("finalize") and not fused:
+            raise ShardError(f"statement {i}: a finalize step cannot be applied to partial results "
+                             "(use the fused peer exchange, which finalizes after the combine)")
         later_reads = [j for j in range(i + 1, len(desc["stmts"]))
                        if any(r[0] == s["write"][0] for r in desc["stmts"][j]["reads"])]
         if later_reads:
@@ -93,7 +102,7 @@ def shard_desc(desc, loop, rank, world):
 def shard_inputs(desc, loop, rank, world, inputs):
     """Slice full host inputs (flat buffers of a contiguous layout) to the rank's block."""
     import numpy as np
-    _, info = shard_desc(desc, loop, rank, world)
+    _, info = shard_desc(desc, loop, rank, world, fused=True)   # slices only
     out = {}
     for name, buf in inputs.items():
         if name not in info["slices"]:
@@ -115,18 +124,67 @@ def allreduce_partials(tensors, info, group=None):
         dist.all_reduce(tensors[name], op=_RED[op], group=group)
 
 
-class ShardedFusedOp:
-    """Plan the rank's sub-operator once; run = fop_run + all-reduce of partials."""
+class PeerExchange:
+    """The exchange buffers of one peer-exchanging plan across a process group
+    (fop.h, peer groups): each rank allocates its zero-filled buffer with
+    fop_peer_alloc, the 64-byte CUDA IPC handles are all-gathered over the
+    process group, and every other rank's buffer is mapped with fop_peer_open
+    (NVLink peer access).  `self.peers` is the fop_peer_group to run with."""
 
-    def __init__(self, desc, loop, group=None, rank=None, world=None, **opts):
+    def __init__(self, nbytes, group=None, rank=None, world=None, _alloc=None, _open=None):
+        from . import fop as F
+        alloc = _alloc or F.peer_alloc
+        open_ = _open or F.peer_open
+        self.rank = dist.get_rank(group) if rank is None else rank
+        self.world = dist.get_world_size(group) if world is None else world
+        self.nbytes = nbytes
+        self.local, handle = alloc(nbytes)
+        handles = [None] * self.world
+        dist.all_gather_object(handles, (self.rank, nbytes, handle), group=group)
+        for q, (r, n, _) in enumerate(handles):
+            if r != q or n != nbytes:
+                raise ShardError(f"rank {q}: exchange buffer of {n} bytes (rank {r}) does not match {nbytes}")
+        self.opened = {q: open_(handles[q][2]) for q in range(self.world) if q != self.rank}
+        self.bufs = [self.local if q == self.rank else self.opened[q] for q in range(self.world)]
+        self.peers = F.PeerGroup(self.rank, self.bufs)
+
+    def close(self, _close=None, _free=None):
+        from . import fop as F
+        for p in self.opened.values():
+            (_close or F.peer_close)(p)
+        (_free or F.peer_free)(self.local)
+        self.opened, self.local = {}, None
+
+
+class ShardedFusedOp:
+    """Plan the rank's sub-operator once; run = the rank's kernels with the
+    partial results combined in the reduction kernel over NVLink
+    (exchange="peer") or fop_run + an NCCL all-reduce (exchange="nccl")."""
+
+    def __init__(self, desc, loop, group=None, rank=None, world=None, exchange="peer", **opts):
         from .fop import FusedOp
         self.group = group
         self.rank = dist.get_rank(group) if rank is None else rank
         self.world = dist.get_world_size(group) if world is None else world
-        self.shard, self.info = shard_desc(desc, loop, self.rank, self.world)
+        self.exchange = exchange
+        fused = exchange == "peer"
+        self.shard, self.info = shard_desc(desc, loop, self.rank, self.world, fused=fused)
+        if fused and self.info["partials"]:
+            opts = dict(opts, peer_world=self.world, peer_loop=loop)
         self.op = FusedOp(self.shard, **opts)
+        self.px = PeerExchange(self.op.peer_bytes, group, self.rank, self.world) if self.op.peer_bytes else None
 
     def run(self, tensors, stream=None):
+        if self.px is not None:
+            self.op.run(tensors, stream=stream, peers=self.px.peers)
+            return
         self.op.run(tensors, stream=stream)
         if self.world > 1:
             allreduce_partials(tensors, self.info, self.group)
+
+    def close(self):
+        if self.px is not None:
+            import torch as _t
+            _t.cuda.synchronize()
+            self.px.close()
+            self.px = None

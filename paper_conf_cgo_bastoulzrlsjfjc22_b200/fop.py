@@ -22,6 +22,7 @@ _lib = C.CDLL(LIB_PATH)
 
 MAX_RANK, MAX_LOOPS, MAX_TENSORS, MAX_STMTS = 8, 8, 16, 8
 MAX_ACC, MAX_NODES, MAX_FIN, MAX_LAUNCH, MAX_SCEN, MAX_DEPS = 8, 48, 8, 8, 8, 16
+MAX_PEERS = 8
 
 DTYPE = {"f32": 0, "f16": 1, "bf16": 2, "i32": 3}
 ROLE = {"in": 1, "out": 2, "inout": 3, "temp": 4}
@@ -66,7 +67,8 @@ class PlanOpts(C.Structure):
     _fields_ = [("w", C.c_double * 5), ("thread_limit", C.c_int32), ("max_scenarios", C.c_int32),
                 ("max_vec_bytes", C.c_int32), ("readings", C.c_int32), ("force_width", C.c_int32),
                 ("coalesce_order", C.c_int32), ("sm_count", C.c_int32), ("jit", C.c_int32),
-                ("autotune", C.c_int32)]
+                ("autotune", C.c_int32), ("peer_world", C.c_int32), ("peer_loop", C.c_int32),
+                ("peer_timeout_ms", C.c_int32)]
 
 
 class LaunchInfo(C.Structure):
@@ -74,7 +76,7 @@ class LaunchInfo(C.Structure):
                 ("vec_loop", C.c_int32), ("width", C.c_int32), ("read_loop", C.c_int32),
                 ("read_width", C.c_int32), ("coal_loop", C.c_int32), ("grid", C.c_int64),
                 ("block", C.c_int32), ("nseq", C.c_int32), ("seq", C.c_int32 * MAX_LOOPS),
-                ("scen_pick", C.c_int32), ("fallback", C.c_int32)]
+                ("scen_pick", C.c_int32), ("fallback", C.c_int32), ("peer_exchange", C.c_int32)]
 
 
 class PlanInfo(C.Structure):
@@ -89,7 +91,7 @@ class PlanInfo(C.Structure):
 
 
 _lib.fop_abi_version.restype = C.c_int
-ABI_VERSION = 2   # the struct layouts above mirror include/fop.h at this version
+ABI_VERSION = 3   # the struct layouts above mirror include/fop.h at this version
 if _lib.fop_abi_version() != ABI_VERSION:
     raise ImportError(f"{LIB_PATH}: ABI version {_lib.fop_abi_version()} != binding {ABI_VERSION}; rebuild "
                       "with python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build")
@@ -117,12 +119,37 @@ _lib.fop_plan_selected.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_char_p),
                                    C.POINTER(C.c_int32)]
 _lib.fop_plan_selected.restype = C.c_int
 _lib.fop_plan_destroy.argtypes = [C.c_void_p]
+
+
+class IpcHandle(C.Structure):
+    _fields_ = [("bytes", C.c_ubyte * 64)]
+
+
+class PeerGroupC(C.Structure):
+    _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("buf", C.c_void_p * MAX_PEERS)]
+
+
+_lib.fop_plan_peer_bytes.argtypes = [C.c_void_p]
+_lib.fop_plan_peer_bytes.restype = C.c_size_t
+_lib.fop_run_peer.argtypes = [C.c_void_p, C.POINTER(C.c_void_p), C.c_int32, C.c_void_p, C.POINTER(PeerGroupC),
+                              C.c_void_p]
+_lib.fop_run_peer.restype = C.c_int
+_lib.fop_peer_alloc.argtypes = [C.c_size_t, C.POINTER(C.c_void_p), C.POINTER(IpcHandle)]
+_lib.fop_peer_alloc.restype = C.c_int
+_lib.fop_peer_free.argtypes = [C.c_void_p]
+_lib.fop_peer_free.restype = C.c_int
+_lib.fop_peer_open.argtypes = [C.POINTER(IpcHandle), C.POINTER(C.c_void_p)]
+_lib.fop_peer_open.restype = C.c_int
+_lib.fop_peer_close.argtypes = [C.c_void_p]
+_lib.fop_peer_close.restype = C.c_int
 _lib.fop_status_str.restype = C.c_char_p
 _lib.fop_last_error.restype = C.c_char_p
 
 ABI_SYMBOLS = ["fop_abi_version", "fop_plan_opts_default", "fop_plan", "fop_plan_info_get",
                "fop_plan_workspace_bytes", "fop_plan_source", "fop_plan_cubin", "fop_run",
-               "fop_run_host", "fop_run_host_many", "fop_plan_selected", "fop_plan_destroy", "fop_status_str", "fop_last_error"]
+               "fop_run_host", "fop_run_host_many", "fop_plan_selected", "fop_plan_destroy", "fop_status_str",
+               "fop_last_error", "fop_plan_peer_bytes", "fop_run_peer", "fop_peer_alloc", "fop_peer_free",
+               "fop_peer_open", "fop_peer_close"]
 
 
 class FopError(RuntimeError):
@@ -253,6 +280,8 @@ class FusedOp:
         self.names = list(desc["tensors"].keys())
         self.loops = list(desc["loops"].keys())
         self._c_desc = marshal(desc)
+        if isinstance(opts.get("peer_loop"), str):
+            opts["peer_loop"] = self.loops.index(opts["peer_loop"])
         self._opts = default_opts(**opts)
         h = C.c_void_p()
         _check(_lib.fop_plan(C.byref(self._c_desc), C.byref(self._opts), C.byref(h)))
@@ -294,7 +323,8 @@ class FusedOp:
                              "read_loop": ln(li.read_loop), "read_width": li.read_width,
                              "coal_loop": ln(li.coal_loop), "grid": li.grid, "block": li.block,
                              "seq": [ln(li.seq[q]) for q in range(li.nseq)],
-                             "scen_pick": li.scen_pick, "fallback": li.fallback})
+                             "scen_pick": li.scen_pick, "fallback": li.fallback,
+                             "peer_exchange": bool(li.peer_exchange)})
         return {"stmts": stmts, "launches": launches, "workspace_bytes": pi.workspace_bytes}
 
     @property
@@ -321,6 +351,11 @@ class FusedOp:
     def workspace_bytes(self):
         return _lib.fop_plan_workspace_bytes(self._h)
 
+    @property
+    def peer_bytes(self):
+        """Exchange-buffer size of a plan with opts.peer_world >= 1 (else 0)."""
+        return _lib.fop_plan_peer_bytes(self._h)
+
     # ------------------------------------------------------------ execution
     def _workspace(self, device):
         import torch
@@ -346,13 +381,18 @@ class FusedOp:
             dev = t.device
         return arr, dev
 
-    def run(self, tensors, workspace=None, stream=None):
-        """Enqueue the fused operator on `stream` (default: torch's current stream)."""
+    def run(self, tensors, workspace=None, stream=None, peers=None):
+        """Enqueue the fused operator on `stream` (default: torch's current stream).
+        peers: a PeerGroup for plans with a cross-GPU exchange (fop_run_peer)."""
         import torch
         arr, dev = self._ptrs(tensors)
         ws = workspace if workspace is not None else self._workspace(dev)
         if stream is None:
             stream = torch.cuda.current_stream(dev)
+        if peers is not None:
+            _check(_lib.fop_run_peer(self._h, arr, len(self.names), None if ws is None else ws.data_ptr(),
+                                     C.byref(peers.c), stream.cuda_stream))
+            return
         _check(_lib.fop_run(self._h, arr, len(self.names),
                             None if ws is None else ws.data_ptr(), stream.cuda_stream))
 
@@ -406,6 +446,46 @@ def run_host_many(items, stream=None):
     if stream is None:
         stream = torch.cuda.current_stream(dev)
     _check(_lib.fop_run_host_many(plans, hp, dp, np_, ws, n, stream.cuda_stream))
+
+
+# ---------------------------------------------------------------- peer groups (fop.h)
+class PeerGroup:
+    """fop_peer_group: this GPU's rank and every rank's exchange buffer as
+    addressed from this process (device pointers as ints)."""
+
+    def __init__(self, rank, bufs):
+        if not 0 <= rank < len(bufs) <= MAX_PEERS:
+            raise ValueError("rank/world out of range")
+        self.rank, self.world = rank, len(bufs)
+        self.bufs = list(bufs)
+        self.c = PeerGroupC()
+        self.c.rank, self.c.world = rank, len(bufs)
+        for q, b in enumerate(bufs):
+            self.c.buf[q] = b
+
+
+def peer_alloc(nbytes):
+    """Zero-filled exchange buffer on the current device: (device pointer, 64-byte IPC handle)."""
+    p, h = C.c_void_p(), IpcHandle()
+    _check(_lib.fop_peer_alloc(nbytes, C.byref(p), C.byref(h)))
+    return p.value, bytes(h.bytes)
+
+
+def peer_free(ptr):
+    _check(_lib.fop_peer_free(ptr))
+
+
+def peer_open(handle):
+    """Map another process's exchange buffer (CUDA IPC; NVLink peer access)."""
+    h = IpcHandle()
+    C.memmove(h.bytes, bytes(handle), 64)
+    p = C.c_void_p()
+    _check(_lib.fop_peer_open(C.byref(h), C.byref(p)))
+    return p.value
+
+
+def peer_close(ptr):
+    _check(_lib.fop_peer_close(ptr))
 
 
 def abi_version():
