@@ -290,9 +290,10 @@ FOP_API fop_status  fop_run_host_many(const fop_plan_t* const* plans, void* cons
  * owner, the 64-byte handle sent to the others by any means, fop_peer_open
  * there; CUDA IPC, so peers are GPUs of one node reached over NVLink /
  * NVSwitch).  Layout of a buffer, per exchanging launch: [2 parities][world
- * senders][slabs][slab columns] fp32 partial sums, then [slabs][world] arrival
- * epochs (written by the senders, release at system scope), then [slabs] local
- * run counters; the LAST 16 bytes hold an error word (nonzero = a wait timed
+ * senders][slabs][slab columns] 64-bit words (fp32 partial sum in the low
+ * half, the run's epoch in the high half: one single-copy-atomic store
+ * carries both the value and its arrival flag), then [slabs] local run
+ * counters; the LAST 16 bytes hold an error word (nonzero = a wait timed
  * out).  The kernels keep the buffer consistent across runs: the buffer must
  * not be touched between runs, and every rank must run the plan the same
  * number of times, in the same order relative to the plan's other runs. */

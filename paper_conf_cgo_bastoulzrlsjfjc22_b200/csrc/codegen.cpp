@@ -1546,6 +1546,13 @@ struct Gen {
     o.l("__shared__ unsigned last_flag;");
     o.l("const unsigned tid = threadIdx.x, cv = tid % " + num(L.gv) + "u, rl = tid / " + num(L.gv) + "u;");
     o.l("const idx_t slab = blockIdx.x % " + num(slabs) + "u, chunk = blockIdx.x / " + num(slabs) + "u;");
+    // peer exchange: the slab's run counter, read in the epilogue (FOP_PEER_EP=0, default) or at kernel
+    // start (1: volatile load, measured 4 us slower on cfg4b; 2: ld.global.cg)
+    const int peer_ep = L.peer ? geometry_knob(L, "FOP_PEER_EP", 0) : 0;
+    if (peer_ep)
+      o.l(std::string("const unsigned xep0_ = ") + (peer_ep == 1 ? "((volatile const unsigned*)" : "__ldcg((const unsigned*)") +
+          "(args.peer[args.rank] + " + num((int64_t)L.peer_off) + "ull + " +
+          num((int64_t)peer_layout(L, p.opts.peer_world).epoch) + "ull)" + (peer_ep == 1 ? ")[slab];" : " + slab);"));
     o.l("idx_t sr = slab;");
     o.l("const idx_t sv = sr % " + num(SVN) + "u; sr /= " + num(SVN) + "u;");
     std::vector<std::pair<int, std::string>> cits;
@@ -1745,60 +1752,74 @@ struct Gen {
     };
     tree();
     // Cross-GPU combine (opts.peer_world >= 1, fop.h peer groups; SURVEY
-    // §8(e)): the block holding this rank's slab sums in red[0 .. SW) pushes
-    // them into slot [parity][rank][slab] of every rank's exchange buffer
-    // (NVLink stores), publishes one epoch flag per receiver (release, system
-    // scope), waits for every rank's flag in its own buffer (acquire), and
-    // sums the world contributions in rank order — the same order on every
-    // rank, so all ranks store identical bits.  The epoch is a per-slab run
-    // counter kept in the local buffer; the two parities let a rank run ahead
-    // by one run without overwriting data a slower rank has not read yet (it
-    // cannot get further: its next wait needs that rank's next push).
+    // §8(e)).  The block holding this rank's slab sums in red[0 .. SW)
+    // pushes each sum, packed with the run's epoch into one 64-bit word
+    // (single-copy atomic, so the epoch doubles as the arrival flag: no
+    // separate flag, fence or release round trip), into slot
+    // [parity][rank][slab][e] of every rank's exchange buffer (NVLink stores
+    // into peer memory), then polls its own buffer until every rank's words
+    // carry this epoch and sums the world contributions in rank order — the
+    // same order on every rank, so all ranks store identical bits.  The epoch
+    // is a per-slab run counter kept in the local buffer (read at kernel
+    // start); the two parities let a rank run ahead by one run without
+    // overwriting words a slower rank has not read yet (it cannot get
+    // further: its next wait needs that rank's next push).
     auto exchange = [&]() {
       if (!L.peer) return;
       const int PW = p.opts.peer_world;
       const PeerLayout pl = peer_layout(L, PW);
       const int64_t S = L.peer_slabs;
+      const int NP = PW * SW;                         // words this block receives
+      const int K = (NP + L.block - 1) / L.block;     // per thread
       const unsigned long long lim =
           (unsigned long long)(p.opts.peer_timeout_ms > 0 ? p.opts.peer_timeout_ms : 10000) * 1000000ull;
       const std::string base = num((int64_t)L.peer_off);
+      const int spins = geometry_knob(L, "FOP_PEER_SPIN", 64);
       o.l("{");
       o.ind++;
-      o.l("__shared__ unsigned xep_, xok_;");
-      o.l("char* const xb_ = args.peer[args.rank] + " + base + "ull;");
-      o.l("if (tid == 0u) {");
-      o.l("  volatile unsigned* c_ = (volatile unsigned*)(xb_ + " + num((int64_t)pl.epoch) + "ull) + slab;");
-      o.l("  xep_ = *c_ + 1u;");
-      o.l("  *c_ = xep_;");
-      o.l("  xok_ = 1u;");
-      o.l("}");
-      o.l("__syncthreads();");
-      o.l("const unsigned xe_ = xep_, xp_ = xe_ & 1u;");
-      o.l("for (unsigned i_ = tid; i_ < " + num(PW * SW) + "u; i_ += " + num(L.block) + "u) {");
+      o.l("__shared__ float xv_[" + num(NP) + "];");
+      if (!geometry_knob(L, "FOP_PEER_EP", 0))
+        o.l("const unsigned xep0_ = ((volatile const unsigned*)(args.peer[args.rank] + " + base + "ull + " +
+            num((int64_t)pl.epoch) + "ull))[slab];");
+      o.l("const unsigned xe_ = xep0_ + 1u, xp_ = xe_ & 1u;");
+      o.l("const u64* const xb_ = (const u64*)(args.peer[args.rank] + " + base + "ull);");
+      o.l("if (tid == 0u) ((volatile unsigned*)(args.peer[args.rank] + " + base + "ull + " + num((int64_t)pl.epoch) +
+          "ull))[slab] = xe_;");
+      o.l("for (unsigned i_ = tid; i_ < " + num(NP) + "u; i_ += " + num(L.block) + "u) {");
       o.l("  const unsigned q_ = i_ / " + num(SW) + "u, e_ = i_ % " + num(SW) + "u;");
-      o.l("  float* d_ = (float*)(args.peer[q_] + " + base + "ull) + ((xp_ * " + num(PW) + "u + args.rank) * " + num(S) +
+      o.l("  u64* d_ = (u64*)(args.peer[q_] + " + base + "ull) + ((xp_ * " + num(PW) + "u + args.rank) * " + num(S) +
           "ull + slab) * " + num(SW) + "u + e_;");
-      o.l("  *d_ = red[e_];");
+      o.l("  fop::st_relaxed_sys_u64(d_, ((u64)xe_ << 32) | __float_as_uint(red[e_]));");
       o.l("}");
-      o.l("__syncthreads();");
-      o.l("if (tid < " + num(PW) + "u) {");
-      o.l("  __threadfence_system();");
-      o.l("  fop::st_release_sys((unsigned*)(args.peer[tid] + " + base + "ull + " + num((int64_t)pl.flags) + "ull) + slab * " +
-          num(PW) + "u + args.rank, xe_);");
-      o.l("  if (!fop::wait_epoch((const unsigned*)(xb_ + " + num((int64_t)pl.flags) + "ull) + slab * " + num(PW) +
-          "u + tid, xe_, " + std::to_string(lim) + "ull)) {");
-      o.l("    xok_ = 0u;");
-      o.l("    atomicExch((unsigned*)(args.peer[args.rank] + " + num((int64_t)(p.peer_bytes - 16)) + "ull), 1u);");
+      o.l("int xok_ = 1;");
+      o.l("u64 xw_[" + num(K) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int k = 0; k < " + num(K) + "; ++k) {   // every word requested before the first is checked");
+      o.l("  const unsigned i_ = tid + k * " + num(L.block) + "u;");
+      o.l("  if (i_ < " + num(NP) + "u) xw_[k] = fop::ld_relaxed_sys_u64(xb_ + ((xp_ * " + num(PW) + "u + i_ / " +
+          num(SW) + "u) * " + num(S) + "ull + slab) * " + num(SW) + "u + i_ % " + num(SW) + "u);");
+      o.l("}");
+      o.l("#pragma unroll");
+      o.l("for (int k = 0; k < " + num(K) + "; ++k) {");
+      o.l("  const unsigned i_ = tid + k * " + num(L.block) + "u;");
+      o.l("  if (i_ < " + num(NP) + "u) {");
+      o.l("    const u64* a_ = xb_ + ((xp_ * " + num(PW) + "u + i_ / " + num(SW) + "u) * " + num(S) + "ull + slab) * " +
+          num(SW) + "u + i_ % " + num(SW) + "u;");
+      o.l("    if ((unsigned)(xw_[k] >> 32) != xe_ && !fop::wait_word(a_, xe_, xw_[k], " + std::to_string(lim) + "ull, " +
+          num(spins) + ")) {");
+      o.l("      xok_ = 0;");
+      o.l("      atomicExch((unsigned*)(args.peer[args.rank] + " + num((int64_t)(p.peer_bytes - 16)) + "ull), 1u);");
+      o.l("    }");
+      o.l("    xv_[i_] = __uint_as_float((unsigned)xw_[k]);");
       o.l("  }");
       o.l("}");
-      o.l("__syncthreads();");
+      o.l("xok_ = __syncthreads_and(xok_);");
       o.l("if (rl == 0u) {");
       o.l("  #pragma unroll");
       o.l("  for (int e = 0; e < " + num(W) + "; ++e) {");
       o.l("    float s_ = " + init + ";");
-      o.l("    for (unsigned q_ = 0; q_ < " + num(PW) + "u; ++q_)");
-      o.l("      s_ = " + comb("s_", "fop::ld_relaxed_sys((const float*)xb_ + ((xp_ * " + num(PW) + "u + q_) * " + num(S) +
-                                  "ull + slab) * " + num(SW) + "u + cv * " + num(W) + "u + e)") + ";");
+      o.l("    for (unsigned q_ = 0; q_ < " + num(PW) + "u; ++q_) s_ = " +
+          comb("s_", "xv_[q_ * " + num(SW) + "u + cv * " + num(W) + "u + e]") + ";");
       o.l("    red[cv * " + num(W) + "u + e] = xok_ ? s_ : __int_as_float(0x7fc00000);");
       o.l("  }");
       o.l("}");

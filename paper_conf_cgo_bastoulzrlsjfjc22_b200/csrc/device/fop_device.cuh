@@ -540,39 +540,41 @@ __device__ __forceinline__ void sts128(u32 addr, u32 a, u32 b, u32 c, u32 d) {
 }
 
 // ---------------------------------------------------------------- peer exchange (multi-GPU)
-// Cross-GPU reduction in a COL_REDUCE epilogue (fop.h, peer groups): plain
-// stores of the partial sums into every rank's exchange buffer (NVLink peer
-// memory), then per receiver one epoch flag stored with release semantics at
-// system scope; receivers poll their own flags with acquire loads.  The
-// block-wide barrier between the data stores and the flag store makes the
-// other threads' stores part of what the release publishes (the same pattern
-// as a grid barrier, at system scope).
-__device__ __forceinline__ void st_release_sys(unsigned* p, unsigned v) {
-  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+// Cross-GPU reduction in a COL_REDUCE epilogue (fop.h, peer groups): each
+// partial sum travels as ONE 64-bit word (fp32 bits | epoch << 32) stored
+// into the receiver's exchange buffer over NVLink.  An aligned 64-bit
+// access is single-copy atomic, so a receiver that reads the current epoch
+// in the high half has the matching sum in the low half: the epoch is the
+// arrival flag (no separate flag store, fence or release/acquire round trip).
+__device__ __forceinline__ void st_relaxed_sys_u64(u64* p, u64 v) {
+  asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
-__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
-  unsigned v;
-  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+__device__ __forceinline__ u64 ld_relaxed_sys_u64(const u64* p) {
+  u64 v;
+  asm volatile("ld.relaxed.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
-__device__ __forceinline__ float ld_relaxed_sys(const float* p) {
-  float v;
-  asm volatile("ld.relaxed.sys.global.f32 %0, [%1];" : "=f"(v) : "l"(p) : "memory");
-  return v;
-}
-// Wait until *flag has reached epoch `ep` (wrap-safe); false after ~limit_ns.
-__device__ __forceinline__ bool wait_epoch(const unsigned* flag, unsigned ep, unsigned long long limit_ns) {
+// Poll *p until its epoch half equals ep (the word lands in `w`); false after
+// ~limit_ns.  The first `spins` polls do not sleep (a peer that is about to
+// arrive costs one round trip, not a scheduler wake-up).
+__device__ __forceinline__ bool wait_word(const u64* p, unsigned ep, u64& w, unsigned long long limit_ns,
+                                          int spins) {
+  for (int k = 0; k < spins; ++k) {
+    w = ld_relaxed_sys_u64(p);
+    if ((unsigned)(w >> 32) == ep) return true;
+  }
   unsigned long long t0 = 0;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
   unsigned ns = 32;
-  while ((int)(ld_acquire_sys(flag) - ep) < 0) {
+  for (;;) {
+    w = ld_relaxed_sys_u64(p);
+    if ((unsigned)(w >> 32) == ep) return true;
     unsigned long long t = 0;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     if (t - t0 > limit_ns) return false;
     __nanosleep(ns);
-    if (ns < 1024) ns *= 2;
+    if (ns < 256) ns *= 2;
   }
-  return true;
 }
 
 }  // namespace fop

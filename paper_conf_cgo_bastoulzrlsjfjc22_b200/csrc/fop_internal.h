@@ -173,19 +173,17 @@ struct Launch {
 };
 
 // Exchange-buffer region of a peer-exchanging COL_REDUCE launch (fop.h, peer
-// groups): [2 parities][world][slabs][SW] fp32 | [slabs][world] u32 epochs
-// written by the senders | [slabs] u32 local run counters.  Offsets relative
-// to Launch::peer_off.
+// groups): [2 parities][world][slabs][SW] u64 words (fp32 sum | epoch << 32)
+// | [slabs] u32 local run counters.  Offsets relative to Launch::peer_off.
 struct PeerLayout {
-  size_t data = 0, flags = 0, epoch = 0, total = 0;
+  size_t data = 0, epoch = 0, total = 0;
 };
 inline PeerLayout peer_layout(const Launch& L, int world) {
   auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
   PeerLayout r;
   const size_t sw = (size_t)L.gv * (size_t)L.width;
   r.data = 0;
-  r.flags = al(2 * (size_t)world * (size_t)L.peer_slabs * sw * sizeof(float));
-  r.epoch = r.flags + al((size_t)L.peer_slabs * (size_t)world * sizeof(unsigned));
+  r.epoch = al(2 * (size_t)world * (size_t)L.peer_slabs * sw * sizeof(uint64_t));
   r.total = r.epoch + al((size_t)L.peer_slabs * sizeof(unsigned));
   return r;
 }

@@ -46,9 +46,9 @@ def test_peer_plan_layout():
     op = FusedOp(W.cfg4b(8192, 1024), peer_world=4, peer_loop="r", jit=0)
     L = op.info()["launches"]
     assert len(L) == 1 and L[0]["class"] == "col_reduce" and L[0]["peer_exchange"]
-    # slab = 8 lanes x 8 f16 = 64 columns -> 16 slabs; [2][4][16][64] f32 | [16][4] u32 | [16] u32 | error word
+    # slab = 8 lanes x 8 f16 = 64 columns -> 16 slabs; [2][4][16][64] u64 | [16] u32 | error word
     al = lambda x: (x + 255) // 256 * 256  # noqa: E731
-    assert op.peer_bytes == al(2 * 4 * 16 * 64 * 4) + al(16 * 4 * 4) + al(16 * 4) + 16
+    assert op.peer_bytes == al(2 * 4 * 16 * 64 * 8) + al(16 * 4) + 16
     assert FusedOp(W.cfg4b(8192, 1024), jit=0).peer_bytes == 0
 
 
@@ -56,7 +56,7 @@ def test_peer_plan_has_no_tuning_variants():
     op = FusedOp(W.cfg4b(4096, 256), peer_world=2, peer_loop="r")
     assert op.selected(0)[0].endswith("_k0")
     src = op.source(0)
-    assert "st_release_sys" in src and "wait_epoch" in src
+    assert "st_relaxed_sys_u64" in src and "wait_word" in src
 
 
 def test_peer_parallel_loop_needs_no_exchange():
@@ -111,28 +111,25 @@ def test_shard_desc_fused_allows_finalize():
 # ---------------------------------------------------------------- CPU: protocol model
 def _simulate(world, runs, seed):
     """Random interleaving of the kernel epilogue's steps on `world` ranks
-    (each rank's runs in stream order).  Checks that every wait reads, from
-    every sender, exactly that sender's data of the same run."""
+    (each rank's runs in stream order).  Every word carries (value, epoch)
+    atomically; a receiver polls each word until its epoch is the run's.
+    Checks that every accepted word is that sender's value of the same run."""
     rng = random.Random(seed)
-    data = [[[None] * world for _ in range(2)] for _ in range(world)]   # data[recv][parity][sender]
-    flags = [[0] * world for _ in range(world)]                         # flags[recv][sender]
+    words = [[[(None, 0)] * world for _ in range(2)] for _ in range(world)]   # [recv][parity][sender]
     ctr = [0] * world
 
     def rank_prog(r):
         for run in range(runs):
-            ctr[r] += 1
-            ep = ctr[r]
+            ep = ctr[r] + 1
+            ctr[r] = ep
             assert ep == run + 1
             for q in rng.sample(range(world), world):       # stores land in any order
-                data[q][ep & 1][r] = (r, ep)
+                words[q][ep & 1][r] = ((r, ep), ep)
                 yield
-            for q in rng.sample(range(world), world):       # flags after all data (release)
-                flags[q][r] = ep
-                yield
-            while any(flags[r][q] - ep < 0 for q in range(world)):
-                yield                                       # acquire-poll
-            for q in range(world):
-                assert data[r][ep & 1][q] == (q, ep), (r, q, ep, data[r][ep & 1][q])
+            for q in rng.sample(range(world), world):       # polls in any order
+                while words[r][ep & 1][q][1] != ep:
+                    yield
+                assert words[r][ep & 1][q][0] == (q, ep), (r, q, ep, words[r][ep & 1][q])
                 yield
     progs = {r: rank_prog(r) for r in range(world)}
     while progs:
