@@ -250,7 +250,29 @@ def run_fop(args):
             o["op"].run(o["dev"], stream=stream)
             allreduce(o)
 
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import run_many
+    many = [(o["op"], o["dev"]) for o in ops if o["px"] is None]
+
+    def chain(st):
+        # the independent ops as one chain (fop_run_many: each op's launch is
+        # processed while the previous kernel runs), then the op whose
+        # partials are combined across GPUs inside its kernel (N > 1)
+        run_many(many, stream=st)
+        for o in ops:
+            if o["px"] is not None:
+                o["op"].run(o["dev"], stream=st, peers=o["px"].peers)
+            else:
+                allreduce(o)
+
+    graph = None
+
     def step(events=None):
+        if events is None and graph is not None:
+            graph.replay()
+            return
+        if events is None and not args.no_pdl:
+            chain(stream)
+            return
         for i, o in enumerate(ops):
             if events is not None:
                 events[i][0].record(stream)
@@ -261,6 +283,23 @@ def run_fop(args):
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
+    # One step as a CUDA graph (kernels tuned during the warm-up): replays
+    # without per-kernel launch gaps.  Not with a host-side collective in the
+    # step (--exchange nccl over gloo / NCCL) — that path stays eager.
+    host_collective = world > 1 and args.exchange == "nccl"
+    if not args.no_graph and not args.no_pdl and not host_collective:
+        g = torch.cuda.CUDAGraph()
+        cap = torch.cuda.Stream(dev)
+        cap.wait_stream(stream)
+        with torch.cuda.stream(cap):
+            with torch.cuda.graph(g, stream=cap):
+                chain(cap)
+        stream.wait_stream(cap)
+        torch.cuda.synchronize()
+        graph = g
+        for _ in range(args.warmup):
+            step()
+        torch.cuda.synchronize()
 
     # ---- timed region: K steps between barrier + sync, CUDA events on the launch stream
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -383,9 +422,14 @@ def run_fop(args):
                     if peer else "cfg4b partials all-reduced over NCCL)"),
                 "l2": "no flush: every input is re-read once per step after >1 GB of other ops' traffic "
                       "(B200 L2 126 MB); cfg2/cfg3 inputs alone exceed L2",
-                "per_op_note": "per-op times come from a second pass of the same K steps with CUDA events "
-                               "around each op; an op also pays the write-back of dirty L2 lines the "
-                               "previous op left (e.g. cfg4b after cfg4a's 50 MB y)",
+                "launch": ("fop_run per op" if args.no_pdl else
+                           ("one CUDA graph per step: " if graph is not None else "eager: ") +
+                           "fop_run_many (the independent ops as one chain, launches with programmatic stream "
+                           "serialization)" + (" + fop_run_peer (cfg4b, in-kernel cross-GPU combine)" if peer else
+                                                " + NCCL all-reduce of cfg4b's partials" if world > 1 else "")),
+                "per_op_note": "per-op times come from a second pass of the same K steps with fop_run per op "
+                               "and CUDA events around each (no overlap); an op also pays the write-back of "
+                               "dirty L2 lines the previous op left (e.g. cfg4b after cfg4a's 50 MB y)",
                 "per_op": per_op_json,
                 "peak_gbs": peak, "peak_source": peak_src,
             },
@@ -420,6 +464,9 @@ def main():
     ap.add_argument("--vec-bytes", type=int, default=0, help="16 or 32 (default: planner default 16)")
     ap.add_argument("--order", choices=["paper", "memory"], default=None)
     ap.add_argument("--no-cpu", action="store_true", help="skip the oracle cpu_baseline leg")
+    ap.add_argument("--no-pdl", action="store_true",
+                    help="launch the ops one by one (fop_run each) instead of one fop_run_many chain")
+    ap.add_argument("--no-graph", action="store_true", help="eager steps instead of replaying a CUDA graph")
     ap.add_argument("--exchange", choices=["peer", "nccl"], default="peer",
                     help="N > 1: combine cfg4b's partial sums inside the kernel over NVLink (peer) or NCCL after it")
     args = ap.parse_args()

@@ -325,6 +325,17 @@ FOP_API fop_status  fop_peer_free(void* dev_ptr);
 FOP_API fop_status  fop_peer_open(const fop_ipc_handle* handle, void** dev_ptr);
 FOP_API fop_status  fop_peer_close(void* dev_ptr);
 
+/* fop_run for n INDEPENDENT plans (no plan reads or writes what another
+ * writes), back to back on `stream` in the given order: plan k's first kernel
+ * is launched with programmatic stream serialization (its launch is
+ * processed while plan k-1's last kernel still runs; the kernels carry no
+ * explicit trigger, so plan k starts when plan k-1 completes and stream
+ * order is kept; later work on `stream` sees every result).  dev_ptrs[k],
+ * nptrs[k], workspaces[k] (may be NULL) as in fop_run.  Plans with a peer
+ * exchange are rejected (FOP_E_INVALID): run them with fop_run_peer. */
+FOP_API fop_status  fop_run_many(const fop_plan_t* const* plans, void* const* const* dev_ptrs,
+                                 const int32_t* nptrs, void* const* workspaces, int32_t n, void* stream);
+
 /* The kernel fop_run launches for `launch` on the current CUDA context (after
  * auto-tuning; the default geometry before the first run): its name, grid and
  * block.  Pointers stay owned by the plan. */

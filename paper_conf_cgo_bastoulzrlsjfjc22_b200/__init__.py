@@ -10,7 +10,7 @@ The binding (and libfop.so) is loaded on first use of an exported name, so
 library exists.
 """
 _EXPORTS = ("FusedOp", "FopError", "abi_version", "marshal", "default_opts", "ABI_SYMBOLS", "LIB_PATH",
-            "run_host_many", "PeerGroup", "peer_alloc", "peer_free", "peer_open", "peer_close")
+            "run_host_many", "run_many", "PeerGroup", "peer_alloc", "peer_free", "peer_open", "peer_close")
 
 __all__ = list(_EXPORTS)
 

@@ -2,6 +2,7 @@
 // Every entry point converts internal failures into a fop_status plus a
 // thread-local message; nothing throws or aborts across the ABI.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <exception>
 #include <new>
@@ -87,8 +88,10 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
         N.cubin.clear();
         N.src.clear();
         fop::finalize_launch_geometry(p, N);
-        N.ws_off = p.launches[i].ws_off;
-        if (N.ws_bytes > p.launches[i].ws_bytes) {
+        // a region of its own: kernels of another geometry place partial sums
+        // and arrival counters at other offsets, so sharing a region would
+        // let one variant's partials overwrite another's counters
+        if (N.ws_bytes) {
           N.ws_off = (p.ws_bytes + 255) & ~size_t(255);
           p.ws_bytes = N.ws_off + N.ws_bytes;
         }
@@ -123,11 +126,7 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
             V.src.clear();
             V.name_suffix = "_v" + std::to_string(k);
             fop::finalize_launch_geometry(p, V);
-            V.ws_off = p.launches[i].ws_off;
-            if (V.ws_bytes > p.launches[i].ws_bytes) {
-              V.ws_off = (p.ws_bytes + 255) & ~size_t(255);
-              p.ws_bytes = V.ws_off + V.ws_bytes;
-            }
+            V.ws_off = p.launches[i].ws_off;   // provisional: the duplicate check compares sources
             fop::generate(p, V, (int)i);
             // identical geometry up to the name: nothing to tune
             std::string body = V.src;
@@ -135,6 +134,12 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
               body.erase(q, V.name_suffix.size());
             if (std::find(seen.begin(), seen.end(), body) != seen.end()) continue;
             seen.push_back(body);
+            if (V.ws_bytes) {   // a region of its own (see the narrow variants above)
+              V.ws_off = (p.ws_bytes + 255) & ~size_t(255);
+              p.ws_bytes = V.ws_off + V.ws_bytes;
+              V.src.clear();
+              fop::generate(p, V, (int)i);
+            }
             fop::jit_compile(V);
             p.variants[i].push_back(V);
           }
@@ -242,6 +247,27 @@ fop_status fop_run_host_many(const fop_plan_t* const* plans, void* const* const*
       ps[k] = &const_cast<fop_plan_t*>(plans[k])->p;
     }
     return fop::run_host_many(ps.data(), host_ptrs, dev_ptrs, nptrs, workspaces, n, stream);
+  });
+}
+
+fop_status fop_run_many(const fop_plan_t* const* plans, void* const* const* dev_ptrs, const int32_t* nptrs,
+                        void* const* workspaces, int32_t n, void* stream) {
+  return guarded([&] {
+    if (n > 0 && (!plans || !dev_ptrs || !nptrs)) fop::fail(FOP_E_INVALID, "NULL argument");
+    for (int k = 0; k < n; k++) {
+      if (!plans[k] || !dev_ptrs[k]) fop::fail(FOP_E_INVALID, "NULL plan or pointer table at " + std::to_string(k));
+      if (plans[k]->p.peer_bytes) fop::fail(FOP_E_INVALID, "plan " + std::to_string(k) + " has a peer exchange: use fop_run_peer");
+    }
+    const char* pe = std::getenv("FOP_RUN_MANY_PDL");   // 0: plain launches (ablation)
+    bool first = true;
+    if (pe && *pe == '0') first = true;
+    for (int k = 0; k < n; k++) {
+      if (pe && *pe == '0') first = true;
+      fop::Plan& p = const_cast<fop_plan_t*>(plans[k])->p;
+      fop::run_plan(p, dev_ptrs[k], nptrs[k], workspaces ? workspaces[k] : nullptr, stream, nullptr, nullptr, !first);
+      if (!p.launches.empty()) first = false;
+    }
+    return FOP_OK;
   });
 }
 

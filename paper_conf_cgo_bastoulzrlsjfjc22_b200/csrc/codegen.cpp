@@ -319,8 +319,16 @@ struct Gen {
           num(t) + " = args.p[" + num(t) + "];");
     }
     o.l("const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;");
+    if ((geometry_knob(L, "FOP_PDL_EMIT", 0) & 1) && geometry_knob(L, "FOP_PDL_POS", 1) == 0)
+      o.l("fop::pdl_trigger();");
   }
   void footer() {
+    const int emit = geometry_knob(L, "FOP_PDL_EMIT", 0);
+    if ((emit & 1) && geometry_knob(L, "FOP_PDL_POS", 1) == 1) o.l("fop::pdl_trigger();");
+    if (emit & 2) {
+      if (geometry_knob(L, "FOP_PDL_WAITALL", 0)) o.l("fop::pdl_wait();");
+      else o.l("if (blockIdx.x == 0u && threadIdx.x == 0u) fop::pdl_wait();");
+    }
     o.ind--;
     o.l("}");
   }
@@ -1086,6 +1094,8 @@ struct Gen {
     o.l("unsigned char* sout = sin + " + num(S * 8192) + ";");
     o.l("u64* full = (u64*)(smem + " + num(NW * (S + 2) * 8192) + ") + wid * " + num(S) + "u;");
     o.l("const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;");
+    if ((geometry_knob(L, "FOP_PDL_EMIT", 0) & 1) && geometry_knob(L, "FOP_PDL_POS", 1) == 0)
+      o.l("fop::pdl_trigger();");
     for (int t = 0; t < d.ntensors; t++) {
       bool used = false;
       for (size_t k = 0; k < L.loads.size(); k++) used |= (int)k != ktr && L.loads[k].tensor == t;

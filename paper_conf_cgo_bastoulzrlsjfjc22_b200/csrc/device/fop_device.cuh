@@ -539,6 +539,19 @@ __device__ __forceinline__ void sts128(u32 addr, u32 a, u32 b, u32 c, u32 d) {
   asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
 }
 
+// ---------------------------------------------------------------- programmatic dependent launch
+// Explicit PDL control, emitted only with FOP_PDL_EMIT (ablation): bit 1 =
+// trigger dependents (at block end, or at start with FOP_PDL_POS=0), bit 2 =
+// wait for the predecessor before completing.  Measured on the bench suite
+// (tools/pdl_time.py): 357 us/step with them vs 277 us without — a dependent
+// grid that launches early competes with the primary's statically
+// partitioned one-wave grid — so by default kernels carry neither and
+// fop_run_many's launches only get programmatic stream serialization, whose
+// implicit trigger at the primary's completion keeps stream order while the
+// dependent's launch is processed early.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // ---------------------------------------------------------------- peer exchange (multi-GPU)
 // Cross-GPU reduction in a COL_REDUCE epilogue (fop.h, peer groups): each
 // partial sum travels as ONE 64-bit word (fp32 bits | epoch << 32) stored

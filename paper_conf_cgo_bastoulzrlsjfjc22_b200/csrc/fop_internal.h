@@ -230,7 +230,7 @@ bool jit_available();
 fop_status run_host_many(Plan* const* plans, void* const* const* host_ptrs, void* const* const* dev_ptrs,
                          const int32_t* nptrs, void* const* ws, int n, void* stream);
 fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream,
-                    void* const* host_ptrs, const fop_peer_group* peers = nullptr);
+                    void* const* host_ptrs, const fop_peer_group* peers = nullptr, bool pdl = false);
 void peer_alloc(size_t bytes, void** dev_ptr, fop_ipc_handle* handle);
 void peer_free(void* dev_ptr);
 void peer_open(const fop_ipc_handle* handle, void** dev_ptr);

@@ -9,7 +9,9 @@
 
 #include <algorithm>
 
+#include <cstddef>
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
@@ -53,6 +55,7 @@ struct Cuda {
   CUresult (*stream_capturing)(CUstream, int*);
   CUresult (*stream_create)(CUstream*, unsigned);
   CUresult (*stream_wait)(CUstream, void*, unsigned);
+  CUresult (*launch_ex)(const void* config, CUfunction, void**, void**);
   CUresult (*mem_alloc)(CUdeviceptr*, size_t);
   CUresult (*mem_free)(CUdeviceptr);
   CUresult (*memset8)(CUdeviceptr, unsigned char, size_t);
@@ -64,6 +67,22 @@ struct Cuda {
                           const unsigned*, int, int, int, int);
 };
 enum { CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES = 8 };
+// cuLaunchKernelEx configuration (layout of cuda.h's CUlaunchConfig /
+// CUlaunchAttribute; the attribute value is a 64-byte union)
+struct LaunchAttr {
+  int id;
+  char pad[4];
+  unsigned char value[64];
+};
+struct LaunchConfig {
+  unsigned grid[3], block[3], smem;
+  CUstream stream;
+  LaunchAttr* attrs;
+  unsigned nattrs;
+};
+enum { CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION = 6 };
+static_assert(sizeof(LaunchAttr) == 72, "CUlaunchAttribute layout");
+static_assert(offsetof(LaunchConfig, stream) == 32 && offsetof(LaunchConfig, nattrs) == 48, "CUlaunchConfig layout");
 enum { TMAP_UINT16 = 1, TMAP_INTERLEAVE_NONE = 0, TMAP_SWIZZLE_128B = 3, TMAP_L2_PROMO_256B = 3, TMAP_OOB_NONE = 0 };
 
 Cuda& cuda() {
@@ -102,6 +121,7 @@ Cuda& cuda() {
     SYM(stream_create, "cuStreamCreate");
     SYM(stream_wait, "cuStreamWaitEvent");
     SYM(tmap_encode, "cuTensorMapEncodeTiled");
+    SYM(launch_ex, "cuLaunchKernelEx");
     SYM(mem_alloc, "cuMemAlloc_v2");
     SYM(mem_free, "cuMemFree_v2");
     SYM(memset8, "cuMemsetD8_v2");
@@ -208,7 +228,7 @@ void* current_context_or_null() {
 }
 
 fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* stream, void* const* host_ptrs,
-                    const fop_peer_group* peers) {
+                    const fop_peer_group* peers, bool pdl) {
   const fop_desc& d = p.desc;
   if (nptrs != d.ntensors) fail(FOP_E_INVALID, "nptrs must equal desc.ntensors");
   if (p.peer_bytes) {   // every argument error is caught before any launch (the peers would wait)
@@ -236,6 +256,12 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
       fail(FOP_E_INVALID, "NULL pointer for tensor " + std::to_string(t));
     if (ptrs[t] && ((uintptr_t)ptrs[t] % esize(d.t[t].dtype)))
       fail(FOP_E_ALIGN, "tensor " + std::to_string(t) + " is not aligned to its element size");
+  }
+  if (const char* dbg = std::getenv("FOP_DEBUG_RUN"); dbg && *dbg == '1') {
+    std::fprintf(stderr, "[fop] run_plan ws=%p stream=%p pdl=%d nlaunch=%zu ptrs:", ws, stream, (int)pdl,
+                 p.launches.size());
+    for (int t = 0; t < nptrs; t++) std::fprintf(stderr, " %p", ptrs[t]);
+    std::fprintf(stderr, "\n");
   }
   bool any_copy = false;
   for (int t = 0; t < d.ntensors && host_ptrs; t++) any_copy |= host_ptrs[t] && span_bytes(d.t[t]) > 0;
@@ -270,6 +296,34 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
 
   std::lock_guard<std::mutex> g(p.mu);
   Plan::Loaded& l = loaded_for(p, ctx);
+  // pdl: the plan's first kernel is launched with programmatic stream
+  // serialization (fop_run_many; the caller guarantees the plans are
+  // independent).  The kernels carry no explicit trigger, so it starts when
+  // the previous kernel completes (stream order kept) but its launch is
+  // processed early (device/fop_device.cuh, programmatic dependent launch)
+  bool pdl_next = pdl;
+  auto launch = [&](CUfunction f, unsigned grid, unsigned block, unsigned smem, void** params, const char* what) {
+    if (pdl_next) {
+      pdl_next = false;
+      LaunchAttr a;
+      std::memset(&a, 0, sizeof a);
+      a.id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+      a.value[0] = 1;
+      LaunchConfig cfg;
+      std::memset(&cfg, 0, sizeof cfg);
+      cfg.grid[0] = grid;
+      cfg.grid[1] = cfg.grid[2] = 1;
+      cfg.block[0] = block;
+      cfg.block[1] = cfg.block[2] = 1;
+      cfg.smem = smem;
+      cfg.stream = st;
+      cfg.attrs = &a;
+      cfg.nattrs = 1;
+      check(c.launch_ex(&cfg, f, params, nullptr), what);
+      return;
+    }
+    check(c.launch(f, grid, 1, 1, block, 1, 1, smem, st, params, nullptr), what);
+  };
   auto launch_one = [&](Launch* G, CUfunction f) {
     if (G->tma) {  // tensor maps for this run's base addresses (cached for the last pair)
       const char* gin = args.p[G->tma_in_tensor] + G->tma_in_base * 2;
@@ -288,12 +342,11 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
         G->tma_last_out = gout;
       }
       void* params[] = {&args, &G->tma_map_in, &G->tma_map_out};
-      check(c.launch(f, (unsigned)G->grid, 1, 1, (unsigned)G->block, 1, 1, (unsigned)G->smem, st, params, nullptr),
-            "cuLaunchKernel(tma)");
+      launch(f, (unsigned)G->grid, (unsigned)G->block, (unsigned)G->smem, params, "cuLaunchKernel(tma)");
       return;
     }
     void* params[] = {&args};
-    check(c.launch(f, (unsigned)G->grid, 1, 1, (unsigned)G->block, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
+    launch(f, (unsigned)G->grid, (unsigned)G->block, 0, params, "cuLaunchKernel");
   };
 
   // Auto-tuning (opts.autotune): the first run of a launch on this context

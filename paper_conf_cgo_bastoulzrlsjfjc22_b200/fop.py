@@ -129,6 +129,9 @@ class PeerGroupC(C.Structure):
     _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("buf", C.c_void_p * MAX_PEERS)]
 
 
+_lib.fop_run_many.argtypes = [C.POINTER(C.c_void_p), C.POINTER(C.POINTER(C.c_void_p)), C.POINTER(C.c_int32),
+                              C.POINTER(C.c_void_p), C.c_int32, C.c_void_p]
+_lib.fop_run_many.restype = C.c_int
 _lib.fop_plan_peer_bytes.argtypes = [C.c_void_p]
 _lib.fop_plan_peer_bytes.restype = C.c_size_t
 _lib.fop_run_peer.argtypes = [C.c_void_p, C.POINTER(C.c_void_p), C.c_int32, C.c_void_p, C.POINTER(PeerGroupC),
@@ -148,7 +151,7 @@ _lib.fop_last_error.restype = C.c_char_p
 ABI_SYMBOLS = ["fop_abi_version", "fop_plan_opts_default", "fop_plan", "fop_plan_info_get",
                "fop_plan_workspace_bytes", "fop_plan_source", "fop_plan_cubin", "fop_run",
                "fop_run_host", "fop_run_host_many", "fop_plan_selected", "fop_plan_destroy", "fop_status_str",
-               "fop_last_error", "fop_plan_peer_bytes", "fop_run_peer", "fop_peer_alloc", "fop_peer_free",
+               "fop_last_error", "fop_run_many", "fop_plan_peer_bytes", "fop_run_peer", "fop_peer_alloc", "fop_peer_free",
                "fop_peer_open", "fop_peer_close"]
 
 
@@ -486,6 +489,33 @@ def peer_open(handle):
 
 def peer_close(ptr):
     _check(_lib.fop_peer_close(ptr))
+
+
+def run_many(items, stream=None):
+    """fop_run_many: independent operators back to back, each plan's first
+    kernel overlapping the previous one's tail (programmatic dependent
+    launch).  `items` is a list of (FusedOp, device tensors[, workspace])."""
+    import torch
+    n = len(items)
+    plans = (C.c_void_p * n)()
+    dp = (C.POINTER(C.c_void_p) * n)()
+    np_ = (C.c_int32 * n)()
+    ws = (C.c_void_p * n)()
+    keep = []
+    dev = None
+    for k, it in enumerate(items):
+        op, devt = it[0], it[1]
+        arr, d = op._ptrs(devt)
+        dev = dev or d
+        w = it[2] if len(it) > 2 and it[2] is not None else op._workspace(d)
+        keep.append(arr)
+        plans[k] = op._h
+        dp[k] = C.cast(arr, C.POINTER(C.c_void_p))
+        np_[k] = len(op.names)
+        ws[k] = None if w is None else w.data_ptr()
+    if stream is None:
+        stream = torch.cuda.current_stream(dev)
+    _check(_lib.fop_run_many(plans, dp, np_, ws, n, stream.cuda_stream))
 
 
 def abi_version():
