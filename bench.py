@@ -44,6 +44,10 @@ OPS = [("cfg2", W.cfg2, "ew"), ("cfg3", W.cfg3, "transpose"), ("cfg4a", W.cfg4a,
 GLOBAL = {"cfg2": (lambda w: W.cfg2(N=128 * w), "n"), "cfg3": (lambda w: W.cfg3(N=256 * w), "n"),
           "cfg4a": (lambda w: W.cfg4a(B=64 * w), "b"), "cfg4b": (lambda w: W.cfg4b(R=65536 * w), "r")}
 FALLBACK_HBM = 6650.0
+METRIC = "achieved HBM GB/s (fused-op suite; per-op GB/s and % of peak in config.per_op)"
+WORKLOAD = ("fused-op suite: cfg2 BN+ReLU+cast [128,64,112,112] f32->f16, cfg3 NCHW->NHWC*s "
+            "[256,256,56,56] f16, cfg4a bias+GELU+row mean/var [64,512,768] f16, cfg4b colsum "
+            "[65536,1024] f16->f32 (BASELINE.json configs[1..3]) per GPU")
 
 
 def peaks():
@@ -169,10 +173,10 @@ def run_reference(args):
         t += tt
     value = b / t / 1e9
     line = {
-        "impl": "reference", "metric": "achieved HBM GB/s (fused-op suite)", "value": value, "unit": "GB/s",
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "GB/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": t / args.steps * 1e3,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": "fused-op suite cfg2+cfg3+cfg4a+cfg4b, bounded sample", "sample": CPU_SAMPLE_TXT},
+        "config": {"workload": WORKLOAD, "global_batch_scale": 1, "sample": CPU_SAMPLE_TXT},
         "cpu_baseline": {"value": value, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": CPU_SAMPLE_TXT},
         "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -407,14 +411,12 @@ def run_fop(args):
 
     if rank == 0:
         line = {
-            "metric": "achieved HBM GB/s (fused-op suite; per-op GB/s and % of peak in config.per_op)",
+            "metric": METRIC,
             "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {
-                "workload": "fused-op suite: cfg2 BN+ReLU+cast [128,64,112,112] f32->f16, cfg3 NCHW->NHWC*s "
-                            "[256,256,56,56] f16, cfg4a bias+GELU+row mean/var [64,512,768] f16, cfg4b colsum "
-                            "[65536,1024] f16->f32 (BASELINE.json configs[1..3]) per GPU",
+                "workload": WORKLOAD,
                 "global_batch_scale": world,
                 "parallelism": ("dp%d (batch-sharded; " % world) + (
                     "no exchange)" if world == 1 else
