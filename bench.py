@@ -159,6 +159,56 @@ def cpu_oracle_step(inputs_cache):
     return total_b, total_t
 
 
+# the same sample on every host core: the oracle unchanged, one process per
+# core, each on a contiguous block of the sample's parallel loop
+# (dist.shard_desc; independent slices, no communication); reported next to
+# the 1-core number, baseline only
+SHARD_LOOP = {"cfg2": "n", "cfg3": "n", "cfg4a": "b", "cfg4b": "c"}
+
+
+def _oracle_shard(job):
+    name, k, n = job
+    from oracle import oracle as O
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc
+    d = dict(CPU_SAMPLE)[name]()
+    sh, _ = shard_desc(d, SHARD_LOOP[name], k, n)
+    x = W.make_inputs(sh, seed_offset=k)
+    t0 = time.perf_counter()
+    O.run(sh, x)
+    return time.perf_counter() - t0
+
+
+def cpu_oracle_all_cores():
+    import multiprocessing as mp
+    cores = os.cpu_count() or 1
+    total_b, wall = 0, 0.0
+    with mp.get_context("spawn").Pool(cores) as pool:
+        pool.map(_oracle_shard, [("cfg2", 0, 32)] * cores)   # warm the workers (imports, oracle build)
+        for name, mk in CPU_SAMPLE:
+            n = _shards(mk(), SHARD_LOOP[name], cores)
+            t0 = time.perf_counter()
+            pool.map(_oracle_shard, [(name, k, n) for k in range(n)])
+            wall += time.perf_counter() - t0
+            total_b += W.algorithmic_bytes(mk())
+    cpu = "unknown CPU"
+    try:
+        with open("/proc/cpuinfo") as f:
+            cpu = next(l.split(":", 1)[1].strip() for l in f if l.startswith("model name"))
+    except Exception:
+        pass
+    return {"value": total_b / wall / 1e9, "unit": "GB/s", "cores": cores, "kind": "oracle",
+            "sample": CPU_SAMPLE_TXT.replace("1 thread", "one process per core, the sample's parallel loop split "
+                                             "in contiguous blocks") + "; host: " + cpu}
+
+
+def _shards(d, loop, cores):
+    E = d["loops"][loop]
+    n = min(cores, E)
+    while E % n:
+        n -= 1
+    return n
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -403,11 +453,16 @@ def run_fop(args):
                                "grid": o["selected"][1], "block": o["selected"][2]}
                    for i, o in enumerate(ops)}
 
-    cpu = None
+    cpu = cpu_all = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cache = {}
         b, tt = cpu_oracle_step(cache)
         cpu = {"value": b / tt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": CPU_SAMPLE_TXT}
+        if not args.no_cpu_all:
+            try:
+                cpu_all = cpu_oracle_all_cores()
+            except Exception as e:  # noqa: BLE001 — baseline only, never fails the bench
+                cpu_all = {"unavailable": f"{type(e).__name__}: {e}"[:200]}
 
     if rank == 0:
         line = {
@@ -440,6 +495,7 @@ def run_fop(args):
                          "traffic": traffic, "alg_bytes_per_launch": ops[dom]["bytes"],
                          "peak_source": peak_src},
             "cpu_baseline": cpu,
+            "cpu_baseline_all_cores": cpu_all,
             "e2e": {"value": step_bytes * world / (e2e_ms / 1e3) / 1e9, "unit": "GB/s",
                     "h2d_bytes_per_step": sum(o["h2d"] for o in ops),
                     "d2h_bytes_per_step": sum(o["d2h"] for o in ops),
@@ -466,6 +522,7 @@ def main():
     ap.add_argument("--vec-bytes", type=int, default=0, help="16 or 32 (default: planner default 16)")
     ap.add_argument("--order", choices=["paper", "memory"], default=None)
     ap.add_argument("--no-cpu", action="store_true", help="skip the oracle cpu_baseline leg")
+    ap.add_argument("--no-cpu-all", action="store_true", help="skip the all-host-cores oracle baseline")
     ap.add_argument("--no-pdl", action="store_true",
                     help="launch the ops one by one (fop_run each) instead of one fop_run_many chain")
     ap.add_argument("--no-graph", action="store_true", help="eager steps instead of replaying a CUDA graph")

@@ -1359,10 +1359,16 @@ struct Gen {
       const XStmt& x = L.stmts[si];
       bool red = x.kind == FOP_REDUCE;
       o.l("// statement " + num(x.stmt) + (red ? " (REDUCE)" : " (ASSIGN)"));
+      // Sums with many sequential terms per lane (long outer reduction loops
+      // over few vectors) use compensated (Kahan) accumulation: the error of
+      // a plain running sum grows with the count (R16's bound assumes a
+      // short per-lane chain), Kahan's stays ~2u * sum|t| whatever the length.
+      const bool kahan = red && x.redop == FOP_RED_SUM && NRO * K * W > 128;
       if (red) {
         o.l(std::string("float acc") + num(x.stmt) + " = " +
             (x.redop == FOP_RED_MAX ? "__uint_as_float(0xff800000u)" : "0.f") + ";");
         if (x.redop == FOP_RED_SUM) o.l("u64 acc" + num(x.stmt) + "p = fop::pk1(0.f);");
+        if (kahan) o.l("float acc" + num(x.stmt) + "c = 0.f; u64 acc" + num(x.stmt) + "cp = fop::pk1(0.f);");
       }
       if (x.kind == FOP_ASSIGN && x.fwd && regmode) o.l("float F" + num(x.stmt) + "[" + num(NRO * K * W) + "];");
       if (rt_ro) {
@@ -1465,7 +1471,20 @@ struct Gen {
             sk.scalar = [&, A, mx](const std::string& v) {
               o.l(A + " = " + (mx ? "fop::op_max(" : "__fadd_rn(") + A + ", " + v + ");");
             };
-            if (!mx) {
+            if (kahan) {   // y = v - c; t = s + y; c = (t - s) - y; s = t
+              sk.scalar = [&, A](const std::string& v) {
+                o.l("{ const float y_ = __fsub_rn(" + v + ", " + A + "c); const float t_ = __fadd_rn(" + A + ", y_); " + A +
+                    "c = __fsub_rn(__fsub_rn(t_, " + A + "), y_); " + A + " = t_; }");
+              };
+              sk.pair = [&, A](const std::string& v, const std::string&) {
+                o.l("{ const u64 y_ = fop::sub2(" + v + ", " + A + "cp); const u64 t_ = fop::add2(" + A + "p, y_); " + A +
+                    "cp = fop::sub2(fop::sub2(t_, " + A + "p), y_); " + A + "p = t_; }");
+              };
+              sk.pair_fma = [&, A](const std::string& a, const std::string& b, const std::string&) {
+                o.l("{ const u64 y_ = fop::sub2(fop::mul2(" + a + ", " + b + "), " + A + "cp); const u64 t_ = fop::add2(" + A +
+                    "p, y_); " + A + "cp = fop::sub2(fop::sub2(t_, " + A + "p), y_); " + A + "p = t_; }");
+              };
+            } else if (!mx) {
               sk.pair = [&, A](const std::string& v, const std::string&) { o.l(A + "p = fop::add2(" + A + "p, " + v + ");"); };
               sk.pair_fma = [&, A](const std::string& a, const std::string& b, const std::string&) {
                 o.l(A + "p = fop::fma2(" + a + ", " + b + ", " + A + "p);");
@@ -1509,7 +1528,10 @@ struct Gen {
       }
       if (red) {
         std::string a = "acc" + num(x.stmt);
-        if (x.redop == FOP_RED_SUM)
+        if (kahan)   // each running sum minus its compensation, then combined
+          o.l(a + " = __fadd_rn(__fsub_rn(" + a + ", " + a + "c), __fadd_rn(__fsub_rn(fop::lo(" + a + "p), fop::lo(" + a +
+              "cp)), __fsub_rn(fop::hi(" + a + "p), fop::hi(" + a + "cp))));");
+        else if (x.redop == FOP_RED_SUM)
           o.l(a + " = __fadd_rn(" + a + ", __fadd_rn(fop::lo(" + a + "p), fop::hi(" + a + "p)));");
         o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::warp_max(" : "fop::warp_sum(") + a + ");");
         if (G > 1) {   // the row's G warp partials, combined in warp order
@@ -1587,13 +1609,27 @@ struct Gen {
           "u;");
     }
     const bool packed = !isMax && W % 2 == 0 && g_packed;
+    // rows one lane accumulates in sequence; a long chain is summed with
+    // compensation (Kahan), as in ROW_REDUCE
+    const int64_t chain = (ROWS + NCH * (int64_t)L.gr - 1) / (NCH * (int64_t)L.gr);
+    const bool kahan = !isMax && chain > 128;
     o.l("float acc[" + num(W) + "];");
     o.l("#pragma unroll");
     o.l("for (int e = 0; e < " + num(W) + "; ++e) acc[e] = " + init + ";");
+    if (kahan) {
+      o.l("float accc[" + num(W) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) accc[e] = 0.f;");
+    }
     if (packed) {
       o.l("u64 accp[" + num(W / 2) + "];");
       o.l("#pragma unroll");
       o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) accp[p] = fop::pk1(0.f);");
+      if (kahan) {
+        o.l("u64 acccp[" + num(W / 2) + "];");
+        o.l("#pragma unroll");
+        o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) acccp[p] = fop::pk1(0.f);");
+      }
     }
     // Software pipeline (default): the U row loads of batch i+1 are issued as
     // raw words before batch i is converted and accumulated, so HBM requests
@@ -1706,6 +1742,22 @@ struct Gen {
           o.l("accp[" + p + "] = fop::fma2(" + a + ", " + b + ", accp[" + p + "]);");
         };
       }
+      if (kahan) {   // y = v - c; t = s + y; c = (t - s) - y; s = t
+        sk.scalar = [&](const std::string& v) {
+          o.l("{ const float y_ = __fsub_rn(" + v + ", accc[e]); const float t_ = __fadd_rn(acc[e], y_); accc[e] = "
+              "__fsub_rn(__fsub_rn(t_, acc[e]), y_); acc[e] = t_; }");
+        };
+        if (packed) {
+          auto kp = [&](const std::string& v, const std::string& p) {
+            o.l("{ const u64 y_ = fop::sub2(" + v + ", acccp[" + p + "]); const u64 t_ = fop::add2(accp[" + p + "], y_); acccp[" +
+                p + "] = fop::sub2(fop::sub2(t_, accp[" + p + "]), y_); accp[" + p + "] = t_; }");
+          };
+          sk.pair = kp;
+          sk.pair_fma = [&, kp](const std::string& a, const std::string& b, const std::string& p) {
+            kp("fop::mul2(" + a + ", " + b + ")", p);
+          };
+        }
+      }
       emit_elems(o, x, var, c, W, sk);
       o.ind--;
       o.l("}");
@@ -1719,6 +1771,14 @@ struct Gen {
     }
     o.ind--;
     o.l("}");
+    if (kahan) {   // running sums minus their compensations
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) acc[e] = __fsub_rn(acc[e], accc[e]);");
+      if (packed) {
+        o.l("#pragma unroll");
+        o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) accp[p] = fop::sub2(accp[p], acccp[p]);");
+      }
+    }
     if (packed) {  // pairs of partial sums back to one accumulator per column
       o.l("#pragma unroll");
       o.l("for (int p = 0; p < " + num(W / 2) + "; ++p) { float a0_, a1_; fop::upk(accp[p], a0_, a1_); "

@@ -86,6 +86,29 @@ def _long_outer_reduction_case():
                        "reads": [("x", ["a", "b", "c"])], "expr": [("load", 0)]}]}
 
 
+def _long_lane_chain_case():
+    """Found by the fuzz campaign (seed 5, case 119): a row reduction whose
+    vector loop holds ONE vector (l3, extent 2) under 3200 outer reduction
+    iterations (l0 x l2, l2 used by no access): one lane summed 6400 terms in
+    sequence and exceeded the 1e-5 normwise bound (ratio 1.61).  Such lanes
+    now accumulate with compensated (Kahan) summation."""
+    return {"name": "long_lane_chain", "loops": {"l0": 32, "l1": 13, "l2": 100, "l3": 2},
+            "tensors": {"x0": {"shape": [32, 13, 2], "dtype": "bf16", "role": "in",
+                               "init": ("normal", 0.0, 1.0, 55826), "strides": [60, 4, 1]},
+                        "x1": {"shape": [13, 2], "dtype": "f16", "role": "in", "init": ("normal", 0.0, 1.0, 55827)},
+                        "out": {"shape": [13], "dtype": "f32", "role": "out"}},
+            "stmts": [{"kind": "reduce", "op": "sum", "loops": ["l0", "l1", "l2", "l3"], "write": ("out", ["l1"]),
+                       "reads": [("x0", ["l0", "l1", "l3"]), ("x1", ["l1", "l3"])],
+                       "expr": [("load", 0), ("load", 1), ("const", 2.0), ("abs", 0), ("add", 3, 1)]}]}
+
+
+def test_long_lane_chain_uses_compensated_sum():
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    src = FusedOp(_long_lane_chain_case(), autotune=0).source(0)
+    assert "cp = fop::sub2(fop::sub2(t_" in src
+    assert "cp = fop::sub2" not in FusedOp(W.cfg4a(2, 8, 768), autotune=0).source(0)
+
+
 @pytest.mark.gpu
 def test_fuzz_regressions():
     from harness import run_gpu, assert_ulp, assert_normwise, abs_terms_desc
@@ -98,3 +121,7 @@ def test_fuzz_regressions():
     got, op = run_gpu(d, x)
     assert op.info()["launches"][0]["class"] == "row_reduce"
     assert_normwise(got["s"], O.run(d, x)["s"], O.run(abs_terms_desc(d, 0), x)["s"], 1e-5, "s")
+    d = _long_lane_chain_case()
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x)
+    assert_normwise(got["out"], O.run(d, x)["out"], O.run(abs_terms_desc(d, 0), x)["out"], 1e-5, "out")

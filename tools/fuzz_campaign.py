@@ -22,10 +22,25 @@ from harness import run_gpu, assert_bitexact, assert_ulp, assert_normwise, abs_t
 from oracle import oracle as O  # noqa: E402
 
 
-def check(d):
+def check(d, repeat=False):
     x = W.make_inputs(d)
     got, op = run_gpu(d, x)
     ref = O.run(d, x, outputs=W.alloc_outputs(d))
+    compare(d, x, got, ref)
+    if repeat:   # the same plan again (tuned geometry), a misaligned run (narrow variant), aligned again
+        import torch
+        from harness import device_tensors, to_host
+        for off in (0, 1, 0):
+            dev = device_tensors(d, x, offset=off)
+            op.run(dev)
+            torch.cuda.synchronize()
+            got = {n: to_host(dev[n], d["tensors"][n]["dtype"]) for n, t in d["tensors"].items()
+                   if t["role"] in ("out", "inout")}
+            compare(d, x, got, ref)
+    return [li["class"] for li in op.info()["launches"]]
+
+
+def compare(d, x, got, ref):
     for si, st in enumerate(d["stmts"]):
         n = st["write"][0]
         t = d["tensors"][n]
@@ -42,20 +57,20 @@ def check(d):
             assert_ulp(got[n], ref[n], 1, n)
         else:
             assert_bitexact(got[n], ref[n], n)
-    return [li["class"] for li in op.info()["launches"]]
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--count", type=int, default=500)
+    ap.add_argument("--repeat", action="store_true", help="also re-run each plan (aligned, misaligned, aligned)")
     a = ap.parse_args()
     rng = np.random.default_rng(a.seed)
     fails, classes = [], {}
     for i in range(a.count):
         d = random_op(rng)
         try:
-            for c in check(d):
+            for c in check(d, a.repeat):
                 classes[c] = classes.get(c, 0) + 1
         except Exception as e:  # noqa: BLE001
             fails.append({"case": i, "error": f"{type(e).__name__}: {str(e)[:300]}", "desc": d,
