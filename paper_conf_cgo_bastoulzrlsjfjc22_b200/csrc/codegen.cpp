@@ -308,7 +308,8 @@ struct Gen {
     o.l("#include \"fop_device.cuh\"");
     o.l("typedef " + idx + " idx_t;");
     o.l("extern \"C\" __global__ void __launch_bounds__(" + num(L.block) + ", " + num(minblocks) + ") " +
-        L.name + "(const FopArgs args) {");
+        (L.row_q > 1 ? "__cluster_dims__(" + num(L.row_q) + ", 1, 1) " : std::string("")) + L.name +
+        "(const FopArgs args) {");
     o.ind++;
     for (int t = 0; t < d.ntensors; t++) {
       bool used = false;
@@ -1222,25 +1223,35 @@ struct Gen {
     // G warp partials of a reduction combined in a fixed order through shared
     // memory, the row loop uniform across the block (it synchronises)
     const int G = std::max(1, L.row_g);
-    const int64_t LN = 32 * (int64_t)G;
-    const int64_t GPB = L.block / LN;
+    // Q CTAs per row (a thread-block cluster; few long rows): the row's lanes
+    // span the cluster, block partials are combined through distributed
+    // shared memory in rank order, identically in every CTA
+    const int Q = std::max(1, L.row_q);
+    const int64_t LNB = 32 * (int64_t)G;   // lanes of one row inside a block
+    const int64_t LN = LNB * Q;            // lanes of one row
+    const bool MULTI = G > 1 || Q > 1;     // the row loop synchronises (block-uniform trip count)
     const int K = (int)((NVD + LN - 1) / LN);
-    const bool jguard = NVD % LN != 0 || G > 1;
     int64_t NRO = 1;
     for (int k = 1; k < L.nsplit; k++) NRO *= L.kl[k].extent;
+    // split mode (geometry: few vectors, long outer reduction loops): lane =
+    // (sub, v), v = lane % NVDP over the vectors, the SPL subgroups take the
+    // outer reduction iterations sub, sub + SPL, ... (runtime loop)
+    const int64_t SPL = L.row_split;
+    const int64_t NVDP = SPL ? LN / SPL : 0;
+    const bool jguard = NVD % LN != 0 || MULTI || SPL;
     int64_t rows = L.work;
     const int64_t WSTRIDE = L.grid * L.block / LN;
     // forwarded rows live in registers when they fit (<= 64 values per lane);
     // longer rows are re-read by the lane that stored them (same thread, same
     // address: program order makes the store visible; L2 serves the re-read)
-    const bool regmode = NRO * K * W <= 64;
+    const bool regmode = NRO * K * W <= 64 && !SPL;
     for (auto& x : L.stmts)
       if (x.kind == FOP_ASSIGN && x.fwd && !regmode && !x.store)
         fail(FOP_E_UNSUPPORTED, "ROW_REDUCE: a long forwarded row must be stored to be re-read");
     // outer reduction iterations: unrolled at compile time while the row can
     // stay in registers, a runtime loop otherwise (no per-vector register
     // arrays are indexed then: no hoisting, prefetch or register forwarding)
-    const bool rt_ro = NRO > 64;
+    const bool rt_ro = NRO > 64 || SPL;
     const int64_t NRO_E = rt_ro ? 1 : NRO;
     const int NP = (int)(NRO_E * K);   // vectors per lane per row held in registers
     // per-load treatment: hoisted (independent of the row: e.g. a bias, loaded
@@ -1277,12 +1288,17 @@ struct Gen {
     };
     header(G == 1 ? "ROW_REDUCE (one warp per row, lanes across d_v vectors, butterfly)"
                   : "ROW_REDUCE (" + std::to_string(G) + " warps per row, butterfly + fixed-order shared-memory combine)", 1);
-    o.l("const idx_t lane = threadIdx.x % " + num(LN) + "u;");
+    if (Q > 1) o.l("const idx_t lane = threadIdx.x % " + num(LNB) + "u + fop::cluster_ctarank() * " + num(LNB) + "u;");
+    else o.l("const idx_t lane = threadIdx.x % " + num(LN) + "u;");
+    if (SPL) o.l("const idx_t vl_ = lane % " + num(NVDP) + "u, sub_ = lane / " + num(NVDP) + "u;");
     if (G > 1) {
-      o.l("const idx_t grp = threadIdx.x / " + num(LN) + "u;");
+      o.l("const idx_t grp = threadIdx.x / " + num(LNB) + "u;");
       for (auto& x : L.stmts)
         if (x.kind == FOP_REDUCE) o.l("__shared__ float RS" + num(x.stmt) + "[" + num(L.block / 32) + "];");
     }
+    if (Q > 1)
+      for (auto& x : L.stmts)
+        if (x.kind == FOP_REDUCE) o.l("__shared__ float RQ" + num(x.stmt) + ";");
     // hoisted row-invariant loads
     for (size_t k = 0; k < L.loads.size(); k++) {
       if (mode[k] != 'H') continue;
@@ -1334,9 +1350,9 @@ struct Gen {
     o.l("idx_t row = ((idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x) / " + num(LN) + "u;");
     emit_prefetch("row", "_p");
     o.l("#pragma unroll 1");
-    if (G > 1) {   // block-uniform trip count: every group reaches the barriers
-      o.l("for (idx_t rb_ = (idx_t)blockIdx.x * " + num(GPB) + "u; rb_ < (idx_t)" + num(rows) + "ull; rb_ += (idx_t)" +
-          num(WSTRIDE) + "ull, row += (idx_t)" + num(WSTRIDE) + "ull) {");
+    if (MULTI) {   // block-uniform trip count: every group (and every CTA of the cluster) reaches the barriers
+      o.l("for (idx_t rb_ = ((idx_t)blockIdx.x * " + num(L.block) + "u) / " + num(LN) + "u; rb_ < (idx_t)" + num(rows) +
+          "ull; rb_ += (idx_t)" + num(WSTRIDE) + "ull, row += (idx_t)" + num(WSTRIDE) + "ull) {");
       o.ind++;
       o.l("const bool rv = row < (idx_t)" + num(rows) + "ull;");
     } else {
@@ -1363,7 +1379,7 @@ struct Gen {
       // over few vectors) use compensated (Kahan) accumulation: the error of
       // a plain running sum grows with the count (R16's bound assumes a
       // short per-lane chain), Kahan's stays ~2u * sum|t| whatever the length.
-      const bool kahan = red && x.redop == FOP_RED_SUM && NRO * K * W > 128;
+      const bool kahan = red && x.redop == FOP_RED_SUM && (SPL ? (NRO + SPL - 1) / SPL : NRO) * K * W > 128;
       if (red) {
         o.l(std::string("float acc") + num(x.stmt) + " = " +
             (x.redop == FOP_RED_MAX ? "__uint_as_float(0xff800000u)" : "0.f") + ";");
@@ -1371,19 +1387,11 @@ struct Gen {
         if (kahan) o.l("float acc" + num(x.stmt) + "c = 0.f; u64 acc" + num(x.stmt) + "cp = fop::pk1(0.f);");
       }
       if (x.kind == FOP_ASSIGN && x.fwd && regmode) o.l("float F" + num(x.stmt) + "[" + num(NRO * K * W) + "];");
-      if (rt_ro) {
-        o.l("#pragma unroll 1");
-        o.l("for (idx_t ro_ = 0; ro_ < " + num(NRO) + "u; ++ro_) {");
-        o.ind++;
-        o.l("idx_t rq_ = ro_;");
-      }
       for (int64_t ro = 0; ro < NRO_E; ro++) {
-        // decomposition of ro over the outer reduction kloops (compile time,
-        // or at run time for the runtime loop)
+        // decomposition of ro over the outer reduction kloops (compile time;
+        // at run time, inside the kk block, for the runtime loop)
         std::vector<std::pair<int, std::string>> its = rits;
-        if (rt_ro) {
-          decompose("rq_", 1, L.nsplit, "_r" + num(si), its);
-        } else {
+        if (!rt_ro) {
           int64_t rem = ro;
           for (int k = 1; k < L.nsplit; k++) {
             its.push_back({k, num(rem % L.kl[k].extent) + "u"});
@@ -1394,9 +1402,27 @@ struct Gen {
           std::string t = "_" + num(si) + "_" + num(ro) + "_" + num(kk);
           o.l("{");
           o.ind++;
-          o.l("[[maybe_unused]] const idx_t iv = (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
-          if (jguard) o.l(std::string("if (") + (G > 1 ? "rv && " : "") + "lane + " + num(LN * kk) + "u < " + num(NVD) + "u) {");
+          if (SPL) {
+            o.l("[[maybe_unused]] const idx_t iv = vl_ * " + num(W) + "u;");
+            o.l(std::string("if (") + (MULTI ? "rv && " : "") + "vl_ < " + num(NVD) + "u) {");
+          } else {
+            o.l("[[maybe_unused]] const idx_t iv = (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
+            if (jguard)
+              o.l(std::string("if (") + (MULTI ? "rv && " : "") + "lane + " + num(LN * kk) + "u < " + num(NVD) + "u) {");
+          }
           auto its2 = its;
+          if (rt_ro) {
+            // the runtime loop over the outer reduction iterations runs
+            // INSIDE the lane's (loop-invariant) guard, unrolled, so the loads
+            // of several iterations are in flight per lane; per lane the
+            // terms are accumulated vector by vector (a fixed order)
+            o.l("#pragma unroll " + num(std::max(1, geometry_knob(L, "FOP_ROW_ROU", 8))));
+            if (SPL) o.l("for (idx_t ro_ = sub_; ro_ < " + num(NRO) + "u; ro_ += " + num(SPL) + "u) {");
+            else o.l("for (idx_t ro_ = 0; ro_ < " + num(NRO) + "u; ++ro_) {");
+            o.ind++;
+            o.l("idx_t rq_ = ro_;");
+            decompose("rq_", 1, L.nsplit, "_r" + num(si), its2);
+          }
           its2.push_back({0, "iv"});
           // loads used by this statement
           std::vector<bool> used(L.loads.size(), false);
@@ -1517,14 +1543,14 @@ struct Gen {
               o.l("for (int e = 0; e < " + num(W) + "; ++e) fop::sstore<" + dt + ">(" +
                   ptr(x.write.tensor, off + " + e * " + num(cw)) + ", R[e]);");
           }
+          if (rt_ro) {
+            o.ind--;
+            o.l("}");
+          }
           if (jguard) o.l("}");
           o.ind--;
           o.l("}");
         }
-      }
-      if (rt_ro) {
-        o.ind--;
-        o.l("}");
       }
       if (red) {
         std::string a = "acc" + num(x.stmt);
@@ -1544,10 +1570,20 @@ struct Gen {
               (x.redop == FOP_RED_MAX ? "fop::op_max(" : "__fadd_rn(") + a + ", " + rs + "[grp * " + num(G) + "u + g_]);");
           o.l("__syncthreads();");
         }
+        if (Q > 1) {   // the cluster's Q block partials, read from every CTA's shared memory in rank order
+          std::string rq = "RQ" + num(x.stmt);
+          o.l("if (threadIdx.x == 0u) " + rq + " = " + a + ";");
+          o.l("fop::cluster_sync();");
+          o.l(a + " = fop::ld_dsmem(&" + rq + ", 0u);");
+          o.l("#pragma unroll");
+          o.l("for (unsigned q_ = 1; q_ < " + num(Q) + "u; ++q_) " + a + " = " +
+              (x.redop == FOP_RED_MAX ? "fop::op_max(" : "__fadd_rn(") + a + ", fop::ld_dsmem(&" + rq + ", q_));");
+          o.l("fop::cluster_sync();");
+        }
         std::string res = fin_expr(o, x, a, "");
         if (x.fwd) o.l("const float S" + num(x.stmt) + " = fop::round_to<" + dtn(x.out_dtype) + ">(" + res + ");");
         if (x.store)
-          o.l(std::string(G > 1 ? "if (rv && lane == 0) " : "if (lane == 0) ") + "fop::sstore<" + std::string(dtn(x.out_dtype)) + ">(" +
+          o.l(std::string(MULTI ? "if (rv && lane == 0) " : "if (lane == 0) ") + "fop::sstore<" + std::string(dtn(x.out_dtype)) + ">(" +
               ptr(x.write.tensor, affine(x.write, rits)) + ", " + res + ");");
       }
     }

@@ -539,6 +539,25 @@ __device__ __forceinline__ void sts128(u32 addr, u32 a, u32 b, u32 c, u32 d) {
   asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
 }
 
+// ---------------------------------------------------------------- thread-block clusters
+// ROW_REDUCE with Q CTAs per row: block partials combined through
+// distributed shared memory (every CTA reads rank 0..Q-1 in order).
+__device__ __forceinline__ unsigned cluster_ctarank() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ float ld_dsmem(const float* p, unsigned rank) {
+  u32 a = (u32)__cvta_generic_to_shared(p), r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(rank));
+  float v;
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(r) : "memory");
+  return v;
+}
+
 // ---------------------------------------------------------------- programmatic dependent launch
 // Explicit PDL control, emitted only with FOP_PDL_EMIT (ablation): bit 1 =
 // trigger dependents (at block end, or at start with FOP_PDL_POS=0), bit 2 =

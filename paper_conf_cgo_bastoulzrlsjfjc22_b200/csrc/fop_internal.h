@@ -140,6 +140,10 @@ struct Launch {
   int col_il = 1;                 // COL: chunks interleave over rows (grid sweeps rows together)
   int row_hoist = 1;              // ROW: keep row-invariant loads in registers across rows
   int row_g = 1;                  // ROW: warps per row (> 1 for few long rows)
+  int row_q = 1;                  // ROW: CTAs per row (a thread-block cluster) for few long rows
+  int row_split = 0;              // ROW: > 0 = lanes also split the outer reduction iterations (S lane
+                                  // subgroups of pow2(#vectors) lanes each), for rows of few vectors
+                                  // under long outer reduction loops (e.g. BN statistics on NCHW)
   // TRANSPOSE through TMA (16-bit data): 64x64 tiles, tensor maps encoded per run
   int tma = 0;
   int tma_rank = 0, tma_stages = 4;

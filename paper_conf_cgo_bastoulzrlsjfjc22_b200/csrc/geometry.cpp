@@ -98,9 +98,15 @@ void collapse_into(const Plan& p, const std::vector<const Affine*>& acc, const s
   }
 }
 
+int64_t pow2_ceil(int64_t x);
 int pow2_floor(int64_t x) {
   int r = 1;
   while ((int64_t)r * 2 <= x) r *= 2;
+  return r;
+}
+int64_t pow2_ceil(int64_t x) {
+  int64_t r = 1;
+  while (r < x) r *= 2;
   return r;
 }
 
@@ -428,17 +434,41 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     // fewer than 4 vectors of the row (measured: G=16 beats 32 at 2-4
     // vectors per lane, profiles/sweep_r01_rowg.log)
     int64_t nvd = EV / W;
+    int64_t nro = 1;
+    for (int k = 1; k < L.nsplit; k++) nro *= L.kl[k].extent;
+    // few vectors along d_v under long outer reduction loops (per-channel
+    // statistics over N,H,W of an NCHW tensor: 7 vectors x 14336 outer
+    // iterations): the lanes also split the outer iterations, else most
+    // lanes idle and one chain walks the whole row
+    const bool split = nvd < 32 && nro * W > 64 && knob("FOP_ROW_SPLIT", 1);
+    const int64_t row_vecs = split ? nvd * nro : nvd;
     int G = 1;
-    while (G < 32 && rows * G < (int64_t)sms * 16 && 256 * (int64_t)G <= nvd) G *= 2;
+    while (G < 32 && rows * G < (int64_t)sms * 16 && 256 * (int64_t)G <= row_vecs) G *= 2;
+    // fewer rows than SMs: each row also spreads over a cluster of Q CTAs
+    // (several SMs; block partials combined through distributed shared
+    // memory), G capped at 8 warps per CTA so the parallelism goes across SMs
+    const int64_t lanes_cap = split ? nvd * nro : nvd;   // lanes one row can keep busy
+    int Q = 1;
+    if (rows < (int64_t)sms) {
+      G = std::min(G, 8);
+      while (Q < 8 && rows * Q * 2 <= (int64_t)sms * 2 && 32 * (int64_t)G * Q * 2 <= lanes_cap) Q *= 2;
+    }
     G = std::max(1, pow2_floor(knob("FOP_ROW_G", G)));
+    Q = std::max(1, std::min(8, pow2_floor(knob("FOP_ROW_Q", Q))));
     L.row_g = G;
+    L.row_q = Q;
+    L.row_split = split ? (int)(32 * (int64_t)G * Q / std::min<int64_t>(32 * (int64_t)G * Q, pow2_ceil(nvd))) : 0;
     if (G > 1) L.block = std::max(L.block, 32 * G);
+    if (Q > 1) L.block = 32 * G;   // one row per CTA
     L.minblocks = knob("FOP_ROW_MINB", L.block >= 1024 ? 1 : (L.block >= 512 ? 2 : 3));
     L.row_prefetch = knob("FOP_ROW_PREFETCH", 1);
     L.row_hoist = knob("FOP_ROW_HOIST", 1);
     int64_t gpb = L.block / (32 * G);
     int64_t need = (rows + gpb - 1) / gpb;
     L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
+    if (Q > 1)   // whole clusters, one row each per pass
+      L.grid = std::max<int64_t>(1, std::min<int64_t>({rows, (int64_t)sms * L.minblocks / Q,
+                                                       (int64_t)knob("FOP_ROW_CLUSTERS", 1 << 30)})) * Q;
     L.unroll = 1;
   } else {  // COL_REDUCE
     int64_t nvd = EV / W;

@@ -102,10 +102,16 @@ def _long_lane_chain_case():
                        "expr": [("load", 0), ("load", 1), ("const", 2.0), ("abs", 0), ("add", 3, 1)]}]}
 
 
-def test_long_lane_chain_uses_compensated_sum():
+def test_long_lane_chain_splits_lanes_or_compensates(monkeypatch):
     from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    # default: the lanes split the 3200 outer iterations (short chains per lane)
     src = FusedOp(_long_lane_chain_case(), autotune=0).source(0)
-    assert "cp = fop::sub2(fop::sub2(t_" in src
+    assert "ro_ = sub_;" in src
+    # lanes over the single vector only: one long chain, summed with compensation
+    monkeypatch.setenv("FOP_ROW_SPLIT", "0")
+    monkeypatch.setenv("FOP_ROW_Q", "1")
+    src = FusedOp(_long_lane_chain_case(), autotune=0).source(0)
+    assert "cp = fop::sub2(fop::sub2(t_" in src and "sub_" not in src.replace("__fsub_rn", "")
     assert "cp = fop::sub2" not in FusedOp(W.cfg4a(2, 8, 768), autotune=0).source(0)
 
 
@@ -123,5 +129,16 @@ def test_fuzz_regressions():
     assert_normwise(got["s"], O.run(d, x)["s"], O.run(abs_terms_desc(d, 0), x)["s"], 1e-5, "s")
     d = _long_lane_chain_case()
     x = W.make_inputs(d)
-    got, _ = run_gpu(d, x)
-    assert_normwise(got["out"], O.run(d, x)["out"], O.run(abs_terms_desc(d, 0), x)["out"], 1e-5, "out")
+    for knobs in ({}, {"FOP_ROW_SPLIT": "0", "FOP_ROW_Q": "1"}):   # split lanes / one compensated chain
+        import os
+        old = {k: os.environ.get(k) for k in knobs}
+        os.environ.update(knobs)
+        try:
+            got, _ = run_gpu(d, x)
+        finally:
+            for k, v in old.items():
+                if v is None:
+                    os.environ.pop(k, None)
+                else:
+                    os.environ[k] = v
+        assert_normwise(got["out"], O.run(d, x)["out"], O.run(abs_terms_desc(d, 0), x)["out"], 1e-5, "out")

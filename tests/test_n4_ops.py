@@ -21,6 +21,9 @@ SMALL = {
     # few long rows: several warps per row (ROW_REDUCE row_g > 1)
     "vocab_softmax": dict(R=5, V=4000),
     "wide_layernorm": dict(R=3, H=12288),
+    # few vectors per row under long outer reduction loops: lanes split the outer iterations
+    "bn_stats_nchw": dict(N=6, C=8, H=14, W=14),
+    "bn_stats_small_hw": dict(N=64, C=8, H=4, W=4),     # 2 vectors per row: lanes split the samples
 }
 
 
@@ -50,6 +53,34 @@ def _assert_layernorm(d, x, got, ref):
 
 
 # ---------------------------------------------------------------- oracle pins (CPU)
+def test_oracle_bn_stats_vs_torch():
+    d = W.N4["bn_stats_nchw"](**SMALL["bn_stats_nchw"])
+    x = W.make_inputs(d)
+    r = O.run(d, x)
+    xt = torch.from_numpy(x["x"].astype(np.float64).reshape(6, 8, 14, 14))
+    var, mean = torch.var_mean(xt, dim=(0, 2, 3), unbiased=False)
+    assert np.allclose(r["mean"], mean.numpy(), rtol=1e-6, atol=1e-7)
+    # var from the f32-rounded mean (R17: later statements read stored values)
+    m32 = torch.from_numpy(r["mean"].astype(np.float64)).view(1, 8, 1, 1)
+    v2 = ((xt - m32) ** 2).mean(dim=(0, 2, 3))
+    assert np.allclose(r["var"], v2.numpy(), rtol=1e-6, atol=0)
+    assert np.allclose(r["var"], var.numpy(), rtol=1e-5, atol=0)
+
+
+def test_bn_stats_row_geometry():
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    # 64 channel rows of 1568 vectors x 128 samples: clusters of 4 CTAs per row
+    op = FusedOp(W.N4["bn_stats_nchw"](), autotune=0)
+    (li,) = op.info()["launches"]
+    assert li["class"] == "row_reduce" and li["vec_loop"] == "w" and li["grid"] == 256
+    src = op.source(0)
+    assert "__cluster_dims__(4, 1, 1)" in src and "fop::ld_dsmem" in src
+    # 4x4 planes: 2 vectors per row under 64 samples -> lanes split the samples
+    src = FusedOp(W.N4["bn_stats_nchw"](N=64, C=8, H=4, W=4), autotune=0).source(0)
+    assert "ro_ = sub_;" in src and "vl_ < 2u" in src
+
+
+
 def test_oracle_layernorm_vs_torch():
     d = W.N4["bert_layernorm"](**SMALL["bert_layernorm"])
     x = W.make_inputs(d)
@@ -138,5 +169,9 @@ def test_n4_gpu_vs_oracle(name, full):
             _assert_layernorm(d, x, v, ref[n])
         elif name in ("bert_softmax", "vocab_softmax"):
             assert_ulp(v, ref[n], 1, n)
+        elif name.startswith("bn_stats"):
+            from harness import abs_terms_desc, assert_normwise
+            si = 0 if n == "mean" else 1
+            assert_normwise(v, ref[n], O.run(abs_terms_desc(d, si), x)[n], 1e-5, n)
         else:
             assert_bitexact(v, ref[n], n)
