@@ -266,7 +266,10 @@ def run_fop(args):
     from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc, allreduce_partials, PeerExchange
     peer = world > 1 and args.exchange == "peer"
     ops = []
-    for name, mk, cls in OPS:
+    order = args.op_order.split(",")
+    if sorted(order) != sorted(n for n, _, _ in OPS):
+        raise SystemExit("--op-order must list cfg2,cfg3,cfg4a,cfg4b once each")
+    for name, mk, cls in sorted(OPS, key=lambda t: order.index(t[0])):
         gmk, loop = GLOBAL[name]
         d, shard_info = shard_desc(gmk(world), loop, rank, world, fused=peer)   # == mk() per rank
         popts = {"peer_world": world, "peer_loop": loop} if peer and shard_info["partials"] else {}
@@ -378,8 +381,9 @@ def run_fop(args):
     for k in range(args.steps):
         step(ev[k])
     torch.cuda.synchronize()
-    per_op = [statistics.mean(ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(args.steps))
-              for i in range(len(ops))]
+    per_op_samples = [[ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(args.steps)] for i in range(len(ops))]
+    per_op = [statistics.mean(v) for v in per_op_samples]
+    per_op_std = [statistics.pstdev(v) for v in per_op_samples]
     t = torch.tensor([ms] + per_op, dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -446,6 +450,7 @@ def run_fop(args):
     for o in ops:
         o["selected"] = o["op"].selected(0)   # kernel the auto-tuner kept (name, grid, block)
     per_op_json = {o["name"]: {"class": o["cls"], "kernel": o["selected"][0], "ms": per_op[i],
+                               "ms_std_rank0": per_op_std[i],
                                "alg_bytes": o["bytes"], "GB_s": o["bytes"] / (per_op[i] / 1e3) / 1e9,
                                "frac_of_measured_peak": o["bytes"] / (per_op[i] / 1e3) / 1e9 / peak,
                                "frac_of_8TBs": o["bytes"] / (per_op[i] / 1e3) / 1e9 / 8000.0,
@@ -473,6 +478,7 @@ def run_fop(args):
             "config": {
                 "workload": WORKLOAD,
                 "global_batch_scale": world,
+                "op_order": [o["name"] for o in ops],
                 "parallelism": ("dp%d (batch-sharded; " % world) + (
                     "no exchange)" if world == 1 else
                     "cfg4b partials combined inside the column-reduction kernel over NVLink peer memory)"
@@ -525,6 +531,8 @@ def main():
     ap.add_argument("--no-cpu-all", action="store_true", help="skip the all-host-cores oracle baseline")
     ap.add_argument("--no-pdl", action="store_true",
                     help="launch the ops one by one (fop_run each) instead of one fop_run_many chain")
+    ap.add_argument("--op-order", default="cfg2,cfg3,cfg4a,cfg4b",
+                    help="order of the (independent) ops in a step")
     ap.add_argument("--no-graph", action="store_true", help="eager steps instead of replaying a CUDA graph")
     ap.add_argument("--exchange", choices=["peer", "nccl"], default="peer",
                     help="N > 1: combine cfg4b's partial sums inside the kernel over NVLink (peer) or NCCL after it")
