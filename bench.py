@@ -44,6 +44,7 @@ OPS = [("cfg2", W.cfg2, "ew"), ("cfg3", W.cfg3, "transpose"), ("cfg4a", W.cfg4a,
 GLOBAL = {"cfg2": (lambda w: W.cfg2(N=128 * w), "n"), "cfg3": (lambda w: W.cfg3(N=256 * w), "n"),
           "cfg4a": (lambda w: W.cfg4a(B=64 * w), "b"), "cfg4b": (lambda w: W.cfg4b(R=65536 * w), "r")}
 FALLBACK_HBM = 6650.0
+L2_BYTES = 126 << 20          # B200 L2 (public figure), for the steady-state copies
 METRIC = "achieved HBM GB/s (fused-op suite; per-op GB/s and % of peak in config.per_op)"
 WORKLOAD = ("fused-op suite: cfg2 BN+ReLU+cast [128,64,112,112] f32->f16, cfg3 NCHW->NHWC*s "
             "[256,256,56,56] f16, cfg4a bias+GELU+row mean/var [64,512,768] f16, cfg4b colsum "
@@ -384,10 +385,38 @@ def run_fop(args):
     per_op_samples = [[ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(args.steps)] for i in range(len(ops))]
     per_op = [statistics.mean(v) for v in per_op_samples]
     per_op_std = [statistics.pstdev(v) for v in per_op_samples]
-    t = torch.tensor([ms] + per_op, dtype=torch.float64, device=dev)
+    # ---- each kernel on its own, in steady state (the tools/sweep.py protocol):
+    # back-to-back launches of ONE op rotating over input/output copies that
+    # together exceed 3x L2, so each launch pays for its own dirty-line
+    # write-back (the previous launch's, same size) and not for another op's
+    steady = [float("nan")] * len(ops)
+    if not args.no_steady:
+        for i, o in enumerate(ops):
+            if o["px"] is not None:
+                continue
+            copies = max(1, min(6, -(-3 * L2_BYTES // o["bytes"])))
+            sets = [o["dev"]] + [{n: t.clone() for n, t in o["dev"].items()} for _ in range(copies - 1)]
+            for k in range(3):
+                o["op"].run(sets[k % copies], stream=stream)
+            reps = 40
+            s3, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            best = float("inf")
+            for _ in range(3):
+                torch.cuda.synchronize()
+                s3.record(stream)
+                for k in range(reps):
+                    o["op"].run(sets[k % copies], stream=stream)
+                e3.record(stream)
+                torch.cuda.synchronize()
+                best = min(best, s3.elapsed_time(e3) / reps)
+            steady[i] = best
+            del sets
+    t = torch.tensor([ms] + per_op + steady, dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms, per_op = float(t[0]), [float(v) for v in t[1:]]
+    ms = float(t[0])
+    per_op = [float(v) for v in t[1:1 + len(ops)]]
+    steady = [float(v) for v in t[1 + len(ops):]]
 
     # ---- end to end through the C ABI with host buffers: fop_run_host_many
     # runs the suite's independent ops with the host<->device copies pipelined
@@ -455,7 +484,10 @@ def run_fop(args):
                                "frac_of_measured_peak": o["bytes"] / (per_op[i] / 1e3) / 1e9 / peak,
                                "frac_of_8TBs": o["bytes"] / (per_op[i] / 1e3) / 1e9 / 8000.0,
                                "vec_loop": o["kernel"]["vec_loop"], "width": o["kernel"]["width"],
-                               "grid": o["selected"][1], "block": o["selected"][2]}
+                               "grid": o["selected"][1], "block": o["selected"][2],
+                               "steady": (None if steady[i] != steady[i] else
+                                          {"ms": steady[i], "GB_s": o["bytes"] / (steady[i] / 1e3) / 1e9,
+                                           "frac_of_measured_peak": o["bytes"] / (steady[i] / 1e3) / 1e9 / peak})}
                    for i, o in enumerate(ops)}
 
     cpu = cpu_all = None
@@ -492,7 +524,10 @@ def run_fop(args):
                                                 " + NCCL all-reduce of cfg4b's partials" if world > 1 else "")),
                 "per_op_note": "per-op times come from a second pass of the same K steps with fop_run per op "
                                "and CUDA events around each (no overlap); an op also pays the write-back of "
-                               "dirty L2 lines the previous op left (e.g. cfg4b after cfg4a's 50 MB y)",
+                               "dirty L2 lines the previous op left (e.g. cfg4b after cfg4a's 50 MB y); "
+                               "per_op.*.steady: the op alone, best of 3 batches of 40 back-to-back launches "
+                               "rotating over input/output copies > 3x L2 (each launch pays only its own "
+                               "write-back)",
                 "per_op": per_op_json,
                 "peak_gbs": peak, "peak_source": peak_src,
             },
@@ -534,6 +569,7 @@ def main():
     ap.add_argument("--op-order", default="cfg2,cfg3,cfg4a,cfg4b",
                     help="order of the (independent) ops in a step")
     ap.add_argument("--no-graph", action="store_true", help="eager steps instead of replaying a CUDA graph")
+    ap.add_argument("--no-steady", action="store_true", help="skip the per-op steady-state pass")
     ap.add_argument("--exchange", choices=["peer", "nccl"], default="peer",
                     help="N > 1: combine cfg4b's partial sums inside the kernel over NVLink (peer) or NCCL after it")
     args = ap.parse_args()

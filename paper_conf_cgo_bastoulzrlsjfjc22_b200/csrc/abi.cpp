@@ -259,10 +259,10 @@ fop_status fop_run_many(const fop_plan_t* const* plans, void* const* const* dev_
       if (plans[k]->p.peer_bytes) fop::fail(FOP_E_INVALID, "plan " + std::to_string(k) + " has a peer exchange: use fop_run_peer");
     }
     const char* pe = std::getenv("FOP_RUN_MANY_PDL");   // 0: plain launches (ablation)
-    bool first = true;
-    if (pe && *pe == '0') first = true;
+    const bool no_pdl = pe && *pe == '0';
+    bool first = true;   // the chain's first kernel waits for prior stream work as usual
     for (int k = 0; k < n; k++) {
-      if (pe && *pe == '0') first = true;
+      if (no_pdl) first = true;
       fop::Plan& p = const_cast<fop_plan_t*>(plans[k])->p;
       fop::run_plan(p, dev_ptrs[k], nptrs[k], workspaces ? workspaces[k] : nullptr, stream, nullptr, nullptr, !first);
       if (!p.launches.empty()) first = false;

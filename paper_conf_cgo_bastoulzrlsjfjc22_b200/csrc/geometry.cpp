@@ -349,7 +349,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     int64_t ntv = EV / W, ntr = L.kl[1].extent / L.read_width;
     int es_out = esize(L.stmts[0].out_dtype);
     int gv = (int)std::min<int64_t>(32, std::max<int64_t>(1, 128 / (W * es_out)));
-    gv = std::min(gv, pow2_floor(ntv));
+    gv = std::min(pow2_floor(std::max(1, std::min(32, knob("FOP_TR_GV", gv)))), pow2_floor(ntv));
     L.gv = gv;
     L.gr = 32 / gv;
     int64_t tvh = (ntv + gv - 1) / gv, trh = (ntr + L.gr - 1) / L.gr;
