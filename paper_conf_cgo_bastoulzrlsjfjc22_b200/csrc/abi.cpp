@@ -117,7 +117,7 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
       if (p.opts.autotune && p.opts.jit && p.tunable) {
         for (size_t i = 0; i < p.launches.size(); i++) {
           if (p.launches[i].peer) continue;   // every rank must run the same geometry (fop_run_peer)
-          auto vs = fop::tuning_variants(p.launches[i]);
+          auto vs = fop::tuning_variants(p.launches[i], p.opts.sm_count > 0 ? p.opts.sm_count : 148);
           std::vector<std::string> seen = {p.launches[i].src};
           for (size_t k = 1; k < vs.size(); k++) {
             fop::Launch V = p.launches[i];

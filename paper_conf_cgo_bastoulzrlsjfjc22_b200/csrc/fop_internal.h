@@ -211,6 +211,8 @@ struct Plan {
     void* ctx;
     std::vector<void*> mods, fns, nmods, nfns;
     std::vector<std::vector<void*>> vfns;   // per launch: functions of variants[i]
+    void* flush_fn = nullptr;               // auto-tuner's L2 flush / dirty kernels (runtime.cpp)
+    void* dirty_fn = nullptr;
     std::vector<int> choice;                // per launch: -1 untuned, 0 = default, k = variants[i][k-1]
   };
   std::vector<Loaded> loaded;
@@ -223,7 +225,7 @@ bool empty_domain(const fop_desc& d, const fop_stmt& st);   // some loop of the 
 void plan_launches(Plan& p);
 void finalize_launch_geometry(const Plan& p, Launch& L);
 int geometry_knob(const Launch& L, const char* name, int dflt);
-std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Launch& L);
+std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Launch& L, int sms);
 // codegen.cpp
 std::string generate(const Plan& p, Launch& L, int launch_index);
 extern const char* kDeviceHeader;   // device/fop_device.cuh, embedded at build time

@@ -143,7 +143,7 @@ int geometry_knob(const Launch& L, const char* name, int dflt) {
 // come from auto-tuners too).  Entry 0 is the default rule.  Chosen
 // from the measured sweeps (profiles/sweep_r01_*.log): streaming kernels
 // prefer few threads with many vectors in flight, ALU-heavy ones more threads.
-std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Launch& L) {
+std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Launch& L, int /*sms*/) {
   typedef std::vector<std::pair<std::string, int>> K;
   std::vector<K> v = {K{}};
   switch (L.kclass) {

@@ -230,6 +230,19 @@ def test_cfg4a_bias_gelu_rowstats(dims):
     _check_rowstats(d, x, got)
 
 
+@pytest.mark.parametrize("knobs", [(160, 5), (800, 1), (96, 8)])
+def test_cfg4a_row_block_geometries(monkeypatch, knobs):
+    """ROW_REDUCE with warp counts per block that are not powers of two (the
+    auto-tuner's balanced-rounds candidate: 5 x 160 threads per SM)."""
+    monkeypatch.setenv("FOP_BLOCK", str(knobs[0]))
+    monkeypatch.setenv("FOP_ROW_MINB", str(knobs[1]))
+    d = W.cfg4a(3, 129, 768)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x, autotune=0)
+    assert op.info()["launches"][0]["block"] == knobs[0]
+    _check_rowstats(d, x, got)
+
+
 def test_row_closed_forms_on_gpu():
     d = W.cfg4a(1, 4, 768)
     d["stmts"][0]["expr"] = [("load", 0)]

@@ -1,0 +1,20 @@
+# auto-tuner from a cold L2 (flush between timed launches) vs the old L2-hot ranking (FOP_TUNE_HOT=1)
+for op in bert_layernorm cfg4a cfg4b bert_softmax cfg1; do
+timeout 600 python tools/sweep.py $op "" "opt:autotune=1" "opt:autotune=1,FOP_TUNE_HOT=1" >> gpurun_out/sweep_tunecold.log 2>&1
+done
+echo sweep=$?
+python - <<'PY'
+import json
+for l in open("gpurun_out/sweep_tunecold.log"):
+    if l.startswith("{"):
+        d=json.loads(l); print(d["op"], d["variant"], round(d.get("us_median",0),2), round(d.get("GBs_median",0)), d.get("selected", ""), d.get("error",""))
+    else: print(l.rstrip()[:200])
+PY
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu_s3f.log 2>&1; echo pytest=$?; tail -2 gpurun_out/pytest_gpu_s3f.log
+python bench.py > gpurun_out/bench_s3f.log 2>&1; echo bench=$?
+python - <<'PY'
+import json
+d=json.loads(open("gpurun_out/bench_s3f.log").read().strip().splitlines()[-1])
+print(d["value"], d["ms_per_step"])
+for k,v in d["config"]["per_op"].items(): print(k, v["kernel"], v["grid"], v["block"], round(v["GB_s"]), v["steady"] and round(v["steady"]["GB_s"]))
+PY

@@ -48,17 +48,19 @@ def main():
                 env[k] = val
         old = {k: os.environ.get(k) for k in env}
         os.environ.update(env)
-        try:
-            op = FusedOp(d, **opts)
-        except Exception as e:
-            print(json.dumps({"op": name, "variant": v, "error": str(e)[:300]}), flush=True)
-            continue
-        finally:
+        def restore():
             for k, val in old.items():
                 if val is None:
                     os.environ.pop(k, None)
                 else:
                     os.environ[k] = val
+        try:
+            op = FusedOp(d, **opts)
+        except Exception as e:
+            restore()
+            print(json.dumps({"op": name, "variant": v, "error": str(e)[:300]}), flush=True)
+            continue
+        # run-time knobs (FOP_TUNE_HOT, ...) stay set until the variant is timed
         for i in range(5):
             op.run(sets[i % copies])
         torch.cuda.synchronize()
@@ -73,10 +75,13 @@ def main():
             torch.cuda.synchronize()
             per.append(s.elapsed_time(e) / n)
         med = statistics.median(per)
+        restore()
         li = op.info()["launches"][0]
+        sel = op.selected(0)
         print(json.dumps({"op": name, "variant": v, "us_median": med * 1e3, "us_min": min(per) * 1e3,
                           "GBs_median": nbytes / med / 1e6, "GBs_best": nbytes / min(per) / 1e6,
-                          "grid": li["grid"], "class": li["class"], "width": li["width"], "copies": copies}),
+                          "grid": li["grid"], "class": li["class"], "width": li["width"], "copies": copies,
+                          "selected": list(sel)}),
               flush=True)
 
 
