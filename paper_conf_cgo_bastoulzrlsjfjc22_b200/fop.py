@@ -185,6 +185,11 @@ def span_elems(t):
 ESIZE = {"f32": 4, "f16": 2, "bf16": 2, "i32": 4}
 
 
+def _torch_dtype(name):
+    import torch
+    return {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16, "i32": torch.int32}[name]
+
+
 def marshal(desc):
     """dict form (workloads/) -> fop_desc."""
     d = Desc()
@@ -370,6 +375,27 @@ class FusedOp:
             self._ws[key] = torch.zeros(n, dtype=torch.uint8, device=device)  # zero-filled (fop.h)
         return self._ws[key]
 
+    def _check_tensor(self, n, t, where):
+        """A buffer handed to the C ABI must hold the descriptor's dtype and every
+        element the descriptor addresses from its base pointer (the library sees
+        pointers only, so this is the last place a short buffer can be caught)."""
+        chk = self.__dict__.get("_chk")
+        if chk is None:   # per tensor: torch dtype and bytes addressed from the base pointer
+            chk = self._chk = {m: (_torch_dtype(sp["dtype"]), span_elems(sp) * ESIZE[sp["dtype"]])
+                               for m, sp in self.desc["tensors"].items()}
+        want, need = chk[n]
+        if t.dtype is not want:
+            if not hasattr(t, "untyped_storage"):
+                raise TypeError(f"tensor {n!r}: expected a torch.Tensor, got {type(t).__name__}")
+            raise TypeError(f"tensor {n!r}: dtype {t.dtype}, the descriptor says "
+                            f"{self.desc['tensors'][n]['dtype']} ({want})")
+        if t.is_cuda != (where == "cuda"):
+            raise ValueError(f"tensor {n!r} is on {t.device}, expected a {'CUDA' if where == 'cuda' else 'host'} tensor")
+        have = t.untyped_storage().nbytes() - t.storage_offset() * t.element_size()
+        if need > have:
+            raise ValueError(f"tensor {n!r}: the descriptor addresses {need} bytes from its base pointer, "
+                             f"the buffer holds {have}")
+
     def _ptrs(self, tensors):
         arr = (C.c_void_p * len(self.names))()
         dev = None
@@ -380,9 +406,18 @@ class FusedOp:
                     raise ValueError(f"tensor {n!r} missing")
                 arr[i] = None
                 continue
+            self._check_tensor(n, t, "cuda")
+            if dev is not None and t.device != dev:
+                raise ValueError(f"tensor {n!r} is on {t.device}, the others on {dev}")
             arr[i] = t.data_ptr()
             dev = t.device
         return arr, dev
+
+    def _check_workspace(self, ws, dev):
+        if ws is not None and self.workspace_bytes:
+            have = ws.untyped_storage().nbytes() - ws.storage_offset() * ws.element_size()
+            if have < self.workspace_bytes or ws.device != dev:
+                raise ValueError(f"workspace: need {self.workspace_bytes} bytes on {dev}, got {have} on {ws.device}")
 
     def run(self, tensors, workspace=None, stream=None, peers=None):
         """Enqueue the fused operator on `stream` (default: torch's current stream).
@@ -390,6 +425,7 @@ class FusedOp:
         import torch
         arr, dev = self._ptrs(tensors)
         ws = workspace if workspace is not None else self._workspace(dev)
+        self._check_workspace(ws, dev)
         if stream is None:
             stream = torch.cuda.current_stream(dev)
         if peers is not None:
@@ -403,11 +439,9 @@ class FusedOp:
         """End to end: H2D copies of inputs from pinned `host`, run, D2H of outputs."""
         import torch
         arr, dev = self._ptrs(device_tensors)
-        harr = (C.c_void_p * len(self.names))()
-        for i, n in enumerate(self.names):
-            h = host.get(n)
-            harr[i] = None if h is None else h.data_ptr()
+        harr = self._host_ptrs(host)
         ws = workspace if workspace is not None else self._workspace(dev)
+        self._check_workspace(ws, dev)
         if stream is None:
             stream = torch.cuda.current_stream(dev)
         _check(_lib.fop_run_host(self._h, harr, arr, len(self.names),
@@ -417,6 +451,8 @@ class FusedOp:
         harr = (C.c_void_p * len(self.names))()
         for i, n in enumerate(self.names):
             h = host.get(n)
+            if h is not None:
+                self._check_tensor(n, h, "host")
             harr[i] = None if h is None else h.data_ptr()
         return harr
 
@@ -440,6 +476,7 @@ def run_host_many(items, stream=None):
         dev = dev or d
         harr = op._host_ptrs(host)
         w = it[3] if len(it) > 3 and it[3] is not None else op._workspace(d)
+        op._check_workspace(w, d)
         keep += [arr, harr]
         plans[k] = op._h
         hp[k] = C.cast(harr, C.POINTER(C.c_void_p))

@@ -213,3 +213,27 @@ def test_ragged_and_small_shapes_compile(desc):
         assert len(op.cubin(i)) > 0
     for opts in ({"force_width": 1}, {"coalesce_order": "memory"}, {"max_vec_bytes": 32}):
         FusedOp(desc, **opts)
+
+
+def test_binding_rejects_wrong_buffers_before_the_abi():
+    """The C ABI sees base pointers only: the binding checks dtype, device and
+    that every element the descriptor addresses lies inside the buffer."""
+    import torch
+    d = W.cfg4a(2, 64, 768)
+    op = FusedOp(d, jit=0)
+    good = {n: torch.zeros(max(1, pkg.fop.span_elems(t)), dtype={"f16": torch.float16, "f32": torch.float32}[t["dtype"]])
+            for n, t in d["tensors"].items() if t["role"] != "temp"}
+    op._host_ptrs(good)                       # host buffers of the right size pass
+    short = dict(good, x=torch.zeros(10, dtype=torch.float16))
+    with pytest.raises(ValueError, match="addresses"):
+        op._host_ptrs(short)
+    wrong = dict(good, x=torch.zeros(good["x"].numel(), dtype=torch.float32))
+    with pytest.raises(TypeError, match="dtype"):
+        op._host_ptrs(wrong)
+    offset = dict(good, x=good["x"][1:])      # a view one element in: one element short
+    with pytest.raises(ValueError, match="addresses"):
+        op._host_ptrs(offset)
+    with pytest.raises(ValueError, match="CUDA"):
+        op.run(good)                          # host tensors where device tensors are required
+    with pytest.raises(ValueError, match="missing"):
+        op.run({n: t for n, t in good.items() if n != "x"})

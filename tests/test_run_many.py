@@ -23,8 +23,9 @@ class _S:
     cuda_stream = 0
 
 
-def test_run_many_rejects_peer_plans_before_launch():
+def test_run_many_rejects_peer_plans_before_launch(monkeypatch):
     op = FusedOp(W.cfg4b(256, 64), peer_world=2, peer_loop="r", jit=0)
+    monkeypatch.setattr(op, "_check_tensor", lambda *a: None)   # host tensors stand in for device pointers
     t = {"x": torch.zeros(256 * 64, dtype=torch.float16), "out": torch.zeros(64)}
     with pytest.raises(FopError, match="fop_run_peer"):
         run_many([(op, t, torch.zeros(max(1, op.workspace_bytes), dtype=torch.uint8))], stream=_S())
