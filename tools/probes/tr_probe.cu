@@ -24,6 +24,18 @@ __device__ __forceinline__ uint4 ldg_stream(const void* p) {
   asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
   return v;
 }
+// with an L2 prefetch-size hint (PF = 128 or 256 bytes)
+template <int PF>
+__device__ __forceinline__ uint4 ldg_pf(const void* p) {
+  uint4 v;
+  if constexpr (PF == 256)
+    asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+  else if constexpr (PF == 128)
+    asm volatile("ld.global.nc.L1::no_allocate.L2::128B.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+  else
+    v = ldg_stream(p);
+  return v;
+}
 
 // 8x8 f16 transpose of rows r[0..7] (each 8 halves) scaled by s -> o[b] = column b
 __device__ __forceinline__ void tr8(const uint4 (&r)[8], uint4 (&o)[8], float s) {
@@ -42,7 +54,7 @@ __device__ __forceinline__ void tr8(const uint4 (&r)[8], uint4 (&o)[8], float s)
   }
 }
 
-template <int U>
+template <int U, int PF = 0>
 __global__ void __launch_bounds__(256, 1) tr_A(const __half* __restrict__ x, __half* __restrict__ y, float s) {
   const unsigned tid = blockIdx.x * 256u + threadIdx.x, nth = gridDim.x * 256u;
   constexpr unsigned TRH = 98u / U;   // hw tiles of 8: 392 = TRH x U x 4
@@ -59,7 +71,7 @@ __global__ void __launch_bounds__(256, 1) tr_A(const __half* __restrict__ x, __h
     for (int u = 0; u < U; ++u) {
       const unsigned hw0 = ((tr_hi * U + u) * 4u + tr_lo) * 8u;
 #pragma unroll
-      for (int a = 0; a < 8; ++a) r[u][a] = ldg_stream(x + ((size_t)n * C + c0 + a) * HW + hw0);
+      for (int a = 0; a < 8; ++a) r[u][a] = ldg_pf<PF>(x + ((size_t)n * C + c0 + a) * HW + hw0);
     }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
@@ -236,6 +248,10 @@ int main() {
       }
     });
   }
+  timeit("A U=2 L2::128B", [&](int r) { tr_A<2, 128><<<sms, 256>>>(xs[r], ys[r], 0.5f); });
+  timeit("A U=2 L2::256B", [&](int r) { tr_A<2, 256><<<sms, 256>>>(xs[r], ys[r], 0.5f); });
+  timeit("A U=1 2xSM L2::256B", [&](int r) { tr_A<1, 256><<<sms * 2, 256>>>(xs[r], ys[r], 0.5f); });
+  timeit("A U=2 (again)", [&](int r) { tr_A<2><<<sms, 256>>>(xs[r], ys[r], 0.5f); });
   tr_E<3><<<sms * 3, 256>>>(xs[0], ys[1], 0.5f); CK(cudaDeviceSynchronize());
   CK(cudaMemcpy(rc.data(), ys[1], bytes, cudaMemcpyDeviceToHost));
   bad = 0;
