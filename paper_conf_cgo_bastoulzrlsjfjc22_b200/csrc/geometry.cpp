@@ -208,7 +208,32 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       collapse_into(p, acc, ord, L.kl);
       if (L.virt_vec) L.kl[0].extent = 1;   // fully sequential statement (row N3)
     } else {
+      // d_v first absorbs the loops that continue it contiguously for every
+      // access, wherever they sit in the order (NHWC -> NCHW: w then h is one
+      // run on both sides, d_v = hw, not w alone), then d_r absorbs its own
+      std::vector<int> vseg = {ord[0]}, others(ord.begin() + 2, ord.end());
+      int64_t vext = p.desc.extent[ord[0]];
+      for (bool grew = true; grew;) {
+        grew = false;
+        for (size_t q = 0; q < others.size() && !grew; q++) {
+          bool ok = true;
+          for (const Affine* a : acc)
+            if (a->coef[others[q]] != a->coef[ord[0]] * vext) ok = false;
+          if (ok) {
+            vseg.push_back(others[q]);
+            vext *= p.desc.extent[others[q]];
+            others.erase(others.begin() + q);
+            grew = true;
+          }
+        }
+      }
+      L.kl.clear();
+      collapse_into(p, acc, vseg, L.kl);
+      seg1.assign(1, ord[1]);
+      seg1.insert(seg1.end(), others.begin(), others.end());
       collapse_into(p, acc, seg1, L.kl);
+      L.order = vseg;
+      L.order.insert(L.order.end(), seg1.begin(), seg1.end());
     }
     L.nsplit = L.kclass == FOP_CLASS_TRANSPOSE ? 2 : 1;
   } else {

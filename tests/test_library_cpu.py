@@ -237,3 +237,16 @@ def test_binding_rejects_wrong_buffers_before_the_abi():
         op.run(good)                          # host tensors where device tensors are required
     with pytest.raises(ValueError, match="missing"):
         op.run({n: t for n, t in good.items() if n != "x"})
+
+
+def test_transpose_vector_loop_absorbs_contiguous_continuations():
+    """NHWC -> NCHW: the store side is contiguous over w then h, and so is the
+    load side's h after w, so the kernel's d_v is the collapsed h*w (3136
+    elements = 392 tiles of 8), not w alone (7 tiles, a ragged warp)."""
+    op = FusedOp(W.nhwc_to_nchw(256, 56, 56, 256), jit=0, autotune=0)
+    li = op.info()["launches"][0]
+    assert (li["class"], li["width"], li["read_width"]) == ("transpose", 8, 8)
+    assert "if (tv >= 392u) continue;" in op.source()
+    # NCHW -> NHWC keeps d_v = c alone and collapses h, w on the read side
+    src = FusedOp(W.cfg3(), jit=0, autotune=0).source()
+    assert "if (tv >= 32u) continue;" in src and "tr_0 < 392u" in src

@@ -204,6 +204,17 @@ def test_transpose_roundtrip_on_gpu():
     assert_bitexact(back["out"], x["x"], "roundtrip")
 
 
+@pytest.mark.parametrize("dims", [(2, 56, 56, 256), (3, 7, 9, 64), (1, 14, 14, 40), (2, 5, 8, 24)])
+def test_nhwc_to_nchw_bitexact(dims):
+    """The reverse layout change: d_v absorbs h after w (one contiguous run of
+    H*W on both sides), so the store tiles span whole NCHW planes."""
+    d = W.nhwc_to_nchw(*dims, s=0.5)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.info()["launches"][0]["class"] == "transpose"
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+
+
 # ---------------------------------------------------------------- ROW_REDUCE
 def _check_rowstats(d, x, got):
     ref = O.run(d, x)
