@@ -1062,6 +1062,102 @@ struct Gen {
     footer();
   }
 
+  // ------------------------------------------------------------ TRANSPOSE via shared memory
+  // For d_r rows too short or odd to carry vectors (a 7x7 plane: 49
+  // elements, 98 B rows) whose d_v rows are adjacent in the load tensor: a
+  // tile of TV whole rows is ONE contiguous chunk of TV*E[d_r] elements.
+  // Phase 1: the CTA copies it into shared memory with 16 B vector loads.
+  // Phase 2: each thread reads W elements down a column (one per row, fixed
+  // d_r index), evaluates the statement and stores a W-vector along d_v;
+  // consecutive lanes take consecutive d_v chunks, so a warp's stores are
+  // contiguous.  Several CTAs per SM overlap one's loads with another's
+  // read-out.
+  void gen_transpose_smem() {
+    const XStmt& x = L.stmts[0];
+    const int W = L.width;
+    const int64_t TV = L.tr_tv, ER = L.kl[1].extent, NVB = L.kl[0].extent / TV;
+    const Affine& ta = L.loads[L.trans_load];
+    const int esi = es(ta.tensor), eso = es(x.write.tensor);
+    const int64_t tile_bytes = TV * ER * esi, nvec = tile_bytes / 16, nj = TV / W, nout = ER * nj;
+    const bool raw = x.move && esi == eso;
+    const std::string dti = dtn(d.t[ta.tensor].dtype), dto = dtn(x.out_dtype);
+    header("TRANSPOSE via shared memory (flat tile of TV rows x E[d_r] in, vectors along d_v out)", 1);
+    o.l("__shared__ __align__(16) unsigned char fop_tile[" + num(tile_bytes) + "];");
+    for (size_t k = 0; k < L.loads.size(); k++) {   // constants (eligibility: no loop in the access)
+      if ((int)k == L.trans_load) continue;
+      const Affine& a = L.loads[k];
+      o.l("const float L" + num(k) + " = fop::sload<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + pol(a, true) +
+          ">(" + ptr(a.tensor, affine(a, {})) + ");");
+    }
+    o.l("#pragma unroll 1");
+    o.l("for (idx_t g = blockIdx.x; g < (idx_t)" + num(L.work) + "ull; g += gridDim.x) {");
+    o.ind++;
+    o.l("[[maybe_unused]] idx_t t = g;");
+    o.l("const idx_t vb = t % " + num(NVB) + "u; t /= " + num(NVB) + "u;");
+    std::vector<std::pair<int, std::string>> outer;
+    decompose("t", 2, (int)L.kl.size(), "", outer);
+    std::vector<std::pair<int, std::string>> in_its = {{0, "vb * " + num(TV) + "u"}};
+    in_its.insert(in_its.end(), outer.begin(), outer.end());
+    o.l("const char* src = " + ptr(ta.tensor, affine(ta, in_its)) + ";");
+    o.l("__syncthreads();   // the previous tile is read out");
+    o.l("#pragma unroll 4");
+    o.l("for (unsigned q = threadIdx.x; q < " + num(nvec) + "u; q += " + num(L.block) + "u) {");
+    o.l("  u32 w[4];");
+    o.l("  fop::ldraw<16, " + pol(ta, false) + ">(w, src + q * 16u);");
+    o.l("  *reinterpret_cast<uint4*>(fop_tile + q * 16u) = make_uint4(w[0], w[1], w[2], w[3]);");
+    o.l("}");
+    o.l("__syncthreads();");
+    o.l("#pragma unroll 2");
+    o.l("for (unsigned q = threadIdx.x; q < " + num(nout) + "u; q += " + num(L.block) + "u) {");
+    o.ind++;
+    o.l("const unsigned j = q % " + num(nj) + "u, r = q / " + num(nj) + "u;");
+    std::vector<std::pair<int, std::string>> out_its = {{0, "(vb * " + num(TV) + "u + j * " + num(W) + "u)"},
+                                                        {1, "r"}};
+    out_its.insert(out_its.end(), outer.begin(), outer.end());
+    std::string dst = ptr(x.write.tensor, affine(x.write, out_its));
+    std::string cell = "fop_tile + ((j * " + num(W) + "u + e) * " + num(ER) + "u + r) * " + num(esi) + "u";
+    if (raw) {
+      o.l("u32 O[" + num(W) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) O[e] = " +
+          std::string(esi == 2 ? "*reinterpret_cast<const u16*>(" : "*reinterpret_cast<const u32*>(") + cell + ");");
+      o.l("fop::vstore_raw<" + num(eso) + ", " + num(W) + ", " + num(L.store_cb[0]) + ", " + spol() + ">(" + dst +
+          ", O);");
+    } else {
+      std::string lt = "L" + num(L.trans_load);
+      o.l("float " + lt + "[" + num(W) + "];");
+      o.l("#pragma unroll");
+      std::string rd = d.t[ta.tensor].dtype == FOP_F16    ? "fop::h2f(*reinterpret_cast<const u16*>(" + cell + "))"
+                       : d.t[ta.tensor].dtype == FOP_BF16 ? "fop::b2f(*reinterpret_cast<const u16*>(" + cell + "))"
+                                                          : "*reinterpret_cast<const float*>(" + cell + ")";
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) " + lt + "[e] = " + rd + ";");
+      DagCtx c;
+      c.tag = "";
+      c.ev = "e";
+      const int tl = L.trans_load;
+      c.load_varies = [tl](int k) { return k == tl; };
+      c.load = [tl](int k, const std::string& e) { return "L" + num(k) + (k == tl ? "[" + e + "]" : std::string()); };
+      c.fwd = [&](int, const std::string&) { return std::string("0.f"); };
+      c.scalar = [&](int) { return std::string("0.f"); };
+      auto var = varies(x, c);
+      emit_nodes(o, x, var, false, c);
+      o.l("float O[" + num(W) + "];");
+      Sink sk;
+      sk.scalar = [&](const std::string& v) { o.l("O[e] = " + v + ";"); };
+      sk.pair = [&](const std::string& v, const std::string& pp) {
+        o.l("fop::upk(" + v + ", O[2 * " + pp + "], O[2 * " + pp + " + 1]);");
+      };
+      emit_elems(o, x, var, c, W, sk);
+      o.l("fop::vstore<" + dto + ", " + num(W) + ", " + num(L.store_cb[0]) + ", " + spol() + ">(" + dst + ", O);");
+    }
+    (void)dti;
+    o.ind--;
+    o.l("}");
+    o.ind--;
+    o.l("}");
+    footer();
+  }
+
   // ------------------------------------------------------------ TRANSPOSE via TMA
   // 64x64 tiles of 16-bit data.  Per CTA (128 threads = two 64-thread tile
   // groups): a pipeline of S smem stages, each holding two 8 KB input tiles
@@ -2048,11 +2144,12 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
     maxv = std::max(maxv, span + 64);
   }
   g.idx = maxv < (int64_t(1) << 31) ? "unsigned" : "unsigned long long";
-  L.name = std::string("fop_") + class_name(L.kclass) + (L.tma ? "_tma" : "") + "_k" + std::to_string(launch_index) +
+  L.name = std::string("fop_") + class_name(L.kclass) + (L.tma ? "_tma" : (L.tr_smem ? "_smem" : "")) + "_k" + std::to_string(launch_index) +
            (L.scalar_variant ? "_narrow" : "") + L.name_suffix;
   switch (L.kclass) {
     case FOP_CLASS_TRANSPOSE:
       if (L.tma) g.gen_transpose_tma();
+      else if (L.tr_smem) g.gen_transpose_smem();
       else g.gen_transpose();
       break;
     case FOP_CLASS_ROW_REDUCE: g.gen_row(); break;

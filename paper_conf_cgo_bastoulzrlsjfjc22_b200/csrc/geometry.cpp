@@ -157,6 +157,12 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       break;
     case FOP_CLASS_TRANSPOSE:
       if (L.tma) break;
+      if (L.tr_smem) {
+        v.push_back({{"FOP_TR_SMEM_MINB", 2}});
+        v.push_back({{"FOP_TR_SMEM_MINB", 6}});
+        v.push_back({{"FOP_TR_SMEM_BYTES", 16384}, {"FOP_TR_SMEM_MINB", 8}});
+        break;
+      }
       v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 2}});
       v.push_back({{"FOP_TR_U", 2}, {"FOP_TR_MINB", 2}});
       v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 3}});
@@ -293,7 +299,35 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     if (L.scalar_variant) wr = 1;
     while (wr > 1 && L.kl[1].extent % wr) wr /= 2;
     L.read_width = wr;
-    if (W == 1 || wr == 1) {  // degenerate tile: plain elementwise with gathers
+    L.tr_smem = 0;
+    if (W >= 2 && wr == 1 && !L.scalar_variant && geometry_knob(L, "FOP_TR_SMEM", 1)) {
+      // d_r cannot carry vectors (odd extent, e.g. a 7x7 plane: 49), but when
+      // consecutive d_v rows are adjacent in the load tensor (coef(d_v) ==
+      // E[d_r]) a tile of TV full rows is one flat contiguous chunk: load it
+      // with 16 B vectors into shared memory and store vectors along d_v
+      // (ResNet stage-4 NCHW [N,2048,7,7] -> NHWC)
+      const int64_t ER = L.kl[1].extent, EVx = L.kl[0].extent;
+      const Affine& t = L.loads[L.trans_load];
+      const int esi = esize(d.t[t.tensor].dtype);
+      bool ok = L.stmts.size() == 1 && coef(L, t, 1) == 1 && coef(L, t, 0) == ER && (t.base * esi) % 16 == 0;
+      for (size_t k = 2; k < L.kl.size() && ok; k++) ok = (coef(L, t, (int)k) * esi) % 16 == 0;
+      for (size_t k = 0; k < L.loads.size() && ok; k++) {
+        if ((int)k == L.trans_load) continue;
+        for (size_t q = 0; q < L.kl.size(); q++) ok &= coef(L, L.loads[k], (int)q) == 0;   // constants only
+      }
+      int64_t TV = 0;
+      const int64_t cap = std::min<int64_t>(EVx, geometry_knob(L, "FOP_TR_SMEM_BYTES", 32768) / (ER * esi));
+      for (int64_t tv = cap - cap % W; ok && tv >= W; tv -= W)
+        if (EVx % tv == 0 && (tv * ER * esi) % 16 == 0) {
+          TV = tv;
+          break;
+        }
+      if (TV) {
+        L.tr_smem = 1;
+        L.tr_tv = TV;
+      }
+    }
+    if ((W == 1 || wr == 1) && !L.tr_smem) {  // degenerate tile: plain elementwise with gathers
       L.kclass = FOP_CLASS_EW;
       L.read_loop = -1;
       L.trans_load = -1;
@@ -327,6 +361,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     int t = L.stmts[k].write.tensor;
     L.align[t] = std::max({L.align[t], L.store_cb[k], esize(d.t[t].dtype)});
   }
+  if (L.tr_smem) L.align[L.loads[L.trans_load].tensor] = std::max(L.align[L.loads[L.trans_load].tensor], 16);
 
   // ---- a5: launch geometry.  Grid-stride classes launch exactly the blocks
   // that are resident at once (SMs x minblocks, guaranteed by
@@ -369,6 +404,17 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       int64_t need = (L.work + (int64_t)L.block * L.unroll - 1) / ((int64_t)L.block * L.unroll);
       L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
     }
+  } else if (L.kclass == FOP_CLASS_TRANSPOSE && L.tr_smem) {
+    // one tile (TV x E[d_r]) per CTA iteration, several CTAs per SM so one
+    // CTA's loads overlap another's shared-memory read-out and stores
+    for (size_t k = 2; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
+    L.block = 256;
+    L.unroll = 1;
+    L.tma = 0;
+    L.minblocks = knob("FOP_TR_SMEM_MINB", 4);
+    L.work = (L.kl[0].extent / L.tr_tv) * prod_rest;
+    L.grid = std::max<int64_t>(1, std::min<int64_t>(L.work, (int64_t)sms * L.minblocks));
+    L.smem = (size_t)L.tr_tv * L.kl[1].extent * esize(d.t[L.loads[L.trans_load].tensor].dtype);
   } else if (L.kclass == FOP_CLASS_TRANSPOSE) {
     for (size_t k = 2; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
     int64_t ntv = EV / W, ntr = L.kl[1].extent / L.read_width;

@@ -250,3 +250,20 @@ def test_transpose_vector_loop_absorbs_contiguous_continuations():
     # NCHW -> NHWC keeps d_v = c alone and collapses h, w on the read side
     src = FusedOp(W.cfg3(), jit=0, autotune=0).source()
     assert "if (tv >= 32u) continue;" in src and "tr_0 < 392u" in src
+
+
+def test_odd_plane_transpose_is_staged_through_shared_memory():
+    """[N,2048,7,7] NCHW -> NHWC: d_r = h*w = 49 cannot carry vectors, the
+    2048 rows of 49 are adjacent, so the plan stages flat tiles through
+    shared memory instead of falling back to a gathering elementwise kernel."""
+    op = FusedOp(W.cfg3(256, 2048, 7, 7), jit=0, autotune=0)
+    li = op.info()["launches"][0]
+    assert (li["class"], li["width"], li["read_width"]) == ("transpose", 8, 1)
+    src = op.source()
+    assert "fop_transpose_smem_k0" in src and "__shared__ __align__(16) unsigned char fop_tile[25088]" in src
+    # the narrow (misaligned-pointer) variant and an opt-out still gather
+    os.environ["FOP_TR_SMEM"] = "0"
+    try:
+        assert FusedOp(W.cfg3(256, 2048, 7, 7), jit=0, autotune=0).info()["launches"][0]["class"] == "ew"
+    finally:
+        del os.environ["FOP_TR_SMEM"]

@@ -204,15 +204,39 @@ def test_transpose_roundtrip_on_gpu():
     assert_bitexact(back["out"], x["x"], "roundtrip")
 
 
-@pytest.mark.parametrize("dims", [(2, 56, 56, 256), (3, 7, 9, 64), (1, 14, 14, 40), (2, 5, 8, 24)])
-def test_nhwc_to_nchw_bitexact(dims):
+@pytest.mark.parametrize("dims,cls", [((2, 56, 56, 256), "transpose"), ((3, 7, 9, 64), "ew"),
+                                      ((1, 14, 14, 40), "transpose"), ((2, 5, 8, 24), "transpose")])
+def test_nhwc_to_nchw_bitexact(dims, cls):
     """The reverse layout change: d_v absorbs h after w (one contiguous run of
-    H*W on both sides), so the store tiles span whole NCHW planes."""
+    H*W on both sides), so the store tiles span whole NCHW planes.  An odd
+    H*W (63) cannot carry store vectors: elementwise with gathers."""
     d = W.nhwc_to_nchw(*dims, s=0.5)
     x = W.make_inputs(d)
     got, op = run_gpu(d, x)
-    assert op.info()["launches"][0]["class"] == "transpose"
+    assert op.info()["launches"][0]["class"] == cls
     assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+
+
+@pytest.mark.parametrize("dims,dtype", [((2, 2048, 7, 7), "f16"), ((3, 64, 3, 3), "f16"), ((2, 40, 5, 7), "f32"),
+                                        ((3, 24, 7, 7), "bf16"), ((2, 1024, 1, 7), "f16")])
+def test_transpose_odd_planes_via_shared_memory(dims, dtype):
+    """NCHW -> NHWC with an odd H*W (a 7x7 plane: 98 B rows cannot carry
+    vectors): flat tiles through shared memory, bit-exact."""
+    d = W.cfg3(*dims, dtype=dtype)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.selected(0)[0].startswith("fop_transpose_smem")
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+
+
+def test_transpose_smem_pure_move_keeps_nan_payloads():
+    d = W.cfg3(2, 64, 7, 7, s=1.0)
+    d["stmts"][0]["expr"] = [("load", 0)]
+    d["tensors"]["x"]["init"] = ("special", 4)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.selected(0)[0].startswith("fop_transpose_smem")
+    assert np.array_equal(got["out"].view(np.uint16), O.run(d, x)["out"].view(np.uint16))
 
 
 # ---------------------------------------------------------------- ROW_REDUCE
