@@ -1073,6 +1073,10 @@ struct Gen {
   // contiguous.  Several CTAs per SM overlap one's loads with another's
   // read-out.
   void gen_transpose_smem() {
+    if (L.tr_smem == 2) {
+      gen_transpose_smem_out();
+      return;
+    }
     const XStmt& x = L.stmts[0];
     const int W = L.width;
     const int64_t TV = L.tr_tv, ER = L.kl[1].extent, NVB = L.kl[0].extent / TV;
@@ -1151,6 +1155,100 @@ struct Gen {
       o.l("fop::vstore<" + dto + ", " + num(W) + ", " + num(L.store_cb[0]) + ", " + spol() + ">(" + dst + ", O);");
     }
     (void)dti;
+    o.ind--;
+    o.l("}");
+    o.ind--;
+    o.l("}");
+    footer();
+  }
+
+  // The mirror of gen_transpose_smem: d_v rows too short or odd to carry
+  // store vectors (an input layer's C = 3, NHWC -> NCHW of a 7x7 plane) while
+  // the output rows are adjacent, so a tile of TR output rows (d_r positions)
+  // x all of d_v is ONE contiguous chunk of the output.  Phase 1 loads the E[d_v]
+  // input rows of the tile with vectors along d_r into shared memory [v][r];
+  // phase 2 writes the flat output chunk with 16 B vectors, each element read
+  // from shared memory at (v, r) = (f % E[d_v], f / E[d_v]).
+  void gen_transpose_smem_out() {
+    const XStmt& x = L.stmts[0];
+    const int64_t TR = L.tr_tv, EV = L.kl[0].extent, ER = L.kl[1].extent, NRB = ER / TR;
+    const Affine& ta = L.loads[L.trans_load];
+    const int esi = es(ta.tensor), eso = es(x.write.tensor);
+    const int WR = L.read_width, OW = 16 / eso;
+    const int64_t nin = EV * (TR / WR), nout = TR * EV / OW;
+    const bool raw = x.move && esi == eso;
+    header("TRANSPOSE via shared memory (vectors along d_r in, flat tile of TR output rows x E[d_v] out)", 1);
+    o.l("__shared__ __align__(16) unsigned char fop_tile[" + num(TR * EV * esi) + "];");
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      if ((int)k == L.trans_load) continue;
+      const Affine& a = L.loads[k];
+      o.l("const float L" + num(k) + " = fop::sload<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + pol(a, true) +
+          ">(" + ptr(a.tensor, affine(a, {})) + ");");
+    }
+    o.l("#pragma unroll 1");
+    o.l("for (idx_t g = blockIdx.x; g < (idx_t)" + num(L.work) + "ull; g += gridDim.x) {");
+    o.ind++;
+    o.l("[[maybe_unused]] idx_t t = g;");
+    o.l("const idx_t rb = t % " + num(NRB) + "u; t /= " + num(NRB) + "u;");
+    std::vector<std::pair<int, std::string>> outer;
+    decompose("t", 2, (int)L.kl.size(), "", outer);
+    std::vector<std::pair<int, std::string>> in_its = {{0, "v"}, {1, "(rb * " + num(TR) + "u + rc * " + num(WR) + "u)"}};
+    in_its.insert(in_its.end(), outer.begin(), outer.end());
+    o.l("__syncthreads();   // the previous tile is written out");
+    o.l("#pragma unroll 4");
+    o.l("for (unsigned q = threadIdx.x; q < " + num(nin) + "u; q += " + num(L.block) + "u) {");
+    o.ind++;
+    o.l("const unsigned rc = q % " + num(TR / WR) + "u, v = q / " + num(TR / WR) + "u;");
+    o.l("u32 w[" + num(WR * esi / 4) + "];");
+    o.l("fop::vload_words<" + std::string(dtn(d.t[ta.tensor].dtype)) + ", " + num(WR) + ", " +
+        num(L.load_cb_r[L.trans_load]) + ", " + pol(ta, false) + ">(w, " + ptr(ta.tensor, affine(ta, in_its)) + ");");
+    o.l("#pragma unroll");
+    o.l("for (int c = 0; c < " + num(WR * esi / 4) + "; ++c) reinterpret_cast<u32*>(fop_tile + (v * " + num(TR) +
+        "u + rc * " + num(WR) + "u) * " + num(esi) + "u)[c] = w[c];");
+    o.ind--;
+    o.l("}");
+    o.l("__syncthreads();");
+    std::vector<std::pair<int, std::string>> out_its = {{1, "rb * " + num(TR) + "u"}};
+    out_its.insert(out_its.end(), outer.begin(), outer.end());
+    o.l("char* dst = " + ptr(x.write.tensor, affine(x.write, out_its)) + ";");
+    o.l("#pragma unroll 2");
+    o.l("for (unsigned q = threadIdx.x; q < " + num(nout) + "u; q += " + num(L.block) + "u) {");
+    o.ind++;
+    std::string cell = "fop_tile + (((q * " + num(OW) + "u + e) % " + num(EV) + "u) * " + num(TR) + "u + (q * " +
+                       num(OW) + "u + e) / " + num(EV) + "u) * " + num(esi) + "u";
+    if (raw) {
+      o.l("u32 O[" + num(OW) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(OW) + "; ++e) O[e] = " +
+          std::string(esi == 2 ? "*reinterpret_cast<const u16*>(" : "*reinterpret_cast<const u32*>(") + cell + ");");
+      o.l("fop::vstore_raw<" + num(eso) + ", " + num(OW) + ", 16, " + spol() + ">(dst + q * 16u, O);");
+    } else {
+      std::string lt = "L" + num(L.trans_load);
+      o.l("float " + lt + "[" + num(OW) + "];");
+      o.l("#pragma unroll");
+      std::string rd = d.t[ta.tensor].dtype == FOP_F16    ? "fop::h2f(*reinterpret_cast<const u16*>(" + cell + "))"
+                       : d.t[ta.tensor].dtype == FOP_BF16 ? "fop::b2f(*reinterpret_cast<const u16*>(" + cell + "))"
+                                                          : "*reinterpret_cast<const float*>(" + cell + ")";
+      o.l("for (int e = 0; e < " + num(OW) + "; ++e) " + lt + "[e] = " + rd + ";");
+      DagCtx c;
+      c.tag = "";
+      c.ev = "e";
+      const int tl = L.trans_load;
+      c.load_varies = [tl](int k) { return k == tl; };
+      c.load = [tl](int k, const std::string& e) { return "L" + num(k) + (k == tl ? "[" + e + "]" : std::string()); };
+      c.fwd = [&](int, const std::string&) { return std::string("0.f"); };
+      c.scalar = [&](int) { return std::string("0.f"); };
+      auto var = varies(x, c);
+      emit_nodes(o, x, var, false, c);
+      o.l("float O[" + num(OW) + "];");
+      Sink sk;
+      sk.scalar = [&](const std::string& v) { o.l("O[e] = " + v + ";"); };
+      sk.pair = [&](const std::string& v, const std::string& pp) {
+        o.l("fop::upk(" + v + ", O[2 * " + pp + "], O[2 * " + pp + " + 1]);");
+      };
+      emit_elems(o, x, var, c, OW, sk);
+      o.l("fop::vstore<" + std::string(dtn(x.out_dtype)) + ", " + num(OW) + ", 16, " + spol() + ">(dst + q * 16u, O);");
+    }
     o.ind--;
     o.l("}");
     o.ind--;

@@ -116,8 +116,9 @@ struct Launch {
   int width = 1;                  // W (elements along d_v)
   int read_loop = -1, read_width = 0;  // TRANSPOSE
   int trans_load = -1;            // TRANSPOSE: index into loads of the transposed access
-  int tr_smem = 0;                // TRANSPOSE staged through shared memory (rows of d_r too short/odd to vectorise)
-  int64_t tr_tv = 0;              // tr_smem: d_v extent of one tile (the tile is tr_tv x E[d_r], flat in the load tensor)
+  int tr_smem = 0;                // TRANSPOSE staged through shared memory: 1 = d_r rows cannot carry vectors (flat
+                                  // input tile), 2 = d_v rows cannot (flat output tile)
+  int64_t tr_tv = 0;              // tr_smem 1: d_v rows per tile (tile = tr_tv x E[d_r]); 2: d_r rows per tile
   int coal_loop = -1;
   std::vector<int> order;         // launch loop order, innermost first (before collapse)
   std::vector<int> seq;           // EW read-modify-write / recurrence: loops walked in order by each thread (outer first)

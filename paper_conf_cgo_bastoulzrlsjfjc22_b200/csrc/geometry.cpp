@@ -327,6 +327,35 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
         L.tr_tv = TV;
       }
     }
+    if (W == 1 && wr >= 2 && !L.scalar_variant && geometry_knob(L, "FOP_TR_SMEM", 1)) {
+      // the mirror case: d_v rows too short/odd for store vectors (an input
+      // layer's C = 3; NHWC -> NCHW of a 7x7 plane), but the output rows are
+      // adjacent (coef_out(d_r) == E[d_v]): a tile of TR whole output rows is
+      // one contiguous chunk of the output, written with 16 B vectors after
+      // the input rows were loaded with vectors along d_r
+      const int64_t ER = L.kl[1].extent, EVx = L.kl[0].extent;
+      const Affine& w = L.stmts[0].write;
+      const int eso = esize(L.stmts[0].out_dtype);
+      bool ok = L.stmts.size() == 1 && coef(L, w, 0) == 1 && coef(L, w, 1) == EVx && (w.base * eso) % 16 == 0;
+      for (size_t k = 2; k < L.kl.size() && ok; k++) ok = (coef(L, w, (int)k) * eso) % 16 == 0;
+      for (size_t k = 0; k < L.loads.size() && ok; k++) {
+        if ((int)k == L.trans_load) continue;
+        for (size_t q = 0; q < L.kl.size(); q++) ok &= coef(L, L.loads[k], (int)q) == 0;   // constants only
+      }
+      const int esi = esize(d.t[L.loads[L.trans_load].tensor].dtype);
+      const int64_t rowb = EVx * std::max(esi, eso);
+      int64_t TR = 0;
+      const int64_t cap = std::min<int64_t>(ER, geometry_knob(L, "FOP_TR_SMEM_BYTES", 32768) / rowb);
+      for (int64_t tr = cap - cap % wr; ok && tr >= wr; tr -= wr)
+        if (ER % tr == 0 && (tr * EVx * eso) % 16 == 0) {
+          TR = tr;
+          break;
+        }
+      if (TR) {
+        L.tr_smem = 2;
+        L.tr_tv = TR;
+      }
+    }
     if ((W == 1 || wr == 1) && !L.tr_smem) {  // degenerate tile: plain elementwise with gathers
       L.kclass = FOP_CLASS_EW;
       L.read_loop = -1;
@@ -361,7 +390,8 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     int t = L.stmts[k].write.tensor;
     L.align[t] = std::max({L.align[t], L.store_cb[k], esize(d.t[t].dtype)});
   }
-  if (L.tr_smem) L.align[L.loads[L.trans_load].tensor] = std::max(L.align[L.loads[L.trans_load].tensor], 16);
+  if (L.tr_smem == 1) L.align[L.loads[L.trans_load].tensor] = std::max(L.align[L.loads[L.trans_load].tensor], 16);
+  if (L.tr_smem == 2) L.align[L.stmts[0].write.tensor] = std::max(L.align[L.stmts[0].write.tensor], 16);
 
   // ---- a5: launch geometry.  Grid-stride classes launch exactly the blocks
   // that are resident at once (SMs x minblocks, guaranteed by
@@ -412,9 +442,15 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.unroll = 1;
     L.tma = 0;
     L.minblocks = knob("FOP_TR_SMEM_MINB", 4);
-    L.work = (L.kl[0].extent / L.tr_tv) * prod_rest;
+    const int esi = esize(d.t[L.loads[L.trans_load].tensor].dtype);
+    if (L.tr_smem == 1) {   // tiles of tr_tv d_v rows
+      L.work = (L.kl[0].extent / L.tr_tv) * prod_rest;
+      L.smem = (size_t)L.tr_tv * L.kl[1].extent * esi;
+    } else {                // tiles of tr_tv d_r positions (output rows)
+      L.work = (L.kl[1].extent / L.tr_tv) * prod_rest;
+      L.smem = (size_t)L.tr_tv * L.kl[0].extent * esi;
+    }
     L.grid = std::max<int64_t>(1, std::min<int64_t>(L.work, (int64_t)sms * L.minblocks));
-    L.smem = (size_t)L.tr_tv * L.kl[1].extent * esize(d.t[L.loads[L.trans_load].tensor].dtype);
   } else if (L.kclass == FOP_CLASS_TRANSPOSE) {
     for (size_t k = 2; k < L.kl.size(); k++) prod_rest *= L.kl[k].extent;
     int64_t ntv = EV / W, ntr = L.kl[1].extent / L.read_width;

@@ -267,3 +267,16 @@ def test_odd_plane_transpose_is_staged_through_shared_memory():
         assert FusedOp(W.cfg3(256, 2048, 7, 7), jit=0, autotune=0).info()["launches"][0]["class"] == "ew"
     finally:
         del os.environ["FOP_TR_SMEM"]
+
+
+def test_tiny_channel_transpose_writes_flat_output_tiles():
+    """NCHW [N,3,224,224] -> NHWC: c = 3 carries no store vector, the NHWC rows
+    of 3 channels are adjacent, so the plan loads vectors along h*w and writes
+    the output tile flat (the mirror of the odd-plane case)."""
+    op = FusedOp(W.cfg3(256, 3, 224, 224), jit=0, autotune=0)
+    li = op.info()["launches"][0]
+    assert (li["class"], li["width"], li["read_width"]) == ("transpose", 1, 8)
+    src = op.source()
+    assert "flat tile of TR output rows" in src and "fop::vstore<fop::F16, 8, 16" in src
+    op2 = FusedOp(W.nhwc_to_nchw(256, 7, 7, 2048), jit=0, autotune=0)
+    assert "flat tile of TR output rows" in op2.source()

@@ -204,12 +204,14 @@ def test_transpose_roundtrip_on_gpu():
     assert_bitexact(back["out"], x["x"], "roundtrip")
 
 
-@pytest.mark.parametrize("dims,cls", [((2, 56, 56, 256), "transpose"), ((3, 7, 9, 64), "ew"),
-                                      ((1, 14, 14, 40), "transpose"), ((2, 5, 8, 24), "transpose")])
+@pytest.mark.parametrize("dims,cls", [((2, 56, 56, 256), "transpose"), ((3, 7, 9, 64), "transpose"),
+                                      ((1, 14, 14, 40), "transpose"), ((2, 5, 8, 24), "transpose"),
+                                      ((2, 7, 7, 2048), "transpose")])
 def test_nhwc_to_nchw_bitexact(dims, cls):
     """The reverse layout change: d_v absorbs h after w (one contiguous run of
     H*W on both sides), so the store tiles span whole NCHW planes.  An odd
-    H*W (63) cannot carry store vectors: elementwise with gathers."""
+    H*W (63, 49) cannot carry store vectors: flat output tiles through shared
+    memory."""
     d = W.nhwc_to_nchw(*dims, s=0.5)
     x = W.make_inputs(d)
     got, op = run_gpu(d, x)
@@ -227,6 +229,30 @@ def test_transpose_odd_planes_via_shared_memory(dims, dtype):
     got, op = run_gpu(d, x)
     assert op.selected(0)[0].startswith("fop_transpose_smem")
     assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+
+
+@pytest.mark.parametrize("dims,dtype", [((2, 3, 16, 24), "f16"), ((2, 3, 8, 8), "f32"), ((2, 5, 8, 16), "bf16"),
+                                        ((1, 3, 224, 224), "f16")])
+def test_transpose_tiny_channels_via_shared_memory(dims, dtype):
+    """NCHW -> NHWC of an input layer (C = 3): no store vector along c, so the
+    output tile (whole NHWC rows of 3 channels) is written flat from shared
+    memory; bit-exact."""
+    d = W.cfg3(*dims, dtype=dtype)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.selected(0)[0].startswith("fop_transpose_smem")
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+
+
+@pytest.mark.parametrize("mirror", [False, True])
+def test_transpose_smem_pure_move_keeps_nan_payloads_both_ways(mirror):
+    d = W.nhwc_to_nchw(2, 7, 7, 64, s=1.0) if mirror else W.cfg3(2, 64, 7, 7, s=1.0)
+    d["stmts"][0]["expr"] = [("load", 0)]
+    d["tensors"]["x"]["init"] = ("special", 4)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.selected(0)[0].startswith("fop_transpose_smem")
+    assert np.array_equal(got["out"].view(np.uint16), O.run(d, x)["out"].view(np.uint16))
 
 
 def test_transpose_smem_pure_move_keeps_nan_payloads():

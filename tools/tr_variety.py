@@ -31,6 +31,7 @@ CASES = [
     ("NCHW->NHWC f16 C=3 [256,3,224,224]", lambda: W.cfg3(256, 3, 224, 224)),
     ("NCHW->NHWC f16 C=2048 [256,2048,7,7]", lambda: W.cfg3(256, 2048, 7, 7)),
     ("NHWC->NCHW f16 [256,56,56,256]", lambda: W.nhwc_to_nchw(256, 56, 56, 256)),
+    ("NHWC->NCHW f16 7x7 [256,7,7,2048]", lambda: W.nhwc_to_nchw(256, 7, 7, 2048)),
     ("2-D f32 [16384,16384]", lambda: W.transpose2d(16384, 16384, "f32")),
     ("2-D f16 [8192,24576]", lambda: W.transpose2d(8192, 24576, "f16")),
 ]
