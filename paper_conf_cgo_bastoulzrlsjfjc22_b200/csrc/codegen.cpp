@@ -922,9 +922,27 @@ struct Gen {
     o.l("idx_t t = g;");
     o.l("const idx_t tv_lo = t % " + num(L.gv) + "u; t /= " + num(L.gv) + "u;");
     o.l("const idx_t tr_lo = t % " + num(L.gr) + "u; t /= " + num(L.gr) + "u;");
-    o.l("const idx_t tv_hi = t % " + num(TVH) + "u; t /= " + num(TVH) + "u;");
-    if (L.kl.size() > 2) o.l("const idx_t tr_hi = t % " + num(TRH) + "u; t /= " + num(TRH) + "u;");
-    else o.l("const idx_t tr_hi = t;");
+    // traversal of the (tv_hi, tr_hi) tile grid by consecutive warps:
+    // 0 = d_v tiles fastest (the resident warps cover a strip along d_v),
+    // 1 = d_r tiles fastest, 2 = blocks of BV d_v tiles x all d_r tiles
+    const int tro = geometry_knob(L, "FOP_TR_ORDER", 0);
+    const int64_t BV = std::max(1, geometry_knob(L, "FOP_TR_BV", 8));
+    if (tro == 1) {
+      o.l("const idx_t tr_hi = t % " + num(TRH) + "u; t /= " + num(TRH) + "u;");
+      if (L.kl.size() > 2) o.l("const idx_t tv_hi = t % " + num(TVH) + "u; t /= " + num(TVH) + "u;");
+      else o.l("const idx_t tv_hi = t;");
+    } else if (tro == 2) {
+      const int64_t TVB = (TVH + BV - 1) / BV;
+      o.l("const idx_t tv_m = t % " + num(BV) + "u; t /= " + num(BV) + "u;");
+      o.l("const idx_t tr_hi = t % " + num(TRH) + "u; t /= " + num(TRH) + "u;");
+      if (L.kl.size() > 2) o.l("const idx_t tv_b = t % " + num(TVB) + "u; t /= " + num(TVB) + "u;");
+      else o.l("const idx_t tv_b = t;");
+      o.l("const idx_t tv_hi = tv_b * " + num(BV) + "u + tv_m;");
+    } else {
+      o.l("const idx_t tv_hi = t % " + num(TVH) + "u; t /= " + num(TVH) + "u;");
+      if (L.kl.size() > 2) o.l("const idx_t tr_hi = t % " + num(TRH) + "u; t /= " + num(TRH) + "u;");
+      else o.l("const idx_t tr_hi = t;");
+    }
     o.l("const idx_t tv = tv_hi * " + num(L.gv) + "u + tv_lo;");
     o.l("if (tv >= " + num(NTV) + "u) continue;");
     o.l("const idx_t iv = tv * " + num(W) + "u;");

@@ -464,6 +464,10 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     // of consecutive tiles complete the same 128 B lines back to back
     L.unroll = std::max(1, knob("FOP_TR_U", 2));
     trh = (ntr + (int64_t)L.gr * L.unroll - 1) / ((int64_t)L.gr * L.unroll);
+    if (knob("FOP_TR_ORDER", 0) == 2) {   // blocked traversal (codegen gen_transpose): whole blocks of BV
+      const int64_t BV = std::max(1, knob("FOP_TR_BV", 8));
+      tvh = (tvh + BV - 1) / BV * BV;
+    }
     L.work = (int64_t)gv * L.gr * tvh * trh * prod_rest;
     L.minblocks = knob("FOP_TR_MINB", L.unroll >= 2 ? 1 : 2);
     int64_t need = (L.work + L.block - 1) / L.block;
