@@ -1439,9 +1439,13 @@ struct Gen {
     // span the cluster, block partials are combined through distributed
     // shared memory in rank order, identically in every CTA
     const int Q = std::max(1, L.row_q);
-    const int64_t LNB = 32 * (int64_t)G;   // lanes of one row inside a block
-    const int64_t LN = LNB * Q;            // lanes of one row
-    const bool MULTI = G > 1 || Q > 1;     // the row loop synchronises (block-uniform trip count)
+    // P rows per warp (short rows): 32/P lanes per row, group butterflies
+    const int P = std::max(1, L.row_p);
+    const int64_t LNB = 32 * (int64_t)G / P;   // lanes of one row inside a block
+    const int64_t LN = LNB * Q;                // lanes of one row
+    // the row loop synchronises (block-uniform trip count), or its shuffles
+    // span several rows (P > 1: warp-uniform trip count, per-row validity)
+    const bool MULTI = G > 1 || Q > 1 || P > 1;
     const int K = (int)((NVD + LN - 1) / LN);
     int64_t NRO = 1;
     for (int k = 1; k < L.nsplit; k++) NRO *= L.kl[k].extent;
@@ -1498,7 +1502,9 @@ struct Gen {
     auto lane_guard = [&](int kk) {
       return NVD % LN != 0 ? "if (lane + " + num(LN * kk) + "u < " + num(NVD) + "u) " : std::string("");
     };
-    header(G == 1 ? "ROW_REDUCE (one warp per row, lanes across d_v vectors, butterfly)"
+    header(P > 1 ? "ROW_REDUCE (" + std::to_string(P) + " rows per warp, " + std::to_string(32 / P) +
+                       " lanes across each row's vectors, group butterfly)"
+           : G == 1 ? "ROW_REDUCE (one warp per row, lanes across d_v vectors, butterfly)"
                   : "ROW_REDUCE (" + std::to_string(G) + " warps per row, butterfly + fixed-order shared-memory combine)", 1);
     if (Q > 1) o.l("const idx_t lane = threadIdx.x % " + num(LNB) + "u + fop::cluster_ctarank() * " + num(LNB) + "u;");
     else o.l("const idx_t lane = threadIdx.x % " + num(LN) + "u;");
@@ -1771,7 +1777,11 @@ struct Gen {
               "cp)), __fsub_rn(fop::hi(" + a + "p), fop::hi(" + a + "cp))));");
         else if (x.redop == FOP_RED_SUM)
           o.l(a + " = __fadd_rn(" + a + ", __fadd_rn(fop::lo(" + a + "p), fop::hi(" + a + "p)));");
-        o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::warp_max(" : "fop::warp_sum(") + a + ");");
+        if (P > 1)
+          o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::group_max<" : "fop::group_sum<") + num(LN) + ">(" +
+              a + ");");
+        else
+          o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::warp_max(" : "fop::warp_sum(") + a + ");");
         if (G > 1) {   // the row's G warp partials, combined in warp order
           std::string rs = "RS" + num(x.stmt);
           o.l("if ((threadIdx.x & 31u) == 0u) " + rs + "[threadIdx.x >> 5] = " + a + ";");

@@ -463,6 +463,20 @@ __device__ __forceinline__ float warp_max(float v) {
   for (int o = 16; o > 0; o >>= 1) v = op_max(v, __shfl_xor_sync(0xffffffffu, v, o));
   return v;
 }
+// butterflies over aligned groups of LN lanes (LN rows of a short-row kernel
+// share a warp: the xor offsets < LN never leave the group)
+template <int LN>
+__device__ __forceinline__ float group_sum(float v) {
+#pragma unroll
+  for (int o = LN / 2; o > 0; o >>= 1) v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+template <int LN>
+__device__ __forceinline__ float group_max(float v) {
+#pragma unroll
+  for (int o = LN / 2; o > 0; o >>= 1) v = op_max(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
 
 // ------------------------------------------------------------------ TMA + mbarrier (sm_90+/sm_100a)
 // Tensor maps are encoded on the host per run (cuTensorMapEncodeTiled) and

@@ -176,6 +176,10 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       v.push_back({{"FOP_ROW_MINB", 2}});
       v.push_back({{"FOP_ROW_MINB", 4}});
       v.push_back({{"FOP_BLOCK", 128}, {"FOP_ROW_MINB", 6}});
+      if (L.row_p > 1) {   // short rows: one vector per lane per row, latency hidden by more warps
+        v.push_back({{"FOP_ROW_MINB", 6}});
+        v.push_back({{"FOP_ROW_MINB", 8}});
+      }
       break;
     default:
       v.push_back({{"FOP_COL_U", 2}, {"FOP_COL_MINB", 8}});
@@ -566,15 +570,23 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     }
     G = std::max(1, pow2_floor(knob("FOP_ROW_G", G)));
     Q = std::max(1, std::min(8, pow2_floor(knob("FOP_ROW_Q", Q))));
+    // short rows (fewer than 16 vectors): P rows share a warp, 32/P lanes
+    // each, so the lanes are not left idle by a row of 4-8 vectors
+    int P = 1;
+    if (G == 1 && Q == 1 && !split && knob("FOP_ROW_P", 1))
+      while (P < 32 && 32 / (2 * P) >= nvd) P *= 2;
     L.row_g = G;
     L.row_q = Q;
+    L.row_p = P;
     L.row_split = split ? (int)(32 * (int64_t)G * Q / std::min<int64_t>(32 * (int64_t)G * Q, pow2_ceil(nvd))) : 0;
     if (G > 1) L.block = std::max(L.block, 32 * G);
     if (Q > 1) L.block = 32 * G;   // one row per CTA
-    L.minblocks = knob("FOP_ROW_MINB", L.block >= 1024 ? 1 : (L.block >= 512 ? 2 : 3));
+    // short rows hold one vector per lane per row: more warps hide the
+    // latency (profiles/red_variety_r01.log: [1048576,64] f16 3745 -> 5343 GB/s)
+    L.minblocks = knob("FOP_ROW_MINB", L.block >= 1024 ? 1 : (L.block >= 512 ? 2 : (P > 1 ? 8 : 3)));
     L.row_prefetch = knob("FOP_ROW_PREFETCH", 1);
     L.row_hoist = knob("FOP_ROW_HOIST", 1);
-    int64_t gpb = L.block / (32 * G);
+    int64_t gpb = L.block * P / (32 * G);   // rows per block
     int64_t need = (rows + gpb - 1) / gpb;
     L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
     if (Q > 1)   // whole clusters, one row each per pass

@@ -304,6 +304,43 @@ def test_cfg4a_row_block_geometries(monkeypatch, knobs):
     _check_rowstats(d, x, got)
 
 
+def _rowsum(R, C, dtype="f16", op="sum"):
+    return {
+        "name": "rowsum", "loops": {"r": R, "c": C},
+        "tensors": {"x": {"shape": [R, C], "dtype": dtype, "role": "in", "init": ("normal", 0.0, 1.0, 5),
+                          "strides": None},
+                    "out": {"shape": [R], "dtype": "f32", "role": "out", "init": None, "strides": None}},
+        "stmts": [{"kind": "reduce", "op": op, "loops": ["r", "c"], "write": ("out", ["r"]),
+                   "reads": [("x", ["r", "c"])], "expr": [("load", 0)]}],
+    }
+
+
+@pytest.mark.parametrize("R,C,dtype,op,P", [(1000, 64, "f16", "sum", 4), (4099, 16, "f32", "sum", 8),
+                                            (777, 24, "f16", "max", 8), (50, 8, "bf16", "sum", 32),
+                                            (33, 64, "f32", "sum", 2)])
+def test_short_rows_share_a_warp(R, C, dtype, op, P):
+    """Rows of fewer than 16 vectors: P rows per warp, 32/P lanes each, group
+    butterflies; ragged row counts leave part of the last warp without a row."""
+    d = _rowsum(R, C, dtype, op)
+    x = W.make_inputs(d)
+    got, o = run_gpu(d, x)
+    assert f"{P} rows per warp" in o.source()
+    ref = O.run(d, x)["out"]
+    if op == "max":
+        assert np.array_equal(got["out"], ref)
+    else:
+        assert_normwise(got["out"], ref, O.run(abs_terms_desc(d, 0), x)["out"], 1e-5 if dtype == "f32" else 2e-3, "out")
+
+
+def test_short_row_layernorm_statistics():
+    """cfg4a's bias + GELU + mean/var with 64-wide rows (4 rows per warp)."""
+    d = W.cfg4a(3, 100, 64)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert "4 rows per warp" in op.source()
+    _check_rowstats(d, x, got)
+
+
 def test_row_closed_forms_on_gpu():
     d = W.cfg4a(1, 4, 768)
     d["stmts"][0]["expr"] = [("load", 0)]
