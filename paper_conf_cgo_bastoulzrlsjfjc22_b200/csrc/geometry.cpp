@@ -171,6 +171,10 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       if (L.row_g > 1) {   // few long rows: neighbouring warps-per-row counts
         v.push_back({{"FOP_ROW_G", L.row_g / 2}});
         if (L.row_g < 32) v.push_back({{"FOP_ROW_G", L.row_g * 2}});
+        if (L.row_q > 1) {   // rows spread over clusters: more CTAs per row / more warps per SM
+          v.push_back({{"FOP_ROW_Q", 8}, {"FOP_ROW_G", 16}});
+          v.push_back({{"FOP_ROW_Q", 8}, {"FOP_ROW_MINB", 4}});
+        }
         break;
       }
       v.push_back({{"FOP_ROW_MINB", 2}});

@@ -48,6 +48,8 @@ CASES = [
     ("rowsum f32 [4194304,16]", lambda: rowsum(4194304, 16, "f32")),
     ("rowsum f16 [64,1048576]", lambda: rowsum(64, 1048576)),
     ("rowsum f32 [8192,4096]", lambda: rowsum(8192, 4096, "f32")),
+    ("rowsum f16 [100,524288]", lambda: rowsum(100, 524288)),
+    ("rowsum f32 [32,1048576]", lambda: rowsum(32, 1048576, "f32")),
 ]
 
 
