@@ -121,6 +121,12 @@ std::string node_name(const XStmt& x, const std::vector<bool>& var, int i, const
 // cone by that expression (e.g. a shared-memory table lookup)
 thread_local const std::vector<std::string>* g_over = nullptr;
 bool overridden(int i) { return g_over && i < (int)g_over->size() && !(*g_over)[i].empty(); }
+// an override of a varying node names its element as $E
+std::string over_at(int i, const std::string& e) {
+  std::string s = (*g_over)[i];
+  for (size_t q = s.find("$E"); q != std::string::npos; q = s.find("$E", q + e.size())) s.replace(q, 2, "(" + e + ")");
+  return s;
+}
 
 // reachable set from the result (not descending into overridden nodes)
 std::vector<bool> reachable(const XStmt& x) {
@@ -143,7 +149,7 @@ void emit_nodes(Out& o, const XStmt& x, const std::vector<bool>& var, bool want,
     if (!reach[i] || var[i] != want || (int)i == skip) continue;
     const XNode& n = x.nodes[i];
     std::string e;
-    if (overridden((int)i)) e = (*g_over)[i];
+    if (overridden((int)i)) e = over_at((int)i, c.ev);
     else if (n.op == FOP_OP_LOAD) e = c.load(n.acc, c.ev);
     else if (n.op == X_FWD) e = c.fwd(n.src, c.ev);
     else if (n.op == X_SELF) e = c.self(c.ev);
@@ -174,6 +180,10 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
     if (!reach[i] || !var[i] || (int)i == skip) continue;
     const XNode& n = x.nodes[i];
     std::string e;
+    if (overridden((int)i)) {   // a per-element table lookup
+      o.l("const u64 " + pair_name(x, (int)i, c) + " = fop::pk(" + over_at((int)i, e0) + ", " + over_at((int)i, e1) + ");");
+      continue;
+    }
     switch (n.op) {
       case FOP_OP_LOAD: e = "fop::pk(" + c.load(n.acc, e0) + ", " + c.load(n.acc, e1) + ")"; break;
       case X_FWD: e = "fop::pk(" + c.fwd(n.src, e0) + ", " + c.fwd(n.src, e1) + ")"; break;
@@ -392,10 +402,18 @@ struct Gen {
         bool frontier = false;   // an invariant operand of a varying node
         for (size_t j = i + 1; j < n; j++)
           if (var[j] && (x.nodes[j].a == (int)i || x.nodes[j].b == (int)i)) frontier = true;
-        if (var[i] || !costly[i] || !frontier || __builtin_popcount(dep[i]) != 1) continue;
+        // a cone over the vector loop alone (NHWC BatchNorm: scale[c] with c
+        // = d_v) whose consumers mix in other loops: tabulated too, looked up
+        // per element (tbl[iv + e]); needs whole vectors (no ragged tail)
+        bool frontier0 = false;
+        for (size_t j = i + 1; j < n; j++)
+          if ((x.nodes[j].a == (int)i || x.nodes[j].b == (int)i) && (dep[j] & ~1u)) frontier0 = true;
+        const bool vec_table = dep[i] == 1u && costly[i] && frontier0 && L.kl.size() > 1 &&
+                               L.kl[0].extent % L.width == 0 && geometry_knob(L, "FOP_SMEM_TABLES_V", 1);
+        if (!vec_table && (var[i] || !costly[i] || !frontier || __builtin_popcount(dep[i]) != 1)) continue;
         int k = __builtin_ctz(dep[i]);
         int64_t E = L.kl[k].extent;
-        if (k == 0 || E > 8192 || bytes + E * 4 > 32 * 1024) continue;
+        if ((k == 0 && !vec_table) || E > 8192 || bytes + E * 4 > 32 * 1024) continue;
         bytes += E * 4;
         Table t{(int)si, (int)i, k, E, "tbl" + num(x.stmt) + "_" + num(i)};
         tables.push_back(t);
@@ -408,7 +426,7 @@ struct Gen {
     if (tables.empty()) return;
     for (const Table& t : tables) {
       const XStmt& x = L.stmts[t.si];
-      o.l("__shared__ float " + t.name + "[" + num(t.E) + "];");
+      o.l("__shared__ __align__(16) float " + t.name + "[" + num(t.E) + "];");
       o.l("for (unsigned ti = threadIdx.x; ti < " + num(t.E) + "u; ti += " + num(L.block) + "u) {");
       o.ind++;
       // the cone of the table node, with its single loop bound to ti
@@ -596,7 +614,21 @@ struct Gen {
           if (tb.si == (int)si)
             for (auto& kv : its[u])
               if (kv.first == tb.k)   // slots past the end (ok false) still evaluate: keep the index in the table
-                ov[tb.node] = tb.name + "[ok" + t + " ? " + kv.second + " : 0u]";
+                if (tb.k == 0) {   // per element: the vector's W entries, read with 16 B shared loads
+                  const std::string tv = "TV" + tb.name.substr(3) + t;
+                  o.l("float " + tv + "[" + num(L.width) + "];");
+                  o.l("#pragma unroll");
+                  if (L.width % 4 == 0)
+                    o.l("for (int q_ = 0; q_ < " + num(L.width / 4) + "; ++q_) reinterpret_cast<float4*>(" + tv +
+                        ")[q_] = reinterpret_cast<const float4*>(&" + tb.name + "[ok" + t + " ? " + kv.second +
+                        " : 0u])[q_];");
+                  else
+                    o.l("for (int q_ = 0; q_ < " + num(L.width) + "; ++q_) " + tv + "[q_] = " + tb.name + "[(ok" + t +
+                        " ? " + kv.second + " : 0u) + q_];");
+                  ov[tb.node] = tv + "[$E]";
+                } else {
+                  ov[tb.node] = tb.name + "[ok" + t + " ? " + kv.second + " : 0u]";
+                }
         g_over = &ov;
         auto var = varies(x, c);
         emit_nodes(o, x, var, false, c);

@@ -66,6 +66,17 @@ def test_cfg2_bn_relu_cast_bitexact(dims):
     assert_bitexact(got["y"], ref["y"], "y")
 
 
+@pytest.mark.parametrize("dims", [(2, 7, 9, 64), (1, 5, 5, 96), (3, 4, 4, 8)])
+def test_cfg2_nhwc_channel_tables_bitexact(dims):
+    """BN on NHWC: scale/shift vary along the vector loop (c), tabulated per CTA
+    in shared memory and read per element; identical IEEE ops, same bits."""
+    d = W.cfg2_nhwc(*dims)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert "__shared__ __align__(16) float tbl" in op.source()
+    assert_bitexact(got["y"], O.run(d, x)["y"], "y")
+
+
 def test_cfg2_orders_widths_agree():
     d = W.cfg2(2, 64, 28, 28)
     x = W.make_inputs(d)
