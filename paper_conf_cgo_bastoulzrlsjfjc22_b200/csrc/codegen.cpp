@@ -1466,6 +1466,7 @@ struct Gen {
     // G warps per row (few long rows): LN lanes across the row's vectors, the
     // G warp partials of a reduction combined in a fixed order through shared
     // memory, the row loop uniform across the block (it synchronises)
+    const bool PEEL = L.row_peel != 0;   // per-row shift to the first aligned element (geometry)
     const int G = std::max(1, L.row_g);
     // Q CTAs per row (a thread-block cluster; few long rows): the row's lanes
     // span the cluster, block partials are combined through distributed
@@ -1492,7 +1493,7 @@ struct Gen {
     // forwarded rows live in registers when they fit (<= 64 values per lane);
     // longer rows are re-read by the lane that stored them (same thread, same
     // address: program order makes the store visible; L2 serves the re-read)
-    const bool regmode = NRO * K * W <= 64 && !SPL;
+    const bool regmode = NRO * K * W + (PEEL ? 1 : 0) <= 64 && !SPL;
     for (auto& x : L.stmts)
       if (x.kind == FOP_ASSIGN && x.fwd && !regmode && !x.store)
         fail(FOP_E_UNSUPPORTED, "ROW_REDUCE: a long forwarded row must be stored to be re-read");
@@ -1517,6 +1518,7 @@ struct Gen {
       int64_t cv = C(a, 0);
       int es_k = es(a.tensor);
       if (rt_ro) continue;
+      if (PEEL && cv != 0) continue;   // vector positions move with each row's shift
       if (L.row_hoist && row_inv && regmode && (cv == 0 || cv == 1) && !written_here(a.tensor)) mode[k] = 'H';
       else if (L.row_prefetch && used0[k] && cv == 1 && W * es_k >= 4 && L.load_cb[k] >= 4 &&
                NP * W * es_k / 4 <= 32 && !written_here(a.tensor))
@@ -1620,6 +1622,25 @@ struct Gen {
     o.l("idx_t rr = row;");
     std::vector<std::pair<int, std::string>> rits;
     decompose("rr", L.nsplit, (int)L.kl.size(), "", rits);
+    if (PEEL) {   // this row's shift to its first W-aligned element, full vectors, scalar head + tail
+      // the shift follows the row-variant vectorised accesses (geometry checked
+      // they agree modulo W); row-invariant vectors are read element-wise
+      auto row_variant = [&](const Affine& a) {
+        for (size_t k = 1; k < L.kl.size(); k++)
+          if (C(a, (int)k) != 0) return true;
+        return false;
+      };
+      const Affine* ref = nullptr;
+      for (auto& a : L.loads)
+        if (!ref && C(a, 0) == 1 && row_variant(a)) ref = &a;
+      for (auto& x : L.stmts)
+        if (!ref && C(x.write, 0) == 1 && row_variant(x.write)) ref = &x.write;
+      const int64_t EVr = L.kl[0].extent;
+      o.l("const unsigned pe_s = (" + num(W) + "u - (unsigned)(" + affine(*ref, rits) + " % " + num(W) + "u)) % " +
+          num(W) + "u;");
+      o.l("const unsigned pe_n = (" + num(EVr) + "u - pe_s) / " + num(W) + "u;");
+      o.l("const unsigned pe_t = " + num(EVr) + "u - pe_n * " + num(W) + "u;");
+    }
     auto load_varies_e = [&](int k) { return C(L.loads[k], 0) != 0; };
     for (size_t si = 0; si < L.stmts.size(); si++) {
       const XStmt& x = L.stmts[si];
@@ -1636,7 +1657,8 @@ struct Gen {
         if (x.redop == FOP_RED_SUM) o.l("u64 acc" + num(x.stmt) + "p = fop::pk1(0.f);");
         if (kahan) o.l("float acc" + num(x.stmt) + "c = 0.f; u64 acc" + num(x.stmt) + "cp = fop::pk1(0.f);");
       }
-      if (x.kind == FOP_ASSIGN && x.fwd && regmode) o.l("float F" + num(x.stmt) + "[" + num(NRO * K * W) + "];");
+      if (x.kind == FOP_ASSIGN && x.fwd && regmode)
+        o.l("float F" + num(x.stmt) + "[" + num(NRO * K * W + (PEEL ? 1 : 0)) + "];");
       for (int64_t ro = 0; ro < NRO_E; ro++) {
         // decomposition of ro over the outer reduction kloops (compile time;
         // at run time, inside the kk block, for the runtime loop)
@@ -1648,7 +1670,10 @@ struct Gen {
             rem /= L.kl[k].extent;
           }
         }
-        for (int kk = 0; kk < K; kk++) {
+        for (int kk = 0; kk < K + (PEEL ? 1 : 0); kk++) {
+          // PEEL: kk == K is the row's head + tail elements, one per lane, scalar
+          const bool scal = PEEL && kk == K;
+          const int Wb = scal ? 1 : W;
           std::string t = "_" + num(si) + "_" + num(ro) + "_" + num(kk);
           o.l("{");
           o.ind++;
@@ -1656,9 +1681,17 @@ struct Gen {
             o.l("[[maybe_unused]] const idx_t iv = vl_ * " + num(W) + "u;");
             o.l(std::string("if (") + (MULTI ? "rv && " : "") + "vl_ < " + num(NVD) + "u) {");
           } else {
-            o.l("[[maybe_unused]] const idx_t iv = (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
-            if (jguard)
-              o.l(std::string("if (") + (MULTI ? "rv && " : "") + "lane + " + num(LN * kk) + "u < " + num(NVD) + "u) {");
+            if (scal) {
+              o.l("[[maybe_unused]] const idx_t iv = lane < pe_s ? lane : pe_n * " + num(W) + "u + lane;");
+              o.l(std::string("if (") + (MULTI ? "rv && " : "") + "lane < pe_t) {");
+            } else if (PEEL) {
+              o.l("[[maybe_unused]] const idx_t iv = pe_s + (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
+              o.l(std::string("if (") + (MULTI ? "rv && " : "") + "lane + " + num(LN * kk) + "u < pe_n) {");
+            } else {
+              o.l("[[maybe_unused]] const idx_t iv = (lane + " + num(LN * kk) + "u) * " + num(W) + "u;");
+              if (jguard)
+                o.l(std::string("if (") + (MULTI ? "rv && " : "") + "lane + " + num(LN * kk) + "u < " + num(NVD) + "u) {");
+            }
           }
           auto its2 = its;
           if (rt_ro) {
@@ -1696,12 +1729,12 @@ struct Gen {
             } else if (cv == 0) {
               o.l("const float " + nm + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
             } else if (cv == 1) {
-              o.l("float " + nm + "[" + num(W) + "];");
-              o.l("fop::vload<" + dt + ", " + num(W) + ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + nm +
-                  ", " + ptr(a.tensor, off) + ");");
+              o.l("float " + nm + "[" + num(Wb) + "];");
+              o.l("fop::vload<" + dt + ", " + num(Wb) + ", " + num(scal ? es(a.tensor) : L.load_cb[k]) + ", " +
+                  pol(a, false) + ">(" + nm + ", " + ptr(a.tensor, off) + ");");
             } else {
-              o.l("float " + nm + "[" + num(W) + "];");
-              o.l("for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = fop::sload<" + dt + ", " +
+              o.l("float " + nm + "[" + num(Wb) + "];");
+              o.l("for (int e = 0; e < " + num(Wb) + "; ++e) " + nm + "[e] = fop::sload<" + dt + ", " +
                   pol(a, false) + ">(" + ptr(a.tensor, off + " + e * " + num(cv)) + ");");
             }
           }
@@ -1716,12 +1749,12 @@ struct Gen {
               int64_t cw = C(pr.write, 0);
               std::string nm = "FW" + num(pr.stmt);
               std::string dt = dtn(pr.out_dtype);
-              o.l("float " + nm + "[" + num(W) + "];");
+              o.l("float " + nm + "[" + num(Wb) + "];");
               if (cw == 1)
-                o.l("fop::vload<" + dt + ", " + num(W) + ", " + num(L.store_cb[s2]) + ", fop::LD_COHERENT>(" + nm +
-                    ", " + ptr(pr.write.tensor, off) + ");");
+                o.l("fop::vload<" + dt + ", " + num(Wb) + ", " + num(scal ? esize(pr.out_dtype) : L.store_cb[s2]) +
+                    ", fop::LD_COHERENT>(" + nm + ", " + ptr(pr.write.tensor, off) + ");");
               else
-                o.l("for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = fop::sload<" + dt +
+                o.l("for (int e = 0; e < " + num(Wb) + "; ++e) " + nm + "[e] = fop::sload<" + dt +
                     ", fop::LD_COHERENT>(" + ptr(pr.write.tensor, off + " + e * " + num(cw)) + ");");
             }
           }
@@ -1731,7 +1764,7 @@ struct Gen {
           c.load = [&](int k, const std::string& e) {
             return C(L.loads[k], 0) != 0 ? "L" + num(k) + "[" + e + "]" : "L" + num(k);
           };
-          int64_t base_idx = (ro * K + kk) * W;
+          int64_t base_idx = (ro * K + kk) * W;   // scal: K * W, the slot after the row's vectors
           c.fwd = [&, base_idx](int s, const std::string& e) {
             return regmode ? "F" + num(L.stmts[s].stmt) + "[" + num(base_idx) + " + " + e + "]"
                            : "FW" + num(L.stmts[s].stmt) + "[" + e + "]";
@@ -1739,7 +1772,7 @@ struct Gen {
           c.scalar = [&](int s) { return "S" + num(L.stmts[s].stmt); };
           auto var = varies(x, c);
           emit_nodes(o, x, var, false, c);
-          if (!red) o.l("float R[" + num(W) + "];");
+          if (!red) o.l("float R[" + num(Wb) + "];");
           std::string A = "acc" + num(x.stmt);
           Sink sk;
           if (red) {
@@ -1781,23 +1814,23 @@ struct Gen {
                     "2 * " + p + " + 1]);");
             };
           }
-          emit_elems(o, x, var, c, W, sk);
+          emit_elems(o, x, var, c, Wb, sk);
           if (!red && x.store) {
             std::string off = affine(x.write, its2);
             int64_t cw = C(x.write, 0);
             std::string dt = dtn(x.out_dtype);
             if (cw == 1)
-              o.l("fop::vstore<" + dt + ", " + num(W) + ", " + num(L.store_cb[si]) + ", " + spol() + ">(" +
-                  ptr(x.write.tensor, off) + ", R);");
+              o.l("fop::vstore<" + dt + ", " + num(Wb) + ", " + num(scal ? esize(x.out_dtype) : L.store_cb[si]) + ", " +
+                  spol() + ">(" + ptr(x.write.tensor, off) + ", R);");
             else
-              o.l("for (int e = 0; e < " + num(W) + "; ++e) fop::sstore<" + dt + ">(" +
+              o.l("for (int e = 0; e < " + num(Wb) + "; ++e) fop::sstore<" + dt + ">(" +
                   ptr(x.write.tensor, off + " + e * " + num(cw)) + ", R[e]);");
           }
           if (rt_ro) {
             o.ind--;
             o.l("}");
           }
-          if (jguard) o.l("}");
+          if (jguard || PEEL) o.l("}");
           o.ind--;
           o.l("}");
         }

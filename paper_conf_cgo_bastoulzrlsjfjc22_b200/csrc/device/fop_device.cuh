@@ -316,8 +316,21 @@ __device__ __forceinline__ float op_relu(float a) { return a > 0.f ? a : 0.f; }
 // max/min: NaN operands ignored, max(-0,+0) = +0, min(-0,+0) = -0 (reading
 // R24).  B200's FMNMX implements exactly this (tools/probes/maxmin_probe.cu,
 // measured), so fmaxf/fminf are single instructions with the oracle's bits.
-__device__ __forceinline__ float op_max(float a, float b) { return fmaxf(a, b); }
-__device__ __forceinline__ float op_min(float a, float b) { return fminf(a, b); }
+// Written as PTX min/max (the same FMNMX fminf/fmaxf compile to): CUDA 12.9's
+// NVVM optimizer crashes the compiling process (SIGILL inside cicc/NVRTC) on
+// min(min(a, b), a + b) and max(max(a, b), a * b) built from the intrinsics
+// (fuzz seed 15 case 161; tools/probes/cicc_minmax.cu); inline PTX is opaque
+// to that rewrite.
+__device__ __forceinline__ float op_max(float a, float b) {
+  float r;
+  asm("max.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+  return r;
+}
+__device__ __forceinline__ float op_min(float a, float b) {
+  float r;
+  asm("min.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+  return r;
+}
 // .ftz forms: MUFU.EX2/RCP without the subnormal pre/post scaling.  In GELU
 // the flushed cases are e < 2^-126 (1 + e == 1 either way) and results below
 // 2^-126 (below fp16/bf16 resolution by 2^-100).

@@ -145,6 +145,8 @@ struct Launch {
   int row_g = 1;                  // ROW: warps per row (> 1 for few long rows)
   int row_q = 1;                  // ROW: CTAs per row (a thread-block cluster) for few long rows
   int row_p = 1;                  // ROW: rows per warp (> 1 for rows of fewer than 16 vectors)
+  int row_peel = 0;               // ROW: rows whose length/pitch admit no static vector: per-row shift to the
+                                  // first aligned element, W-vectors in between, head + tail elements scalar
   int row_split = 0;              // ROW: > 0 = lanes also split the outer reduction iterations (S lane
                                   // subgroups of pow2(#vectors) lanes each), for rows of few vectors
                                   // under long outer reduction loops (e.g. BN statistics on NCHW)

@@ -293,9 +293,34 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   }
   int64_t EV = L.kl[0].extent;
   bool tail_ok = L.kclass == FOP_CLASS_EW && L.kl.size() == 1;
+  // ROW over rows of odd length / odd pitch (GPT-2's 50257-entry vocabulary,
+  // LayerNorm over 1023): keep the full vector width and peel per row — the
+  // kernel shifts each row to its first W-aligned element (the same shift for
+  // every vectorised access: their offsets agree modulo W), runs W-vectors in
+  // between and takes the <= 2(W-1) head/tail elements as scalars
+  L.row_peel = 0;
+  if (L.kclass == FOP_CLASS_ROW_REDUCE && W > 1 && EV % W != 0 && EV >= 4 * W && L.nsplit == 1 &&
+      L.seq.empty() && geometry_knob(L, "FOP_ROW_PEEL", 1)) {
+    const Affine* ref = nullptr;
+    bool ok = true;
+    auto row_invariant = [&](const Affine* a) {
+      for (size_t k = 1; k < L.kl.size(); k++)
+        if (coef(L, *a, (int)k) != 0) return false;
+      return true;
+    };
+    for (const Affine* a : acc) {
+      // row-invariant vectors (LayerNorm's gamma/beta) keep their own
+      // positions: loaded element-wise (cached), not part of the congruence
+      if (coef(L, *a, 0) != 1 || row_invariant(a)) continue;
+      if (!ref) ref = a;
+      ok &= ((a->base - ref->base) % W + W) % W == 0;
+      for (size_t k = 1; k < L.kl.size(); k++) ok &= ((coef(L, *a, (int)k) - coef(L, *ref, (int)k)) % W + W) % W == 0;
+    }
+    if (ok && ref) L.row_peel = 1;
+  }
   if (tail_ok) {
     if (EV < W) W = pow2_floor(EV);
-  } else {
+  } else if (!L.row_peel) {
     while (W > 1 && EV % W) W /= 2;
   }
   L.width = W;
@@ -351,6 +376,8 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
         for (size_t q = 0; q < L.kl.size(); q++) ok &= coef(L, L.loads[k], (int)q) == 0;   // constants only
       }
       const int esi = esize(d.t[L.loads[L.trans_load].tensor].dtype);
+      // the input rows are read with whole vectors along d_r: every row start aligned
+      ok &= chunk_bytes(p, L, L.loads[L.trans_load], 1, wr * esi) == wr * esi;
       const int64_t rowb = EVx * std::max(esi, eso);
       int64_t TR = 0;
       const int64_t cap = std::min<int64_t>(ER, geometry_knob(L, "FOP_TR_SMEM_BYTES", 32768) / rowb);
@@ -389,6 +416,17 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   L.store_cb.assign(L.stmts.size(), 0);
   for (size_t k = 0; k < L.stmts.size(); k++)
     if (coef(L, L.stmts[k].write, 0) == 1) L.store_cb[k] = vec_cb(L.stmts[k].write, 0, W);
+  if (L.row_peel) {   // alignment comes from the per-row shift, not from the static coefficients
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      if (coef(L, L.loads[k], 0) != 1) continue;
+      bool rinv = true;
+      for (size_t q = 1; q < L.kl.size(); q++) rinv &= coef(L, L.loads[k], (int)q) == 0;
+      const int es_k = esize(d.t[L.loads[k].tensor].dtype);
+      L.load_cb[k] = rinv ? es_k : std::min(vmax, W * es_k);   // row-invariant: element-wise
+    }
+    for (size_t k = 0; k < L.stmts.size(); k++)
+      if (coef(L, L.stmts[k].write, 0) == 1) L.store_cb[k] = std::min(vmax, W * esize(L.stmts[k].out_dtype));
+  }
   L.align.assign(d.ntensors, 1);
   for (size_t k = 0; k < L.loads.size(); k++) {
     int t = L.loads[k].tensor;
@@ -577,7 +615,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     // short rows (fewer than 16 vectors): P rows share a warp, 32/P lanes
     // each, so the lanes are not left idle by a row of 4-8 vectors
     int P = 1;
-    if (G == 1 && Q == 1 && !split && knob("FOP_ROW_P", 1))
+    if (G == 1 && Q == 1 && !split && !L.row_peel && knob("FOP_ROW_P", 1))
       while (P < 32 && 32 / (2 * P) >= nvd) P *= 2;
     L.row_g = G;
     L.row_q = Q;

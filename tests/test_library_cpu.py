@@ -280,3 +280,32 @@ def test_tiny_channel_transpose_writes_flat_output_tiles():
     assert "flat tile of TR output rows" in src and "fop::vstore<fop::F16, 8, 16" in src
     op2 = FusedOp(W.nhwc_to_nchw(256, 7, 7, 2048), jit=0, autotune=0)
     assert "flat tile of TR output rows" in op2.source()
+
+
+def test_min_of_min_and_sum_compiles():
+    """CUDA 12.9's NVVM crashed the process (SIGILL inside NVRTC) on
+    min(min(a, b), a + b) written with fminf (fuzz seed 15, case 161); the
+    device header's min/max are inline PTX.  Compiling it must not kill us."""
+    d = {
+        "name": "minmin", "loops": {"l0": 24},
+        "tensors": {"x0": {"shape": [24], "dtype": "bf16", "role": "in", "init": ("normal", 0.0, 1.0, 1), "strides": [1]},
+                    "out": {"shape": [24], "dtype": "bf16", "role": "out", "init": None, "strides": [1]}},
+        "stmts": [{"kind": "assign", "loops": ["l0"], "write": ("out", ["l0"]), "reads": [("x0", ["l0"])],
+                   "expr": [("load", 0), ("relu", 0), ("add", 0, 1), ("min", 0, 1), ("sub", 0, 0), ("min", 3, 2)]}],
+    }
+    for fw in (0, 1):   # the vector kernel and the scalar (narrow) form that crashed
+        FusedOp(d, force_width=fw) if fw else FusedOp(d)
+
+
+def test_mirrored_smem_transpose_needs_aligned_input_rows():
+    """Fuzz seed 18 case 260: x0[3,128,1] read as x0[l3,l2,l0] into out[.,.,128,3]:
+    the input rows along d_r are not 16-byte aligned for every l3, so the
+    flat-output shared-memory path must not be chosen (it compiles either way)."""
+    d = {"name": "tr_small", "loops": {"l0": 1, "l1": 24, "l2": 128, "l3": 3},
+         "tensors": {"x0": {"shape": [3, 128, 1], "dtype": "bf16", "role": "in", "init": ("normal", 0.0, 1.0, 1),
+                            "strides": None},
+                     "out": {"shape": [1, 24, 128, 3], "dtype": "bf16", "role": "out", "init": None, "strides": None}},
+         "stmts": [{"kind": "assign", "loops": ["l0", "l1", "l2", "l3"], "write": ("out", ["l0", "l1", "l2", "l3"]),
+                    "reads": [("x0", ["l3", "l2", "l0"])],
+                    "expr": [("load", 0), ("const", 0.5), ("add", 1, 0), ("div", 2, 2), ("cast", 3, "bf16")]}]}
+    FusedOp(d)

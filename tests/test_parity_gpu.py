@@ -352,6 +352,57 @@ def test_short_row_layernorm_statistics():
     _check_rowstats(d, x, got)
 
 
+@pytest.mark.parametrize("dims", [(2, 64, 771), (1, 9, 1023), (3, 5, 45)])
+def test_cfg4a_odd_rows_peeled(dims):
+    """Rows of odd length: each row shifted to its first 16-byte-aligned
+    element, 8-vectors in between, head and tail elements scalar."""
+    d = W.cfg4a(*dims)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert "pe_s" in op.source()
+    _check_rowstats(d, x, got)
+
+
+@pytest.mark.parametrize("name,kw", [("vocab_softmax", {"R": 5, "V": 50257}), ("bert_layernorm", {"B": 1, "S": 37, "H": 1023}),
+                                     ("vocab_softmax", {"R": 3, "V": 30522})])
+def test_odd_row_softmax_layernorm_peeled(name, kw):
+    from test_n4_ops import _assert_layernorm
+    d = W.N4[name](**kw)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert "pe_s" in op.source()
+    ref = O.run(d, x)
+    for n, v in got.items():
+        if name == "bert_layernorm":
+            _assert_layernorm(d, x, v, ref[n])
+        else:
+            assert_ulp(v, ref[n], 1, n)
+
+
+def test_peeled_rows_shift_follows_the_row_variant_access():
+    """Fuzz seed 17 case 231: a row-invariant vector (bf16 x0[l1]) listed
+    before the padded rows (f16 x1, pitch 102): the per-row shift must come
+    from x1, not from x0 (misaligned vector loads otherwise)."""
+    d = {"name": "peel_ref", "loops": {"l0": 100, "l1": 100},
+         "tensors": {"x0": {"shape": [100], "dtype": "bf16", "role": "in", "init": ("normal", 0.0, 1.0, 1), "strides": [1]},
+                     "x1": {"shape": [100, 100], "dtype": "f16", "role": "in", "init": ("normal", 0.0, 1.0, 2),
+                            "strides": [102, 1]},
+                     "out": {"shape": [100], "dtype": "f32", "role": "out", "init": None, "strides": None}},
+         "stmts": [{"kind": "reduce", "op": "sum", "loops": ["l0", "l1"], "write": ("out", ["l0"]),
+                    "reads": [("x0", ["l1"]), ("x1", ["l0", "l1"])], "expr": [("load", 0), ("load", 1), ("mul", 0, 1)]}]}
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert "pe_s" in op.source()
+    assert_normwise(got["out"], O.run(d, x)["out"], O.run(abs_terms_desc(d, 0), x)["out"], 2e-3, "out")
+
+
+def test_odd_rows_misaligned_pointers_use_narrow_variant():
+    d = W.cfg4a(2, 16, 771)
+    x = W.make_inputs(d)
+    got, _ = run_gpu(d, x, offset=1)
+    _check_rowstats(d, x, got)
+
+
 def test_row_closed_forms_on_gpu():
     d = W.cfg4a(1, 4, 768)
     d["stmts"][0]["expr"] = [("load", 0)]

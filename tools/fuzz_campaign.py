@@ -64,11 +64,14 @@ def main():
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--count", type=int, default=500)
     ap.add_argument("--repeat", action="store_true", help="also re-run each plan (aligned, misaligned, aligned)")
+    ap.add_argument("--trace", action="store_true", help="print each case index before running it (crash triage)")
     a = ap.parse_args()
     rng = np.random.default_rng(a.seed)
     fails, classes = [], {}
     for i in range(a.count):
         d = random_op(rng)
+        if a.trace:
+            print("case", i, d["name"], flush=True)
         try:
             for c in check(d, a.repeat):
                 classes[c] = classes.get(c, 0) + 1

@@ -50,6 +50,10 @@ CASES = [
     ("rowsum f32 [8192,4096]", lambda: rowsum(8192, 4096, "f32")),
     ("rowsum f16 [100,524288]", lambda: rowsum(100, 524288)),
     ("rowsum f32 [32,1048576]", lambda: rowsum(32, 1048576, "f32")),
+    ("vocab softmax f16 [256,32000]", lambda: W.N4["vocab_softmax"](R=256, V=32000)),
+    ("vocab softmax f16 [256,50257] (odd)", lambda: W.N4["vocab_softmax"](R=256, V=50257)),
+    ("layernorm f16 [16384,1023] (odd)", lambda: dict(W.N4["bert_layernorm"](B=32, S=512, H=1023), name="ln_odd")),
+    ("layernorm f16 [16384,1024]", lambda: dict(W.N4["bert_layernorm"](B=32, S=512, H=1024), name="ln")),
 ]
 
 
@@ -85,13 +89,14 @@ def main():
         sets = [{n: to_device(x[n] if t["role"] == "in" else o[n], t["dtype"], "cuda")
                  for n, t in d["tensors"].items() if t["role"] != "temp"} for _ in range(copies)]
         ms = time_op(lambda s: op.run(s), sets)
-        src = [s["x"].view(torch.uint8).reshape(-1) for s in sets]
+        xin = [n for n, t in d["tensors"].items() if t["role"] == "in"][0]
+        src = [s[xin].view(torch.uint8).reshape(-1) for s in sets]
         rms = time_op(lambda k: torch.sum(src[k][: src[k].numel() // 4].view(torch.int32), dtype=torch.int64),
                       list(range(copies)))
         li = op.info()["launches"]
         print(json.dumps({"case": name, "classes": [q["class"] for q in li], "selected": list(op.selected(0)),
                           "us": ms * 1e3, "GB_s": nbytes / ms / 1e6,
-                          "torch_sum_read_GB_s": x["x"].nbytes / rms / 1e6}), flush=True)
+                          "torch_sum_read_GB_s": x[xin].nbytes / rms / 1e6}), flush=True)
         del sets, src
         torch.cuda.empty_cache()
 
