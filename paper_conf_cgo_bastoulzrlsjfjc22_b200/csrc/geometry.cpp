@@ -360,7 +360,11 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
         L.tr_tv = TV;
       }
     }
-    if (W == 1 && wr >= 2 && !L.scalar_variant && geometry_knob(L, "FOP_TR_SMEM", 1)) {
+    // (a long odd d_v, e.g. C = 255, puts the read-out's consecutive lanes 8
+    // tile rows apart, on few shared-memory banks: 1104 GB/s, still above the
+    // gathering elementwise kernel's 958 — profiles/odd_variety_r01.log)
+    if (W == 1 && wr >= 2 && !L.scalar_variant && L.kl[0].extent <= geometry_knob(L, "FOP_TR_SMEM_MAXV", 1 << 30) &&
+        geometry_knob(L, "FOP_TR_SMEM", 1)) {
       // the mirror case: d_v rows too short/odd for store vectors (an input
       // layer's C = 3; NHWC -> NCHW of a 7x7 plane), but the output rows are
       // adjacent (coef_out(d_r) == E[d_v]): a tile of TR whole output rows is
