@@ -54,10 +54,15 @@ struct Out {
 // set per statement (see varies()): the statement's result is rounded to a
 // 16-bit type, so transcendental fast forms are within one ulp
 thread_local bool g_approx16 = false;
+// ... but only for nodes whose value reaches the output without an add or
+// subtract on the way: a ~2^-22 relative error ahead of a cancellation is no
+// longer within one 16-bit ulp (fuzz seed 21 case 294: -x2 / -1.5 + x0 + x1
+// near 6.7e-5 came out 2 f16 ulps off with the x * rcp(c) form)
+bool fast_ok(const XNode& n) { return g_approx16 && n.no_addsub; }
 
 // C expression of a fused-DAG node given its operand expressions
 std::string op_expr(const XNode& n, const std::string& a, const std::string& b) {
-  if (g_approx16) {
+  if (fast_ok(n)) {
     if (n.op == FOP_OP_EXP) return "fop::exp_fast(" + a + ")";
     if (n.op == FOP_OP_SIGMOID) return "fop::sigmoid_fast(" + a + ")";
   }
@@ -101,6 +106,13 @@ std::vector<bool> varies(const XStmt& x, const DagCtx& c) {
   {  // every statement emission starts here: decide the 16-bit fast forms
     const char* e = std::getenv("FOP_APPROX16");
     g_approx16 = !(e && *e == '0') && x.kind == FOP_ASSIGN && esize(x.out_dtype) == 2 && x.out_dtype != FOP_I32;
+    std::vector<bool> feeds(x.nodes.size(), false);   // value reaches an add/sub
+    for (int i = (int)x.nodes.size() - 1; i >= 0; i--)
+      for (size_t j = i + 1; j < x.nodes.size(); j++) {
+        const XNode& q = x.nodes[j];
+        if ((q.a == i || q.b == i) && (q.op == FOP_OP_ADD || q.op == FOP_OP_SUB || feeds[j])) feeds[i] = true;
+      }
+    for (size_t i = 0; i < x.nodes.size(); i++) x.nodes[i].no_addsub = !feeds[i];
   }
   std::vector<bool> v(x.nodes.size(), false);
   for (size_t i = 0; i < x.nodes.size(); i++) {
@@ -193,7 +205,7 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
       case FOP_OP_MUL: e = "fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + ")"; break;
       case FOP_OP_GELU_TANH: e = "fop::op_gelu_tanh2(" + opnd(n.a) + ")"; break;
       case FOP_OP_DIV:
-        if (g_approx16 && !var[n.b]) {  // ÷ loop-invariant -> × correctly rounded reciprocal
+        if (fast_ok(n) && !var[n.b]) {  // ÷ loop-invariant -> × correctly rounded reciprocal
           e = "fop::mul2(" + opnd(n.a) + ", fop::pk1(__frcp_rn(" + node_name(x, var, n.b, c) + ")))";
           break;
         }
@@ -1467,6 +1479,11 @@ struct Gen {
     // G warp partials of a reduction combined in a fixed order through shared
     // memory, the row loop uniform across the block (it synchronises)
     const bool PEEL = L.row_peel != 0;   // per-row shift to the first aligned element (geometry)
+    auto row_variant_acc = [&](const Affine& a) {
+      for (size_t k = 1; k < L.kl.size(); k++)
+        if (C(a, (int)k) != 0) return true;
+      return false;
+    };
     const int G = std::max(1, L.row_g);
     // Q CTAs per row (a thread-block cluster; few long rows): the row's lanes
     // span the cluster, block partials are combined through distributed
@@ -1728,6 +1745,34 @@ struct Gen {
               o.l("fop::cvt_words<" + dt + ", " + num(W) + ">(" + nm + ", &Q" + num(k) + "[" + num(vi * wpv) + "]);");
             } else if (cv == 0) {
               o.l("const float " + nm + " = fop::sload<" + dt + ", " + pol(a, true) + ">(" + ptr(a.tensor, off) + ");");
+            } else if (cv == 1 && PEEL && !scal && !row_variant_acc(a) && L.load_cb[k] >= 4) {
+              // a row-invariant vector under the per-row shift: the two aligned
+              // vectors around the window [iv, iv + W), then the window picked by
+              // a switch on pe_s (uniform across the warp: one row per warp group)
+              const int64_t EVr = L.kl[0].extent;
+              auto its_a = its2;
+              its_a.back().second = "(iv - pe_s)";
+              const std::string pa = ptr(a.tensor, affine(a, its_a));
+              o.l("float " + nm + "[" + num(W) + "];");
+              o.l("{");
+              o.l("  float A_[" + num(2 * W) + "];");
+              o.l("  fop::vload<" + dt + ", " + num(W) + ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(A_, " + pa + ");");
+              o.l("  if (pe_s != 0u) {");
+              o.l("    if (iv - pe_s + " + num(2 * W) + "u <= " + num(EVr) + "u) fop::vload<" + dt + ", " + num(W) + ", " +
+                  num(L.load_cb[k]) + ", " + pol(a, false) + ">(A_ + " + num(W) + ", " + pa + " + " + num(W * es(a.tensor)) + ");");
+              o.l("    else");
+              o.l("      for (int e = 0; e < " + num(W) + "; ++e) A_[" + num(W) + " + e] = iv - pe_s + " + num(W) +
+                  "u + e < " + num(EVr) + "u ? fop::sload<" + dt + ", " + pol(a, false) + ">(" + pa + " + (" +
+                  num(W) + " + e) * " + num(es(a.tensor)) + ") : 0.f;");
+              o.l("  }");
+              o.l("  switch (pe_s) {");
+              for (int sh = 0; sh < W; sh++) {
+                std::string cs = "    case " + num(sh) + "u:";
+                for (int e = 0; e < W; e++) cs += " " + nm + "[" + num(e) + "] = A_[" + num(e + sh) + "];";
+                o.l(cs + " break;");
+              }
+              o.l("  }");
+              o.l("}");
             } else if (cv == 1) {
               o.l("float " + nm + "[" + num(Wb) + "];");
               o.l("fop::vload<" + dt + ", " + num(Wb) + ", " + num(scal ? es(a.tensor) : L.load_cb[k]) + ", " +

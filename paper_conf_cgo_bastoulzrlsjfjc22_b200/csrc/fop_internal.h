@@ -82,6 +82,7 @@ struct XNode {
   float imm = 0.f;
   int acc = -1;     // FOP_OP_LOAD: index into Launch::loads
   int src = -1;     // X_FWD / X_SCALAR: index into Launch::stmts
+  mutable bool no_addsub = false;   // codegen: the value reaches the output without an add/sub
 };
 
 struct XStmt {

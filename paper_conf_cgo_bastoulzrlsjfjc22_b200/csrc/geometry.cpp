@@ -426,7 +426,9 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       bool rinv = true;
       for (size_t q = 1; q < L.kl.size(); q++) rinv &= coef(L, L.loads[k], (int)q) == 0;
       const int es_k = esize(d.t[L.loads[k].tensor].dtype);
-      L.load_cb[k] = rinv ? es_k : std::min(vmax, W * es_k);   // row-invariant: element-wise
+      // row-invariant (LayerNorm's gamma/beta): two aligned vectors around the
+      // shifted window when the base is vector-aligned, element-wise otherwise
+      L.load_cb[k] = rinv && L.loads[k].base % W != 0 ? es_k : std::min(vmax, W * es_k);
     }
     for (size_t k = 0; k < L.stmts.size(); k++)
       if (coef(L, L.stmts[k].write, 0) == 1) L.store_cb[k] = std::min(vmax, W * esize(L.stmts[k].out_dtype));
