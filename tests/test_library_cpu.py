@@ -309,3 +309,31 @@ def test_mirrored_smem_transpose_needs_aligned_input_rows():
                     "reads": [("x0", ["l3", "l2", "l0"])],
                     "expr": [("load", 0), ("const", 0.5), ("add", 1, 0), ("div", 2, 2), ("cast", 3, "bf16")]}]}
     FusedOp(d)
+
+
+def test_peel_chosen_for_odd_rows_only():
+    """Per-row peel: rows of odd length keep the full vector width; even rows
+    plan exactly as before (no shift code)."""
+    assert "pe_s" in FusedOp(W.cfg4a(2, 64, 771), jit=0, autotune=0).source()
+    assert "pe_s" not in FusedOp(W.cfg4a(2, 64, 768), jit=0, autotune=0).source()
+    li = FusedOp(W.N4["vocab_softmax"](R=4, V=50257), jit=0, autotune=0).info()["launches"][0]
+    assert (li["class"], li["width"]) == ("row_reduce", 8)
+
+
+def test_fast_forms_not_ahead_of_add_or_subtract():
+    """16-bit fast forms (÷ invariant as × rcp) only where the value reaches the
+    output without an add/sub (fuzz seed 21 case 294)."""
+    def op(expr):
+        return {"name": "fast", "loops": {"a": 64, "b": 256},
+                "tensors": {"x": {"shape": [64, 256], "dtype": "f32", "role": "in", "init": ("normal", 0.0, 1.0, 1),
+                                  "strides": None},
+                            "y": {"shape": [64, 256], "dtype": "f32", "role": "in", "init": ("normal", 0.0, 1.0, 2),
+                                  "strides": None},
+                            "out": {"shape": [64, 256], "dtype": "f16", "role": "out", "init": None, "strides": None}},
+                "stmts": [{"kind": "assign", "loops": ["a", "b"], "write": ("out", ["a", "b"]),
+                           "reads": [("x", ["a", "b"]), ("y", ["a", "b"])], "expr": expr}]}
+    direct = FusedOp(op([("load", 0), ("const", -1.5), ("div", 0, 1)]), jit=0, autotune=0).source()
+    assert "__frcp_rn" in direct                       # x / c -> x * rcp(c): result stored directly
+    summed = FusedOp(op([("load", 0), ("const", -1.5), ("div", 0, 1), ("load", 1), ("add", 2, 3)]),
+                     jit=0, autotune=0).source()
+    assert "__frcp_rn" not in summed and "__fdiv_rn" in summed
