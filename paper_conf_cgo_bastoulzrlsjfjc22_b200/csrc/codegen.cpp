@@ -205,8 +205,13 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
       case FOP_OP_MUL: e = "fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + ")"; break;
       case FOP_OP_GELU_TANH: e = "fop::op_gelu_tanh2(" + opnd(n.a) + ")"; break;
       case FOP_OP_DIV:
-        if (fast_ok(n) && !var[n.b]) {  // ÷ loop-invariant -> × correctly rounded reciprocal
-          e = "fop::mul2(" + opnd(n.a) + ", fop::pk1(__frcp_rn(" + node_name(x, var, n.b, c) + ")))";
+        if (g_approx16 && !var[n.b]) {
+          // ÷ loop-invariant d -> × r = RN(1/d), then one remainder step
+          // (q = RN(a r); q += RN(a - q d) r, the remainder exact by FMA):
+          // the quotient to within an fp32 ulp (Markstein's correction) even
+          // where an add/sub follows and cancels, 1.5 packed FMAs per element
+          const std::string dn = node_name(x, var, n.b, c), pa = opnd(n.a);
+          e = "fop::div2_by(" + pa + ", " + dn + ")";
           break;
         }
         [[fallthrough]];

@@ -399,6 +399,15 @@ __device__ __forceinline__ u64 fma2(u64 a, u64 b, u64 c) {
   return r;
 }
 
+// a / d for a pair by a loop-invariant d: q0 = RN(a r) with r = RN(1/d),
+// remainder a - q0 d exact by FMA, q = RN(q0 + rem r) (codegen: 16-bit outputs)
+__device__ __forceinline__ u64 div2_by(u64 a, float d) {
+  const float r = __frcp_rn(d);
+  const u64 q0 = mul2(a, pk1(r));
+  const u64 rem = fma2(q0, pk1(-d), a);
+  return fma2(rem, pk1(r), q0);
+}
+
 // GELU, tanh form: 0.5 v (1 + tanh u) == v * sigmoid(2u) = v / (1 + 2^(v * (C2 + C1 v^2)))
 // with u = sqrt(2/pi)(v + 0.044715 v^3), C2 = -2 sqrt(2/pi) log2(e), C1 = 0.044715 C2.
 // MUFU.EX2 + MUFU.RCP: relative error ~1e-6, far inside one fp16/bf16 ulp

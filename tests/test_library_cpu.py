@@ -321,7 +321,8 @@ def test_peel_chosen_for_odd_rows_only():
 
 
 def test_fast_forms_not_ahead_of_add_or_subtract():
-    """16-bit fast forms (÷ invariant as × rcp) only where the value reaches the
+    """16-bit fast forms: ÷ invariant as × rcp with a remainder correction
+    everywhere; exp/sigmoid approximations only where the value reaches the
     output without an add/sub (fuzz seed 21 case 294)."""
     def op(expr):
         return {"name": "fast", "loops": {"a": 64, "b": 256},
@@ -332,8 +333,12 @@ def test_fast_forms_not_ahead_of_add_or_subtract():
                             "out": {"shape": [64, 256], "dtype": "f16", "role": "out", "init": None, "strides": None}},
                 "stmts": [{"kind": "assign", "loops": ["a", "b"], "write": ("out", ["a", "b"]),
                            "reads": [("x", ["a", "b"]), ("y", ["a", "b"])], "expr": expr}]}
+    # division by an invariant: x * rcp(c) plus one remainder correction, also ahead of an add
     direct = FusedOp(op([("load", 0), ("const", -1.5), ("div", 0, 1)]), jit=0, autotune=0).source()
-    assert "__frcp_rn" in direct                       # x / c -> x * rcp(c): result stored directly
     summed = FusedOp(op([("load", 0), ("const", -1.5), ("div", 0, 1), ("load", 1), ("add", 2, 3)]),
                      jit=0, autotune=0).source()
-    assert "__frcp_rn" not in summed and "__fdiv_rn" in summed
+    assert "fop::div2_by(" in direct and "fop::div2_by(" in summed
+    # exp's fast form only where no add/sub follows
+    e_direct = FusedOp(op([("load", 0), ("exp", 0)]), jit=0, autotune=0).source()
+    e_summed = FusedOp(op([("load", 0), ("exp", 0), ("load", 1), ("add", 1, 2)]), jit=0, autotune=0).source()
+    assert "fop::exp_fast(" in e_direct and "fop::exp_fast(" not in e_summed
