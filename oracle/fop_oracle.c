@@ -23,6 +23,12 @@
  *      fp32, then the finalize DAG (fp32) and the conversion (readings R16,
  *      R19);
  *   5. later statements read the stored (rounded) values (reading R17).
+ *   6. an INTEGER statement (its target is i32, reading R30) evaluates its
+ *      DAG on int32 values: every i32 load, constant and + - * max min neg
+ *      abs relu result is computed in int64 and reduced modulo 2^32 to the
+ *      two's-complement int32 range (wrap-around); REDUCE sums modulo 2^32
+ *      (wrapping after every term), MAX keeps the maximum.  Float statements never read i32 tensors, and integer
+ *      statements never read float tensors, except a pure element move.
  * No blocking, no reordering, no threads.
  */
 #include "fop_oracle.h"
@@ -160,6 +166,32 @@ static float apply(const orc_node *n, const float *val, float acc, float loaded)
   return NAN;
 }
 
+/* Integer statements (reading R30): int32 values, two's-complement wrap-around
+ * after every operation (the int64 result reduced modulo 2^32).            */
+static long long wrap32(long long v) {
+  unsigned long long u = (unsigned long long)v & 0xFFFFFFFFull;
+  return u >= 0x80000000ull ? (long long)u - 0x100000000ll : (long long)u;
+}
+
+static long long apply_int(const orc_node *n, const long long *val, long long acc, long long loaded) {
+  long long a = n->x >= 0 ? val[n->x] : 0;
+  long long b = n->y >= 0 ? val[n->y] : 0;
+  switch (n->kind) {
+    case ORC_LOAD: return loaded;
+    case ORC_CONST: return wrap32((long long)n->c);
+    case ORC_ACC: return acc;
+    case ORC_ADD: return wrap32(a + b);
+    case ORC_SUB: return wrap32(a - b);
+    case ORC_MUL: return wrap32(a * b); /* |a|, |b| <= 2^31: the product fits in int64 */
+    case ORC_MAX: return a > b ? a : b;
+    case ORC_MIN: return a < b ? a : b;
+    case ORC_NEG: return wrap32(-a);
+    case ORC_ABS: return wrap32(a < 0 ? -a : a);
+    case ORC_RELU: return a > 0 ? a : 0;
+  }
+  return 0;
+}
+
 /* ---------------------------------------------------------------------- */
 /* Element addressing and typed load/store.                               */
 
@@ -177,19 +209,23 @@ static float load_elem(const orc_array *arr, long long o) {
     case ORC_F32: return ((const float *)arr->data)[o];
     case ORC_F16: return orc_f16_to_f32(((const uint16_t *)arr->data)[o]);
     case ORC_BF16: return orc_bf16_to_f32(((const uint16_t *)arr->data)[o]);
-    case ORC_I32: return (float)((const int32_t *)arr->data)[o];
+    case ORC_I32: break; /* i32 elements are read by integer statements only (load_int) */
   }
   return NAN;
 }
+
+static long long load_int(const orc_array *arr, long long o) { return ((const int32_t *)arr->data)[o]; }
 
 static void store_elem(orc_array *arr, long long o, float v) {
   switch (arr->elem) {
     case ORC_F32: ((float *)arr->data)[o] = v; break;
     case ORC_F16: ((uint16_t *)arr->data)[o] = orc_f32_to_f16(v); break;
     case ORC_BF16: ((uint16_t *)arr->data)[o] = orc_f32_to_bf16(v); break;
-    case ORC_I32: ((int32_t *)arr->data)[o] = (int32_t)v; break;
+    case ORC_I32: break; /* written by integer statements only (store_int) */
   }
 }
+
+static void store_int(orc_array *arr, long long o, long long v) { ((int32_t *)arr->data)[o] = (int32_t)wrap32(v); }
 
 static long long array_span(const orc_array *a) {
   long long s = 1;
@@ -244,12 +280,51 @@ static int check_dag(const orc_node *nodes, int n, int nreads, int allow_acc, in
   return 0;
 }
 
+/* Element types of a statement (reading R30): a pure element move copies any
+ * type; a statement writing an i32 tensor is an integer statement (i32 reads,
+ * integer operations, integral constants); any other statement is a float
+ * statement and reads no i32 tensor. */
+static int is_move(const orc_statement *st, const orc_array *arrays) {
+  return !st->reduce && st->nnodes == 1 && st->nodes[0].kind == ORC_LOAD &&
+         arrays[st->reads[st->nodes[0].x].array].elem == arrays[st->target.array].elem;
+}
+
+static int int_node_ok(const orc_node *q) {
+  switch (q->kind) {
+    case ORC_LOAD: case ORC_ACC: case ORC_ADD: case ORC_SUB: case ORC_MUL: case ORC_MAX:
+    case ORC_MIN: case ORC_NEG: case ORC_ABS: case ORC_RELU: return 1;
+    case ORC_CONST: return q->c == floor(q->c) && q->c >= -2147483648.0 && q->c < 2147483648.0;
+  }
+  return 0;
+}
+
+static int check_types(const orc_statement *st, const orc_array *arrays, int s, char *err, int errlen) {
+  if (is_move(st, arrays)) return 0;
+  int integer = arrays[st->target.array].elem == ORC_I32;
+  for (int r = 0; r < st->nreads; r++)
+    if ((arrays[st->reads[r].array].elem == ORC_I32) != integer)
+      return fail(err, errlen, integer ? "integer statement reads a float tensor"
+                                       : "float statement reads an i32 tensor", s);
+  for (int i = 0; i < st->nnodes; i++) {
+    if (integer && !int_node_ok(&st->nodes[i])) return fail(err, errlen, "operation not defined on i32", s);
+    if (!integer && st->nodes[i].kind == ORC_CAST && st->nodes[i].elem == ORC_I32)
+      return fail(err, errlen, "cast to i32", s);
+  }
+  for (int i = 0; st->reduce && i < st->nfin; i++) {
+    if (integer && !int_node_ok(&st->fin[i])) return fail(err, errlen, "operation not defined on i32", s);
+    if (!integer && st->fin[i].kind == ORC_CAST && st->fin[i].elem == ORC_I32)
+      return fail(err, errlen, "cast to i32", s);
+  }
+  return 0;
+}
+
 /* ---------------------------------------------------------------------- */
 
 static int run_statement(const orc_statement *st, const long long *ext, orc_array *arrays,
                          int narrays, int s, char *err, int errlen) {
   long long it[ORC_LOOPS] = {0};
   float val[ORC_NODES];
+  long long ival[ORC_NODES];
   orc_array *tgt = &arrays[st->target.array];
   double *acc = NULL;
   unsigned char *seen = NULL;
@@ -258,15 +333,18 @@ static int run_statement(const orc_statement *st, const long long *ext, orc_arra
   for (int k = 0; k < st->nloops; k++) total *= ext[st->loops[k]];
 
   /* a pure element move (transpose / copy of any type) keeps the raw bits */
-  int move = !st->reduce && st->nnodes == 1 && st->nodes[0].kind == ORC_LOAD &&
-             arrays[st->reads[st->nodes[0].x].array].elem == tgt->elem;
+  int move = is_move(st, arrays);
+  int integer = !move && tgt->elem == ORC_I32;
+  long long *iacc = NULL;
 
   if (st->reduce) {
     span = array_span(tgt);
     acc = (double *)malloc(sizeof(double) * (size_t)(span > 0 ? span : 1));
     seen = (unsigned char *)calloc((size_t)(span > 0 ? span : 1), 1);
-    if (!acc || !seen) {
+    iacc = (long long *)malloc(sizeof(long long) * (size_t)(span > 0 ? span : 1));
+    if (!acc || !seen || !iacc) {
       free(acc);
+      free(iacc);
       free(seen);
       return fail(err, errlen, "out of memory", s);
     }
@@ -280,6 +358,28 @@ static int run_statement(const orc_statement *st, const long long *ext, orc_arra
       long long so = ref_offset(src, r, it), to = ref_offset(tgt, &st->target, it);
       size_t es = (src->elem == ORC_F32 || src->elem == ORC_I32) ? 4 : 2;
       memcpy((char *)tgt->data + to * (long long)es, (const char *)src->data + so * (long long)es, es);
+    } else if (integer) {
+      for (int i = 0; i < st->nnodes; i++) {
+        const orc_node *q = &st->nodes[i];
+        long long loaded = 0;
+        if (q->kind == ORC_LOAD) {
+          const orc_ref *r = &st->reads[q->x];
+          loaded = load_int(&arrays[r->array], ref_offset(&arrays[r->array], r, it));
+        }
+        ival[i] = apply_int(q, ival, 0, loaded);
+      }
+      long long v = ival[st->nnodes - 1];
+      long long to = ref_offset(tgt, &st->target, it);
+      if (!st->reduce) {
+        store_int(tgt, to, v);
+      } else {
+        if (!seen[to]) {
+          seen[to] = 1;
+          iacc[to] = st->reduce_max ? v : 0;
+        }
+        /* max exact; the sum wraps after every term (arithmetic modulo 2^32) */
+        iacc[to] = st->reduce_max ? (v > iacc[to] ? v : iacc[to]) : wrap32(iacc[to] + v);
+      }
     } else {
       for (int i = 0; i < st->nnodes; i++) {
         const orc_node *q = &st->nodes[i];
@@ -313,7 +413,17 @@ static int run_statement(const orc_statement *st, const long long *ext, orc_arra
     }
   }
 
-  if (st->reduce) {
+  if (st->reduce && integer) {
+    for (long long o = 0; o < span; o++) {
+      if (!seen[o]) continue;
+      long long r = wrap32(iacc[o]);
+      if (st->nfin > 0) {
+        for (int i = 0; i < st->nfin; i++) ival[i] = apply_int(&st->fin[i], ival, r, 0);
+        r = ival[st->nfin - 1];
+      }
+      store_int(tgt, o, r);
+    }
+  } else if (st->reduce) {
     for (long long o = 0; o < span; o++) {
       if (!seen[o]) continue;
       float r = (float)acc[o];
@@ -323,7 +433,10 @@ static int run_statement(const orc_statement *st, const long long *ext, orc_arra
       }
       store_elem(tgt, o, r);
     }
+  }
+  if (st->reduce) {
     free(acc);
+    free(iacc);
     free(seen);
   }
   (void)narrays;
@@ -349,6 +462,7 @@ int orc_run(int nloops, const long long *extents, int narrays, orc_array *arrays
       if (check_ref(&st->reads[r], st, narrays, arrays, extents, s, err, errlen)) return 1;
     if (check_dag(st->nodes, st->nnodes, st->nreads, 0, s, err, errlen)) return 1;
     if (st->reduce && st->nfin > 0 && check_dag(st->fin, st->nfin, 0, 1, s, err, errlen)) return 1;
+    if (check_types(st, arrays, s, err, errlen)) return 1;
     if (st->reduce)
       for (int r = 0; r < st->nreads; r++)
         if (st->reads[r].array == st->target.array)

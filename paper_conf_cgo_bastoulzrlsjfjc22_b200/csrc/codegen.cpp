@@ -102,18 +102,24 @@ struct DagCtx {
   std::string ev = "e";                                      // scalar element loop variable
 };
 
+// Decide the 16-bit fast forms of one statement (g_approx16, XNode::no_addsub).
+// Called before ANY of the statement's nodes is emitted — per-CTA tables
+// included — so every geometry variant of a launch makes the same choice and
+// produces the same bits.
+void decide_fast(const XStmt& x) {
+  const char* e = std::getenv("FOP_APPROX16");
+  g_approx16 = !(e && *e == '0') && x.kind == FOP_ASSIGN && esize(x.out_dtype) == 2 && x.out_dtype != FOP_I32;
+  std::vector<bool> feeds(x.nodes.size(), false);   // value reaches an add/sub
+  for (int i = (int)x.nodes.size() - 1; i >= 0; i--)
+    for (size_t j = i + 1; j < x.nodes.size(); j++) {
+      const XNode& q = x.nodes[j];
+      if ((q.a == i || q.b == i) && (q.op == FOP_OP_ADD || q.op == FOP_OP_SUB || feeds[j])) feeds[i] = true;
+    }
+  for (size_t i = 0; i < x.nodes.size(); i++) x.nodes[i].no_addsub = !feeds[i];
+}
+
 std::vector<bool> varies(const XStmt& x, const DagCtx& c) {
-  {  // every statement emission starts here: decide the 16-bit fast forms
-    const char* e = std::getenv("FOP_APPROX16");
-    g_approx16 = !(e && *e == '0') && x.kind == FOP_ASSIGN && esize(x.out_dtype) == 2 && x.out_dtype != FOP_I32;
-    std::vector<bool> feeds(x.nodes.size(), false);   // value reaches an add/sub
-    for (int i = (int)x.nodes.size() - 1; i >= 0; i--)
-      for (size_t j = i + 1; j < x.nodes.size(); j++) {
-        const XNode& q = x.nodes[j];
-        if ((q.a == i || q.b == i) && (q.op == FOP_OP_ADD || q.op == FOP_OP_SUB || feeds[j])) feeds[i] = true;
-      }
-    for (size_t i = 0; i < x.nodes.size(); i++) x.nodes[i].no_addsub = !feeds[i];
-  }
+  decide_fast(x);   // every statement emission starts here
   std::vector<bool> v(x.nodes.size(), false);
   for (size_t i = 0; i < x.nodes.size(); i++) {
     const XNode& n = x.nodes[i];
@@ -237,7 +243,7 @@ struct Sink {
   std::function<void(const std::string&, const std::string&)> pair;        // packed value, pair var
   std::function<void(const std::string&, const std::string&, const std::string&)> pair_fma;  // a, b, pair var
 };
-bool g_packed = true;
+thread_local bool g_packed = true;
 void emit_elems(Out& o, const XStmt& x, const std::vector<bool>& var, const DagCtx& c, int W, const Sink& s) {
   bool packed = g_packed && W % 2 == 0 && s.pair;
   if (!packed) {
@@ -443,6 +449,7 @@ struct Gen {
     if (tables.empty()) return;
     for (const Table& t : tables) {
       const XStmt& x = L.stmts[t.si];
+      decide_fast(x);   // the table's nodes take the same forms as the statement's own emission
       o.l("__shared__ __align__(16) float " + t.name + "[" + num(t.E) + "];");
       o.l("for (unsigned ti = threadIdx.x; ti < " + num(t.E) + "u; ti += " + num(L.block) + "u) {");
       o.ind++;
@@ -2221,9 +2228,16 @@ struct Gen {
       o.l("{");
       o.ind++;
       o.l("__shared__ float xv_[" + num(NP) + "];");
-      if (!geometry_knob(L, "FOP_PEER_EP", 0))
-        o.l("const unsigned xep0_ = ((volatile const unsigned*)(args.peer[args.rank] + " + base + "ull + " +
+      if (!geometry_knob(L, "FOP_PEER_EP", 0)) {
+        // one thread reads the run counter and shares it: thread 0 writes the
+        // next value below, and a warp still to read the global counter would
+        // see it (the epoch would be off by one on that warp only)
+        o.l("__shared__ unsigned xeps_;");
+        o.l("if (tid == 0u) xeps_ = ((volatile const unsigned*)(args.peer[args.rank] + " + base + "ull + " +
             num((int64_t)pl.epoch) + "ull))[slab];");
+        o.l("__syncthreads();");
+        o.l("const unsigned xep0_ = xeps_;");
+      }
       o.l("const unsigned xe_ = xep0_ + 1u, xp_ = xe_ & 1u;");
       o.l("const u64* const xb_ = (const u64*)(args.peer[args.rank] + " + base + "ull);");
       o.l("if (tid == 0u) ((volatile unsigned*)(args.peer[args.rank] + " + base + "ull + " + num((int64_t)pl.epoch) +
@@ -2375,6 +2389,7 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
   {
     const char* e = std::getenv("FOP_PACKED");   // 0: scalar fp32 DAG evaluation (ablation)
     g_packed = !(e && *e == '0');
+    g_approx16 = false;                           // set per statement by decide_fast()
   }
   Gen g(p, L);
   // 32-bit index arithmetic when every offset and work index fits

@@ -400,12 +400,32 @@ __device__ __forceinline__ u64 fma2(u64 a, u64 b, u64 c) {
 }
 
 // a / d for a pair by a loop-invariant d: q0 = RN(a r) with r = RN(1/d),
-// remainder a - q0 d exact by FMA, q = RN(q0 + rem r) (codegen: 16-bit outputs)
+// remainder rem = RN(a - q0 d) by FMA, q = RN(q0 + rem r).  With r the
+// correctly rounded reciprocal and q0 within one ulp of a/d this is
+// Markstein's correction: q == RN(a/d), the same bits as __fdiv_rn
+// (tests/test_fastdiv.py checks the formula against exact rational division).
+// Outside the range where the theorem's premises hold the lane takes
+// __fdiv_rn itself: d zero, subnormal, huge, inf or NaN (r not a normal
+// number: uniform over the launch, d is invariant); a quotient that overflows,
+// underflows or is not a number (q0 outside [2^-100, FLT_MAX]); a dividend
+// below 2^-100 (its remainder would be subnormal, hence inexact); a = +-0 keeps
+// q0 (the correction would turn -0 into +0).
+__device__ __forceinline__ bool div_by_ok(float d) { return fabsf(d) >= 0x1p-125f && fabsf(d) <= 0x1p125f; }
+__device__ __forceinline__ float div_by_fix(float q, float q0, float a, float d) {
+  const float m = fabsf(q0);
+  if (m >= 0x1p-100f && m <= 0x1.fffffep127f && fabsf(a) >= 0x1p-100f) return q;
+  return a == 0.0f ? q0 : __fdiv_rn(a, d);
+}
 __device__ __forceinline__ u64 div2_by(u64 a, float d) {
+  if (!div_by_ok(d)) return pk(__fdiv_rn(lo(a), d), __fdiv_rn(hi(a), d));
   const float r = __frcp_rn(d);
   const u64 q0 = mul2(a, pk1(r));
   const u64 rem = fma2(q0, pk1(-d), a);
-  return fma2(rem, pk1(r), q0);
+  const u64 q = fma2(rem, pk1(r), q0);
+  const float m0 = fabsf(lo(q0)), m1 = fabsf(hi(q0));
+  const float a0 = fabsf(lo(a)), a1 = fabsf(hi(a));
+  if (fminf(fminf(m0, m1), fminf(a0, a1)) >= 0x1p-100f && fmaxf(m0, m1) <= 0x1.fffffep127f) return q;
+  return pk(div_by_fix(lo(q), lo(q0), lo(a), d), div_by_fix(hi(q), hi(q0), hi(a), d));
 }
 
 // GELU, tanh form: 0.5 v (1 + tanh u) == v * sigmoid(2u) = v / (1 + 2^(v * (C2 + C1 v^2)))

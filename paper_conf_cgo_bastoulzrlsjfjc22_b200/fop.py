@@ -365,12 +365,15 @@ class FusedOp:
         return _lib.fop_plan_peer_bytes(self._h)
 
     # ------------------------------------------------------------ execution
-    def _workspace(self, device):
+    def _workspace(self, device, stream):
+        """The cached zero-filled workspace for (device, stream).  Runs of one plan on
+        DIFFERENT streams may overlap, and a workspace holds per-run state (COL_REDUCE
+        partial sums and arrival counters, TEMP tensors), so each stream gets its own."""
         import torch
         n = self.workspace_bytes
         if n == 0:
             return None
-        key = str(device)
+        key = (str(device), int(stream.cuda_stream))
         if key not in self._ws:
             self._ws[key] = torch.zeros(n, dtype=torch.uint8, device=device)  # zero-filled (fop.h)
         return self._ws[key]
@@ -391,6 +394,14 @@ class FusedOp:
                             f"{self.desc['tensors'][n]['dtype']} ({want})")
         if t.is_cuda != (where == "cuda"):
             raise ValueError(f"tensor {n!r} is on {t.device}, expected a {'CUDA' if where == 'cuda' else 'host'} tensor")
+        # the library addresses memory from data_ptr() with the DESCRIPTOR's strides: a strided
+        # view (x.t(), x[:, :768], an expand) would silently read or write other elements
+        if not t.is_contiguous():
+            sp = self.desc["tensors"][n]
+            st = _strides(sp)
+            if t.dim() != len(sp["shape"]) or any(a != b for a, b, e in zip(t.stride(), st, sp["shape"]) if e > 1):
+                raise ValueError(f"tensor {n!r}: a non-contiguous view (strides {tuple(t.stride())}) whose strides "
+                                 f"differ from the descriptor's {tuple(st)}; pass .contiguous() or describe its strides")
         have = t.untyped_storage().nbytes() - t.storage_offset() * t.element_size()
         if need > have:
             raise ValueError(f"tensor {n!r}: the descriptor addresses {need} bytes from its base pointer, "
@@ -424,10 +435,10 @@ class FusedOp:
         peers: a PeerGroup for plans with a cross-GPU exchange (fop_run_peer)."""
         import torch
         arr, dev = self._ptrs(tensors)
-        ws = workspace if workspace is not None else self._workspace(dev)
-        self._check_workspace(ws, dev)
         if stream is None:
             stream = torch.cuda.current_stream(dev)
+        ws = workspace if workspace is not None else self._workspace(dev, stream)
+        self._check_workspace(ws, dev)
         if peers is not None:
             _check(_lib.fop_run_peer(self._h, arr, len(self.names), None if ws is None else ws.data_ptr(),
                                      C.byref(peers.c), stream.cuda_stream))
@@ -440,10 +451,10 @@ class FusedOp:
         import torch
         arr, dev = self._ptrs(device_tensors)
         harr = self._host_ptrs(host)
-        ws = workspace if workspace is not None else self._workspace(dev)
-        self._check_workspace(ws, dev)
         if stream is None:
             stream = torch.cuda.current_stream(dev)
+        ws = workspace if workspace is not None else self._workspace(dev, stream)
+        self._check_workspace(ws, dev)
         _check(_lib.fop_run_host(self._h, harr, arr, len(self.names),
                                  None if ws is None else ws.data_ptr(), stream.cuda_stream))
 
@@ -470,12 +481,15 @@ def run_host_many(items, stream=None):
     ws = (C.c_void_p * n)()
     keep = []
     dev = None
+    for it in items:
+        dev = dev or it[0]._ptrs(it[2])[1]
+    if stream is None:
+        stream = torch.cuda.current_stream(dev)
     for k, it in enumerate(items):
         op, host, devt = it[0], it[1], it[2]
         arr, d = op._ptrs(devt)
-        dev = dev or d
         harr = op._host_ptrs(host)
-        w = it[3] if len(it) > 3 and it[3] is not None else op._workspace(d)
+        w = it[3] if len(it) > 3 and it[3] is not None else op._workspace(d, stream)
         op._check_workspace(w, d)
         keep += [arr, harr]
         plans[k] = op._h
@@ -483,8 +497,6 @@ def run_host_many(items, stream=None):
         dp[k] = C.cast(arr, C.POINTER(C.c_void_p))
         np_[k] = len(op.names)
         ws[k] = None if w is None else w.data_ptr()
-    if stream is None:
-        stream = torch.cuda.current_stream(dev)
     _check(_lib.fop_run_host_many(plans, hp, dp, np_, ws, n, stream.cuda_stream))
 
 
@@ -540,18 +552,20 @@ def run_many(items, stream=None):
     ws = (C.c_void_p * n)()
     keep = []
     dev = None
+    for it in items:
+        dev = dev or it[0]._ptrs(it[1])[1]
+    if stream is None:
+        stream = torch.cuda.current_stream(dev)
     for k, it in enumerate(items):
         op, devt = it[0], it[1]
         arr, d = op._ptrs(devt)
-        dev = dev or d
-        w = it[2] if len(it) > 2 and it[2] is not None else op._workspace(d)
+        w = it[2] if len(it) > 2 and it[2] is not None else op._workspace(d, stream)
+        op._check_workspace(w, d)
         keep.append(arr)
         plans[k] = op._h
         dp[k] = C.cast(arr, C.POINTER(C.c_void_p))
         np_[k] = len(op.names)
         ws[k] = None if w is None else w.data_ptr()
-    if stream is None:
-        stream = torch.cuda.current_stream(dev)
     _check(_lib.fop_run_many(plans, dp, np_, ws, n, stream.cuda_stream))
 
 

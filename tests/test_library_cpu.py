@@ -237,6 +237,15 @@ def test_binding_rejects_wrong_buffers_before_the_abi():
         op.run(good)                          # host tensors where device tensors are required
     with pytest.raises(ValueError, match="missing"):
         op.run({n: t for n, t in good.items() if n != "x"})
+    # strided views: the library would address them with the descriptor's strides
+    big = torch.zeros(2 * 64, 2 * 768, dtype=torch.float16)
+    with pytest.raises(ValueError, match="non-contiguous"):
+        op._host_ptrs(dict(good, x=big[:, :768]))          # a column slice: pitch 1536, not 768
+    with pytest.raises(ValueError, match="non-contiguous"):
+        op._host_ptrs(dict(good, x=torch.zeros(768, 2 * 64, dtype=torch.float16).t()))
+    op._host_ptrs(dict(good, x=torch.zeros(2, 64, 768, dtype=torch.float16)))   # contiguous, any shape
+    ok = torch.zeros(2, 64, 768, dtype=torch.float16)[:, :, :]                   # a view with matching strides
+    op._host_ptrs(dict(good, x=ok))
 
 
 def test_transpose_vector_loop_absorbs_contiguous_continuations():

@@ -576,7 +576,7 @@ def test_cuda_graph_capture_and_replay(warm):
     ops = [FusedOp(d) for d in descs]
     xs = [W.make_inputs(d) for d in descs]
     devs = [device_tensors(d, x) for d, x in zip(descs, xs)]
-    wss = [op._workspace(torch.device("cuda")) for op in ops]
+    wss = [op._workspace(torch.device("cuda"), torch.cuda.current_stream()) for op in ops]
     if warm:
         for op, dv, ws in zip(ops, devs, wss):
             op.run(dv, workspace=ws)
