@@ -161,18 +161,20 @@ def cpu_oracle_step(inputs_cache):
 
 
 # the same sample on every host core: the oracle unchanged, one process per
-# core, each on a contiguous block of the sample's parallel loop
-# (dist.shard_desc; independent slices, no communication); reported next to
-# the 1-core number, baseline only
+# core, each on a contiguous block of the sample's parallel loop — the same
+# operator built at the block's extent (the blocks are independent: no
+# communication); reported next to the 1-core number, baseline only.  Built
+# here from workloads/ alone: this leg imports nothing from the product.
 SHARD_LOOP = {"cfg2": "n", "cfg3": "n", "cfg4a": "b", "cfg4b": "c"}
+SHARD_BUILD = {"cfg2": lambda e: W.cfg2(N=e), "cfg3": lambda e: W.cfg3(N=e),
+               "cfg4a": lambda e: W.cfg4a(B=e), "cfg4b": lambda e: W.cfg4b(R=65536, C=e)}
 
 
 def _oracle_shard(job):
     name, k, n = job
     from oracle import oracle as O
-    from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc
     d = dict(CPU_SAMPLE)[name]()
-    sh, _ = shard_desc(d, SHARD_LOOP[name], k, n)
+    sh = SHARD_BUILD[name](d["loops"][SHARD_LOOP[name]] // n)
     x = W.make_inputs(sh, seed_offset=k)
     t0 = time.perf_counter()
     O.run(sh, x)

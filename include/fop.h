@@ -49,7 +49,7 @@ extern "C" {
 #define FOP_API
 #endif
 
-#define FOP_ABI_VERSION 3
+#define FOP_ABI_VERSION 4
 
 #define FOP_MAX_RANK     8   /* tensor rank */
 #define FOP_MAX_LOOPS    8   /* loops of the fused operator */
@@ -182,6 +182,11 @@ typedef struct {
   int32_t peer_timeout_ms;       /* bound on a kernel's wait for its peers; 0 = 10000.  On timeout the
                                     run's exchanged outputs are NaN and the exchange buffer's error word
                                     is set (fop_peer_group) */
+  int32_t variant;               /* -1 (default): auto-tune as above.  k >= 0: no timing; every launch runs
+                                    its tuning candidate k (0 = the default geometry; a launch with fewer
+                                    candidates, see fop_launch_info.nvariants, runs its default).  Lets a
+                                    test run each candidate the tuner could pick (they must all agree with
+                                    the oracle: schedules are semantics preserving). */
 } fop_plan_opts;
 
 typedef enum {
@@ -210,6 +215,7 @@ typedef struct {
                                 explicit vector type, 3 fully sequential (every loop carries a
                                 dependence) */
   int32_t peer_exchange;     /* 1: this launch combines partial results across the peer group */
+  int32_t nvariants;         /* tuning candidates compiled for this launch, the default geometry included */
 } fop_launch_info;
 
 typedef struct {

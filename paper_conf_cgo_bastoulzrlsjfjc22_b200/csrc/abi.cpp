@@ -60,6 +60,7 @@ void fop_plan_opts_default(fop_plan_opts* o) {
   o->sm_count = 148;
   o->jit = 1;
   o->autotune = 1;
+  o->variant = -1;
 }
 
 fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t** out) {
@@ -77,6 +78,7 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
           p.opts.max_vec_bytes != 32)
         fop::fail(FOP_E_INVALID, "max_vec_bytes must be 4, 8, 16 or 32");
       if (p.opts.peer_world < 0 || p.opts.peer_timeout_ms < 0) fop::fail(FOP_E_INVALID, "negative peer option");
+      if (p.opts.variant < -1) fop::fail(FOP_E_INVALID, "variant must be -1 (auto-tune) or >= 0");
       fop::validate(p.desc);
       fop::plan_launches(p);
       // narrow (scalar) variants for misaligned base pointers: geometry now,
@@ -114,7 +116,7 @@ fop_status fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fop_plan_t*
         }
       }
       p.variants.assign(p.launches.size(), {});
-      if (p.opts.autotune && p.opts.jit && p.tunable) {
+      if ((p.opts.autotune || p.opts.variant > 0) && p.opts.jit && p.tunable) {
         for (size_t i = 0; i < p.launches.size(); i++) {
           if (p.launches[i].peer) continue;   // every rank must run the same geometry (fop_run_peer)
           auto vs = fop::tuning_variants(p.launches[i], p.opts.sm_count > 0 ? p.opts.sm_count : 148);
@@ -188,6 +190,7 @@ fop_status fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* o) {
       li.scen_pick = L.scen_pick;
       li.fallback = L.fallback;
       li.peer_exchange = L.peer ? 1 : 0;
+      li.nvariants = 1 + (i < p.variants.size() ? (int32_t)p.variants[i].size() : 0);
     }
     o->workspace_bytes = p.ws_bytes;
     for (int s = 0; s < p.desc.nstmts; s++) {

@@ -637,7 +637,7 @@ struct Gen {
         for (const Table& tb : tables)
           if (tb.si == (int)si)
             for (auto& kv : its[u])
-              if (kv.first == tb.k)   // slots past the end (ok false) still evaluate: keep the index in the table
+              if (kv.first == tb.k) {  // slots past the end (ok false) still evaluate: keep the index in the table
                 if (tb.k == 0) {   // per element: the vector's W entries, read with 16 B shared loads
                   const std::string tv = "TV" + tb.name.substr(3) + t;
                   o.l("float " + tv + "[" + num(L.width) + "];");
@@ -653,6 +653,7 @@ struct Gen {
                 } else {
                   ov[tb.node] = tb.name + "[ok" + t + " ? " + kv.second + " : 0u]";
                 }
+              }
         g_over = &ov;
         auto var = varies(x, c);
         emit_nodes(o, x, var, false, c);

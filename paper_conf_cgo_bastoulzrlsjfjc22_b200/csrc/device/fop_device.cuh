@@ -483,7 +483,12 @@ __device__ __forceinline__ void round2(float a, float b, float& ra, float& rb) {
     rb = b;
   }
 }
-__device__ __forceinline__ float op_gelu_erf(float v) { return 0.5f * v * erfcf(-0.70710678118654752f * v); }
+// GELU, erf form: 0.5 v (1 + erf(v / sqrt 2)) = v Phi(v).  normcdff evaluates Phi
+// without first rounding v / sqrt 2 to fp32 (an erfcf(-v * 0.7071f) form
+// amplifies that rounding by ~v^2 in the negative tail); CUDA documents it to
+// 5 ulp over the whole range, so v * normcdff(v) is within 6 fp32 ulp
+// (tests/test_transcendental_gpu.py).
+__device__ __forceinline__ float op_gelu_erf(float v) { return __fmul_rn(v, normcdff(v)); }
 __device__ __forceinline__ float op_sigmoid(float v) { return __frcp_rn(1.0f + expf(-v)); }
 
 // Fast forms, used only for statements whose result is rounded to fp16/bf16

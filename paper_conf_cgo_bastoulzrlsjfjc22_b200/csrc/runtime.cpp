@@ -511,7 +511,9 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
       continue;
     }
     int ch = l.choice[i];
-    if (ch < 0) {
+    if (ch < 0 && p.opts.variant >= 0) {   // a forced candidate (fop.h: opts.variant), no timing
+      l.choice[i] = ch = p.opts.variant <= (int)p.variants[i].size() ? p.opts.variant : 0;
+    } else if (ch < 0) {
       int t = tune(i);
       if (t >= 0) l.choice[i] = ch = t;
       else ch = 0;   // capturing: default geometry, tune on a later eager run

@@ -68,7 +68,7 @@ class PlanOpts(C.Structure):
                 ("max_vec_bytes", C.c_int32), ("readings", C.c_int32), ("force_width", C.c_int32),
                 ("coalesce_order", C.c_int32), ("sm_count", C.c_int32), ("jit", C.c_int32),
                 ("autotune", C.c_int32), ("peer_world", C.c_int32), ("peer_loop", C.c_int32),
-                ("peer_timeout_ms", C.c_int32)]
+                ("peer_timeout_ms", C.c_int32), ("variant", C.c_int32)]
 
 
 class LaunchInfo(C.Structure):
@@ -76,7 +76,8 @@ class LaunchInfo(C.Structure):
                 ("vec_loop", C.c_int32), ("width", C.c_int32), ("read_loop", C.c_int32),
                 ("read_width", C.c_int32), ("coal_loop", C.c_int32), ("grid", C.c_int64),
                 ("block", C.c_int32), ("nseq", C.c_int32), ("seq", C.c_int32 * MAX_LOOPS),
-                ("scen_pick", C.c_int32), ("fallback", C.c_int32), ("peer_exchange", C.c_int32)]
+                ("scen_pick", C.c_int32), ("fallback", C.c_int32), ("peer_exchange", C.c_int32),
+                ("nvariants", C.c_int32)]
 
 
 class PlanInfo(C.Structure):
@@ -91,7 +92,7 @@ class PlanInfo(C.Structure):
 
 
 _lib.fop_abi_version.restype = C.c_int
-ABI_VERSION = 3   # the struct layouts above mirror include/fop.h at this version
+ABI_VERSION = 4   # the struct layouts above mirror include/fop.h at this version
 if _lib.fop_abi_version() != ABI_VERSION:
     raise ImportError(f"{LIB_PATH}: ABI version {_lib.fop_abi_version()} != binding {ABI_VERSION}; rebuild "
                       "with python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build")
@@ -332,7 +333,7 @@ class FusedOp:
                              "coal_loop": ln(li.coal_loop), "grid": li.grid, "block": li.block,
                              "seq": [ln(li.seq[q]) for q in range(li.nseq)],
                              "scen_pick": li.scen_pick, "fallback": li.fallback,
-                             "peer_exchange": bool(li.peer_exchange)})
+                             "peer_exchange": bool(li.peer_exchange), "nvariants": li.nvariants})
         return {"stmts": stmts, "launches": launches, "workspace_bytes": pi.workspace_bytes}
 
     @property

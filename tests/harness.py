@@ -109,6 +109,14 @@ def assert_normwise(got, ref, scale, tol, name=""):
     got = np.asarray(got, np.float64)
     ref = np.asarray(ref, np.float64)
     scale = np.asarray(scale, np.float64)
+    # non-finite results must match exactly (NaN where the oracle has NaN, the same infinities);
+    # a NaN would otherwise pass every `err > bound` test
+    nf = ~np.isfinite(ref) | ~np.isfinite(got)
+    same_nf = (np.isnan(got) & np.isnan(ref)) | (got == ref)
+    bad_nf = np.flatnonzero(nf & ~same_nf)
+    assert bad_nf.size == 0, f"{name}: non-finite mismatch at {bad_nf[:5]}: got {got.reshape(-1)[bad_nf[:5]]} " \
+                             f"ref {ref.reshape(-1)[bad_nf[:5]]}"
+    got, ref, scale = np.where(nf, 0, got), np.where(nf, 0, ref), np.where(nf, 0, scale)
     err = np.abs(got - ref)
     bound = tol * np.maximum(scale, np.finfo(np.float32).tiny)
     bad = np.flatnonzero(err > bound)

@@ -1,0 +1,69 @@
+"""Full-size parity of exactly what bench.py times: every auto-tuning candidate
+of cfg2 / cfg3 / cfg4a / cfg4b (BASELINE.json configs[1..3] at full size),
+forced one by one with opts.variant, compared with the oracle on the WHOLE
+output (not sampled slices).
+
+Schedules are semantics preserving (§IV-A1): whichever
+geometry the tuner picks must give the oracle's result — bit-exact for the
+ASSIGN outputs (cfg2, cfg3, cfg4a's y), the reading-R16 normwise bound for the
+reductions (cfg4a's mean/var, cfg4b's column sums), and identical bits for
+every candidate of one plan on the same inputs where the association order is
+the same.
+"""
+import numpy as np
+import pytest
+import torch
+
+import workloads as W
+from oracle import oracle as O
+
+from harness import abs_terms_desc, assert_bitexact, assert_normwise, assert_ulp, device_tensors, to_host
+
+pytestmark = [pytest.mark.gpu, pytest.mark.full_size]
+
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+
+def _run_variant(desc, dev_in, k):
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    op = FusedOp(desc, variant=k)
+    dev = dict(dev_in)
+    outs = W.alloc_outputs(desc)
+    from harness import to_device
+    for n, buf in outs.items():
+        dev[n] = to_device(buf, desc["tensors"][n]["dtype"])          # NaN-filled for every candidate
+    op.run(dev)
+    torch.cuda.synchronize()
+    name = op.selected(0)[0]
+    res = {n: to_host(dev[n], desc["tensors"][n]["dtype"]) for n in outs}
+    del dev
+    return res, name
+
+
+@pytest.mark.parametrize("name", ["cfg2", "cfg3", "cfg4a", "cfg4b"])
+def test_every_tuning_candidate_full_size_whole_output(name):
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    d = W.CONFIGS[name]()
+    nv = FusedOp(d, jit=1).info()["launches"][0]["nvariants"]
+    assert nv >= 2, "the bench's tuner has candidates to choose from"
+    x = W.make_inputs(d)
+    ref = O.run(d, x)
+    scale = {}
+    if name == "cfg4a":
+        scale = {"mean": O.run(abs_terms_desc(d, 1), x)["mean"], "var": O.run(abs_terms_desc(d, 2), x)["var"]}
+    elif name == "cfg4b":
+        scale = {"out": O.run(abs_terms_desc(d, 0), x)["out"]}
+    dev_in = device_tensors({**d, "tensors": {n: t for n, t in d["tensors"].items() if t["role"] == "in"}}, x)
+    seen = set()
+    for k in range(nv):
+        got, kname = _run_variant(d, dev_in, k)
+        seen.add(kname)
+        for n, v in got.items():
+            if n in scale:
+                assert_normwise(v, ref[n], scale[n], 1e-5, f"{name} candidate {k} ({kname}) {n}")
+            elif name == "cfg4a":
+                assert_ulp(v, ref[n], 1, f"{name} candidate {k} ({kname}) {n}")
+            else:
+                assert_bitexact(v, ref[n], f"{name} candidate {k} ({kname}) {n}")
+    assert len(seen) == nv, seen        # each candidate really ran its own kernel

@@ -30,7 +30,7 @@ def test_abi_symbols_match_header():
     out = subprocess.run(["nm", "-D", "--defined-only", pkg.LIB_PATH], capture_output=True, text=True).stdout
     exported = set(re.findall(r" T (fop_\w+)", out))
     assert exported == declared
-    assert pkg.abi_version() == 3
+    assert pkg.abi_version() == 4
 
 
 def test_library_has_no_hard_cuda_dependency():
