@@ -11,9 +11,14 @@ operators of BASELINE.json configs[1..3] back to back on every GPU
 Each launched through libfop's C ABI (fop_run) on torch's current stream.
 value = algorithmic bytes of all ranks / device time (max over ranks).
 
-Multi-GPU (torchrun, one process per GPU, NCCL): weak scaling — every rank
-runs the same per-GPU batch (the global batch is N x; N = 4 is
-BASELINE.json's cfg5 "4x the above batch").  cfg4b's reduced axis (rows) is
+Multi-GPU (torchrun, one process per GPU, NCCL).  --scaling weak (default):
+every rank runs the same per-GPU batch (the global batch is N x).  --scaling
+strong: BASELINE.json's cfg5 — the global batch is fixed at 4x the base and
+split over the N GPUs (at N = 1 one GPU holds the whole 4x tensors, the t1 of
+the scaling ratio); per-rank kernels shrink as N grows, so the exchange's
+latency shows.  At N > 1 the exchanged result is checked inside the bench
+(identical bits on every rank, reading R16's bound against a float64 sum
+over the ranks: config.exchange_check).  cfg4b's reduced axis (rows) is
 the sharded axis: its [1024] fp32 partial sums are combined across the GPUs
 INSIDE the column-reduction kernel (--exchange peer, default: each rank's
 kernel pushes its partials into every rank's exchange buffer over NVLink peer
@@ -21,6 +26,7 @@ memory and sums all ranks' contributions in rank order), or all-reduced over
 NCCL after it (--exchange nccl, the baseline).  Nothing else communicates.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl fop|reference] [--exchange peer|nccl]
+                  [--scaling weak|strong]
 """
 import argparse
 import json
@@ -43,12 +49,16 @@ OPS = [("cfg2", W.cfg2, "ew"), ("cfg3", W.cfg3, "transpose"), ("cfg4a", W.cfg4a,
 # global operator at `world` GPUs (batch loop scaled by world) and the loop it is sharded along
 GLOBAL = {"cfg2": (lambda w: W.cfg2(N=128 * w), "n"), "cfg3": (lambda w: W.cfg3(N=256 * w), "n"),
           "cfg4a": (lambda w: W.cfg4a(B=64 * w), "b"), "cfg4b": (lambda w: W.cfg4b(R=65536 * w), "r")}
+STRONG_SCALE = 4              # BASELINE.json configs[4]: "4x the above batch"
 FALLBACK_HBM = 6650.0
 L2_BYTES = 126 << 20          # B200 L2 (public figure), for the steady-state copies
 METRIC = "achieved HBM GB/s (fused-op suite; per-op GB/s and % of peak in config.per_op)"
 WORKLOAD = ("fused-op suite: cfg2 BN+ReLU+cast [128,64,112,112] f32->f16, cfg3 NCHW->NHWC*s "
             "[256,256,56,56] f16, cfg4a bias+GELU+row mean/var [64,512,768] f16, cfg4b colsum "
             "[65536,1024] f16->f32 (BASELINE.json configs[1..3]) per GPU")
+WORKLOAD_STRONG = ("cfg5 (BASELINE.json configs[4]): the fused-op suite at 4x the batch — cfg2 [512,64,112,112], "
+                   "cfg3 [1024,256,56,56], cfg4a [256,512,768], cfg4b [262144,1024] — fixed, split over the GPUs "
+                   "along the batch (rows for cfg4b, whose [1024] partial sums are combined across GPUs)")
 
 
 def peaks():
@@ -272,9 +282,13 @@ def run_fop(args):
     order = args.op_order.split(",")
     if sorted(order) != sorted(n for n, _, _ in OPS):
         raise SystemExit("--op-order must list cfg2,cfg3,cfg4a,cfg4b once each")
+    # weak: the global batch is world x the base batch (each rank runs configs[1..3] as is);
+    # strong: BASELINE.json's cfg5 — the global batch is fixed at 4x the base, split over the ranks
+    # (at N = 1 one GPU holds the whole 4x tensors: the t1 of the scaling ratio)
+    gscale = STRONG_SCALE if args.scaling == "strong" else world
     for name, mk, cls in sorted(OPS, key=lambda t: order.index(t[0])):
         gmk, loop = GLOBAL[name]
-        d, shard_info = shard_desc(gmk(world), loop, rank, world, fused=peer)   # == mk() per rank
+        d, shard_info = shard_desc(gmk(gscale), loop, rank, world, fused=peer)   # weak: == mk() per rank
         popts = {"peer_world": world, "peer_loop": loop} if peer and shard_info["partials"] else {}
         op = FusedOp(d, **({"max_vec_bytes": args.vec_bytes} if args.vec_bytes else {}),
                      **({"coalesce_order": args.order} if args.order else {}), **popts)
@@ -420,6 +434,39 @@ def run_fop(args):
     per_op = [float(v) for v in t[1:1 + len(ops)]]
     steady = [float(v) for v in t[1 + len(ops):]]
 
+    # ---- N > 1: parity of the exchanged reduction (cfg4b's column sums over the sharded rows).
+    # Every rank must hold identical bits, and they must equal the global column sum within
+    # reading R16's normwise bound; the reference is a float64 torch sum of each rank's shard,
+    # summed over ranks with the process group (a check of the plumbing, not the product path).
+    exchange_check = None
+    if world > 1:
+        exchange_check = {}
+        for o in ops:
+            parts = o["shard"].get("partials") or []
+            for tn, red in parts:
+                got = o["dev"][tn].float()
+                xs = [n for n, tt in o["desc"]["tensors"].items() if tt["role"] == "in"][0]
+                sp = o["desc"]["tensors"][xs]["shape"]
+                xv = o["dev"][xs].reshape(sp).double()
+                ref = xv.sum(0) if red == "sum" else xv.max(0).values
+                scale = xv.abs().sum(0)
+                cpu = dist.get_backend() == "gloo"       # FOP_BENCH_ONE_GPU plumbing
+                rr = torch.stack([ref, scale])
+                rr = rr.cpu() if cpu else rr
+                dist.all_reduce(rr, op=dist.ReduceOp.SUM if red == "sum" else dist.ReduceOp.MAX)
+                rr = rr.to(dev)
+                bits = got.view(torch.int32).to(torch.int64)
+                lo, hi = (bits.cpu() if cpu else bits.clone()), (bits.cpu() if cpu else bits.clone())
+                dist.all_reduce(lo, op=dist.ReduceOp.MIN)
+                dist.all_reduce(hi, op=dist.ReduceOp.MAX)
+                same = bool(torch.equal(lo, hi))
+                err = (got.double() - rr[0]).abs()
+                ok = same and bool((err <= 1e-5 * rr[1] + 1e-30).all())
+                exchange_check[f"{o['name']}.{tn}"] = {"identical_on_all_ranks": same, "within_R16": ok,
+                                                       "max_err_over_sum_abs": float((err / rr[1].clamp_min(1e-30)).max())}
+                if not ok:
+                    raise SystemExit(f"exchanged {o['name']}.{tn} failed its parity check: {exchange_check}")
+
     # ---- end to end through the C ABI with host buffers: fop_run_host_many
     # runs the suite's independent ops with the host<->device copies pipelined
     # (inputs in on one copy stream, outputs out on another, kernels in
@@ -507,11 +554,12 @@ def run_fop(args):
         line = {
             "metric": METRIC,
             "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+            "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {
-                "workload": WORKLOAD,
-                "global_batch_scale": world,
+                "workload": WORKLOAD if args.scaling == "weak" else WORKLOAD_STRONG,
+                "global_batch_scale": gscale,
+                "exchange_check": exchange_check,
                 "op_order": [o["name"] for o in ops],
                 "parallelism": ("dp%d (batch-sharded; " % world) + (
                     "no exchange)" if world == 1 else
@@ -572,6 +620,8 @@ def main():
                     help="order of the (independent) ops in a step")
     ap.add_argument("--no-graph", action="store_true", help="eager steps instead of replaying a CUDA graph")
     ap.add_argument("--no-steady", action="store_true", help="skip the per-op steady-state pass")
+    ap.add_argument("--scaling", choices=["weak", "strong"], default="weak",
+                    help="weak: configs[1..3] per GPU (global batch N x); strong: cfg5, 4x the batch split over N")
     ap.add_argument("--exchange", choices=["peer", "nccl"], default="peer",
                     help="N > 1: combine cfg4b's partial sums inside the kernel over NVLink (peer) or NCCL after it")
     args = ap.parse_args()

@@ -54,6 +54,9 @@ struct Out {
 // set per statement (see varies()): the statement's result is rounded to a
 // 16-bit type, so transcendental fast forms are within one ulp
 thread_local bool g_approx16 = false;
+// set with it: the statement's result is fp16 (the GELU's short ftz form is
+// exact enough down to fp16's subnormals; bf16/fp32 results take the wide form)
+thread_local bool g_out_f16 = false;
 // ... but only for nodes whose value reaches the output without an add or
 // subtract on the way: a ~2^-22 relative error ahead of a cancellation is no
 // longer within one 16-bit ulp (fuzz seed 21 case 294: -x2 / -1.5 + x0 + x1
@@ -63,8 +66,8 @@ bool fast_ok(const XNode& n) { return g_approx16 && n.no_addsub; }
 // C expression of a fused-DAG node given its operand expressions
 std::string op_expr(const XNode& n, const std::string& a, const std::string& b) {
   if (fast_ok(n)) {
-    if (n.op == FOP_OP_EXP) return "fop::exp_fast(" + a + ")";
-    if (n.op == FOP_OP_SIGMOID) return "fop::sigmoid_fast(" + a + ")";
+    if (n.op == FOP_OP_EXP) return std::string(g_out_f16 ? "fop::exp_fast(" : "fop::exp_fast_wide(") + a + ")";
+    if (n.op == FOP_OP_SIGMOID) return std::string(g_out_f16 ? "fop::sigmoid_fast(" : "fop::sigmoid_fast_wide(") + a + ")";
   }
   switch (n.op) {
     case FOP_OP_CONST: return fimm(n.imm);
@@ -82,7 +85,7 @@ std::string op_expr(const XNode& n, const std::string& a, const std::string& b) 
     case FOP_OP_LOG: return "logf(" + a + ")";
     case FOP_OP_TANH: return "tanhf(" + a + ")";
     case FOP_OP_SIGMOID: return "fop::op_sigmoid(" + a + ")";
-    case FOP_OP_GELU_TANH: return "fop::op_gelu_tanh(" + a + ")";
+    case FOP_OP_GELU_TANH: return std::string(g_out_f16 ? "fop::op_gelu_tanh(" : "fop::op_gelu_tanh_wide(") + a + ")";
     case FOP_OP_GELU_ERF: return "fop::op_gelu_erf(" + a + ")";
     case FOP_OP_CAST: return std::string("fop::round_to<") + dtn(n.cvt) + ">(" + a + ")";
   }
@@ -109,6 +112,7 @@ struct DagCtx {
 void decide_fast(const XStmt& x) {
   const char* e = std::getenv("FOP_APPROX16");
   g_approx16 = !(e && *e == '0') && x.kind == FOP_ASSIGN && esize(x.out_dtype) == 2 && x.out_dtype != FOP_I32;
+  g_out_f16 = x.kind == FOP_ASSIGN && x.out_dtype == FOP_F16;
   std::vector<bool> feeds(x.nodes.size(), false);   // value reaches an add/sub
   for (int i = (int)x.nodes.size() - 1; i >= 0; i--)
     for (size_t j = i + 1; j < x.nodes.size(); j++) {
@@ -209,7 +213,9 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
       case FOP_OP_ADD: e = "fop::add2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
       case FOP_OP_SUB: e = "fop::sub2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
       case FOP_OP_MUL: e = "fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + ")"; break;
-      case FOP_OP_GELU_TANH: e = "fop::op_gelu_tanh2(" + opnd(n.a) + ")"; break;
+      case FOP_OP_GELU_TANH:
+        e = std::string(g_out_f16 ? "fop::op_gelu_tanh2(" : "fop::op_gelu_tanh2_wide(") + opnd(n.a) + ")";
+        break;
       case FOP_OP_DIV:
         if (g_approx16 && !var[n.b]) {
           // ÷ loop-invariant d -> × r = RN(1/d), then one remainder step
@@ -276,6 +282,7 @@ void emit_elems(Out& o, const XStmt& x, const std::vector<bool>& var, const DagC
 
 std::string fin_expr(Out& o, const XStmt& x, const std::string& acc, const std::string& tag) {
   if (x.fin.empty()) return acc;
+  g_out_f16 = x.out_dtype == FOP_F16;   // (finalize nodes never take the fast forms: no_addsub unset)
   for (size_t i = 0; i < x.fin.size(); i++) {
     const XNode& n = x.fin[i];
     std::string nm = "f" + num(x.stmt) + "_" + num(i) + tag;
@@ -2391,6 +2398,7 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
     const char* e = std::getenv("FOP_PACKED");   // 0: scalar fp32 DAG evaluation (ablation)
     g_packed = !(e && *e == '0');
     g_approx16 = false;                           // set per statement by decide_fast()
+    g_out_f16 = false;
   }
   Gen g(p, L);
   // 32-bit index arithmetic when every offset and work index fits

@@ -466,6 +466,26 @@ __device__ __forceinline__ u64 op_gelu_tanh2(u64 v) {
 #endif
 }
 
+// GELU for bf16 and fp32 results: their range reaches down to 2^-133 / 2^-149,
+// where v / (1 + 2^a) overflows 2^a (a > 128) and the .ftz forms flush.  With
+// e = 2^-|a| <= 1 (never overflows; subnormal e kept by the non-ftz ex2):
+// 1 / (1 + 2^a) = (a > 0 ? e : 1) / (1 + e).  Same MUFU count; f16 results
+// (whose smallest subnormal is 2^-24) keep the shorter form above.
+__device__ __forceinline__ float ex2_approx_sub(float x) {
+  float r;
+  asm("ex2.approx.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float op_gelu_tanh_wide(float v) {
+  const float a = __fmul_rn(fmaf(v * v, FOP_GELU_C1, FOP_GELU_C2), v);
+  const float e = ex2_approx_sub(-fabsf(a));
+  const float r = rcp_approx(1.0f + e);
+  return __fmul_rn(v, a > 0.0f ? __fmul_rn(e, r) : r);
+}
+__device__ __forceinline__ u64 op_gelu_tanh2_wide(u64 v) {
+  return pk(op_gelu_tanh_wide(lo(v)), op_gelu_tanh_wide(hi(v)));
+}
+
 // value rounded to DT and back, for a pair; the packed conversion is the same
 // instruction the vector store issues, so the compiler computes it once
 template <int DT>
@@ -497,6 +517,14 @@ __device__ __forceinline__ float op_sigmoid(float v) { return __frcp_rn(1.0f + e
 __device__ __forceinline__ float exp_fast(float x) { return ex2_approx(x * 1.4426950408889634f); }
 __device__ __forceinline__ float sigmoid_fast(float x) {
   return rcp_approx(1.0f + ex2_approx(x * -1.4426950408889634f));
+}
+// bf16 results reach down to 2^-133: no flush to zero, no 2^|x| overflow
+// (the GELU wide form's identity 1 / (1 + e^-x) = (x < 0 ? e : 1) / (1 + e), e = e^-|x|)
+__device__ __forceinline__ float exp_fast_wide(float x) { return ex2_approx_sub(x * 1.4426950408889634f); }
+__device__ __forceinline__ float sigmoid_fast_wide(float x) {
+  const float e = ex2_approx_sub(fabsf(x) * -1.4426950408889634f);
+  const float r = rcp_approx(1.0f + e);
+  return x < 0.0f ? e * r : r;
 }
 
 // ------------------------------------------------------------------ reductions

@@ -154,6 +154,10 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       v.push_back({{"FOP_EW_U", 2}, {"FOP_EW_MINB", 4}});
       v.push_back({{"FOP_EW_U", 1}, {"FOP_EW_MINB", 8}});
       v.push_back({{"FOP_EW_U", 4}, {"FOP_EW_MINB", 3}});
+      // 32-byte vectors (LDG/STG.256), 8 warps per SM with 4 vectors in flight each:
+      // cfg2 6112 -> 6525 GB/s (profiles/r02/sweep_r02_vec32.log)
+      v.push_back({{"FOP_VEC_BYTES", 32}, {"FOP_EW_U", 4}, {"FOP_EW_MINB", 1}});
+      v.push_back({{"FOP_VEC_BYTES", 32}, {"FOP_EW_U", 4}, {"FOP_EW_MINB", 2}, {"FOP_BLOCK", 128}});
       break;
     case FOP_CLASS_TRANSPOSE:
       if (L.tma) break;
@@ -166,6 +170,8 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 2}});
       v.push_back({{"FOP_TR_U", 2}, {"FOP_TR_MINB", 2}});
       v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 3}});
+      // 32-byte stores along d_v over 16-byte loads along d_r (cfg3 5986 -> 6028 GB/s)
+      v.push_back({{"FOP_VEC_BYTES", 32}, {"FOP_TR_WR_BYTES", 16}, {"FOP_TR_U", 1}, {"FOP_TR_MINB", 1}});
       break;
     case FOP_CLASS_ROW_REDUCE:
       if (L.row_g > 1) {   // few long rows: neighbouring warps-per-row counts
@@ -200,7 +206,11 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   const fop_plan_opts& o = p.opts;
   auto acc = all_accesses(L);
   int sms = o.sm_count > 0 ? o.sm_count : 148;
-  int vmax = o.max_vec_bytes >= 32 ? 32 : 16;
+  // vector bytes: the planner option, or a tuning candidate's FOP_VEC_BYTES
+  // (LDG/STG.256 stores measured +3-7 % on copies, profiles/r02/bw_probe2_r02.log)
+  int vbytes = geometry_knob(L, "FOP_VEC_BYTES", o.max_vec_bytes);
+  if (vbytes != 4 && vbytes != 8 && vbytes != 16 && vbytes != 32) vbytes = o.max_vec_bytes;
+  int vmax = vbytes >= 32 ? 32 : 16;
 
   // ---- loop order + collapse
   L.kl.clear();
@@ -279,7 +289,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       min_es = std::min(min_es, esize(d.t[a->tensor].dtype));
       any_vec = true;
     }
-  int W = any_vec ? std::max(1, o.max_vec_bytes / min_es) : 1;
+  int W = any_vec ? std::max(1, vbytes / min_es) : 1;
   if (o.force_width > 0) W = std::min(W, pow2_floor(o.force_width));
   if (L.scalar_variant || L.force_w1) W = 1;
   if (!L.seq.empty() && any_vec) {
@@ -327,7 +337,9 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
 
   if (L.kclass == FOP_CLASS_TRANSPOSE) {
     const Affine& t = L.loads[L.trans_load];
-    int wr = std::max(1, o.max_vec_bytes / esize(d.t[t.tensor].dtype));
+    // read-side vector bytes: the store side's by default; FOP_TR_WR_BYTES sets them
+    // apart (32 B loads along d_r under 16 B stores along d_v: an 8 x 16 tile of 16-bit data)
+    int wr = std::max(1, std::min<int>(32, geometry_knob(L, "FOP_TR_WR_BYTES", vbytes)) / esize(d.t[t.tensor].dtype));
     if (o.force_width > 0) wr = std::min(wr, pow2_floor(o.force_width));
     if (L.scalar_variant) wr = 1;
     while (wr > 1 && L.kl[1].extent % wr) wr /= 2;
@@ -406,20 +418,23 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   }
 
   // ---- a4: per-access chunks
-  auto vec_cb = [&](const Affine& a, int vk, int w) {
+  // loads may move wider chunks than the stores (FOP_LD_BYTES=32: LDG.256 under
+  // STG.128, the copy pattern measured fastest at 0.4-1 GB, profiles/r02/bw_probe3_r02.log)
+  const int vmax_ld = geometry_knob(L, "FOP_LD_BYTES", vmax) >= 32 ? 32 : vmax;
+  auto vec_cb = [&](const Affine& a, int vk, int w, int cap) {
     int es = esize(d.t[a.tensor].dtype);
-    return chunk_bytes(p, L, a, vk, std::min(vmax, w * es));
+    return chunk_bytes(p, L, a, vk, std::min(cap, w * es));
   };
   L.load_cb.assign(L.loads.size(), 0);
   L.load_cb_r.assign(L.loads.size(), 0);
   for (size_t k = 0; k < L.loads.size(); k++) {
-    if (coef(L, L.loads[k], 0) == 1) L.load_cb[k] = vec_cb(L.loads[k], 0, W);
+    if (coef(L, L.loads[k], 0) == 1) L.load_cb[k] = vec_cb(L.loads[k], 0, W, vmax_ld);
     if (L.kclass == FOP_CLASS_TRANSPOSE && coef(L, L.loads[k], 0) != 1 && coef(L, L.loads[k], 1) == 1)
-      L.load_cb_r[k] = vec_cb(L.loads[k], 1, L.read_width);
+      L.load_cb_r[k] = vec_cb(L.loads[k], 1, L.read_width, 32);
   }
   L.store_cb.assign(L.stmts.size(), 0);
   for (size_t k = 0; k < L.stmts.size(); k++)
-    if (coef(L, L.stmts[k].write, 0) == 1) L.store_cb[k] = vec_cb(L.stmts[k].write, 0, W);
+    if (coef(L, L.stmts[k].write, 0) == 1) L.store_cb[k] = vec_cb(L.stmts[k].write, 0, W, vmax);
   if (L.row_peel) {   // alignment comes from the per-row shift, not from the static coefficients
     for (size_t k = 0; k < L.loads.size(); k++) {
       if (coef(L, L.loads[k], 0) != 1) continue;
@@ -636,7 +651,9 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.row_hoist = knob("FOP_ROW_HOIST", 1);
     int64_t gpb = L.block * P / (32 * G);   // rows per block
     int64_t need = (rows + gpb - 1) / gpb;
-    L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
+    // one resident wave walking the rows (default), or FOP_ROW_ONEPASS=1: a block per
+    // group of rows, the hardware block scheduler balancing the SMs as blocks retire
+    L.grid = std::max<int64_t>(1, knob("FOP_ROW_ONEPASS", 0) ? need : std::min<int64_t>(need, (int64_t)sms * L.minblocks));
     if (Q > 1)   // whole clusters, one row each per pass
       L.grid = std::max<int64_t>(1, std::min<int64_t>({rows, (int64_t)sms * L.minblocks / Q,
                                                        (int64_t)knob("FOP_ROW_CLUSTERS", 1 << 30)})) * Q;

@@ -123,3 +123,23 @@ def assert_normwise(got, ref, scale, tol, name=""):
     assert bad.size == 0, f"{name}: {bad.size} exceed tol*sum|t| (worst ratio " \
                           f"{(err / bound).max():.3g}) first {bad[:5]}"
     return float((err / np.maximum(scale, 1e-30)).max(initial=0))
+
+
+def check_rowstats(d, x, got, ulp_y=1):
+    """cfg4a-shaped operators (y = f16(gelu(x + b)), mean/var over y): y within
+    `ulp_y` of the oracle; the statistics against the oracle run on the GPU's
+    OWN y (isolates the reduction from y's last-bit rounding: R16's 1e-5
+    normwise bound) and end to end against the oracle (2e-3 for fp16 data)."""
+    import copy
+    from oracle import oracle as O
+    ref = O.run(d, x)
+    assert_ulp(got["y"], ref["y"], ulp_y, "y")
+    d2 = copy.deepcopy(d)
+    d2["tensors"]["y"]["role"] = "in"
+    xin = dict(x)
+    xin["y"] = got["y"]
+    ref2 = O.run(d2, xin, stmts=[1, 2])
+    for si, name in [(1, "mean"), (2, "var")]:
+        scale = O.run(abs_terms_desc(d2, si), xin, stmts=[1, 2])[name]
+        assert_normwise(got[name], ref2[name], scale, 1e-5, name)
+        assert_normwise(got[name], ref[name], O.run(abs_terms_desc(d, si), x)[name], 2e-3, name)

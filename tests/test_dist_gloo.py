@@ -111,3 +111,25 @@ def test_shard_desc_rules():
     assert info["partials"] == [] and sh["tensors"]["mean"]["shape"] == [2, 6]
     with pytest.raises(ShardError):
         shard_desc(W.cfg2(3, 8, 6, 10), "n", 0, 2)   # 3 not divisible by 2
+
+
+@pytest.mark.parametrize("world", [1, 2, 4, 8])
+def test_strong_scaling_shards_tile_cfg5(world):
+    """bench.py --scaling strong: BASELINE.json's cfg5 (4x the batch of configs[1..3]) split over
+    N ranks — the shards' batch blocks are disjoint, cover the global operator, carry equal
+    algorithmic bytes, and only cfg4b (rows = its reduced axis) produces partials."""
+    import bench
+    for name, (gmk, loop) in bench.GLOBAL.items():
+        g = gmk(bench.STRONG_SCALE)
+        E = g["loops"][loop]
+        blocks, nbytes = [], set()
+        for r in range(world):
+            sh, info = shard_desc(g, loop, r, world, fused=True)
+            assert sh["loops"][loop] == E // world
+            blocks += [info["slices"][n][1:] for n in info["slices"]][:1]
+            nbytes.add(W.algorithmic_bytes(sh))
+            assert [p[0] for p in info["partials"]] == (["out"] if name == "cfg4b" else [])
+        assert sorted(blocks) == [(r * E // world, (r + 1) * E // world) for r in range(world)]
+        assert len(nbytes) == 1
+        if world == 1:
+            assert nbytes.pop() == W.algorithmic_bytes(g)

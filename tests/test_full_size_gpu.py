@@ -5,10 +5,9 @@ output (not sampled slices).
 
 Schedules are semantics preserving (§IV-A1): whichever
 geometry the tuner picks must give the oracle's result — bit-exact for the
-ASSIGN outputs (cfg2, cfg3, cfg4a's y), the reading-R16 normwise bound for the
-reductions (cfg4a's mean/var, cfg4b's column sums), and identical bits for
-every candidate of one plan on the same inputs where the association order is
-the same.
+ASSIGN outputs of cfg2 and cfg3, <= 1 fp16 ulp for cfg4a's y (GELU), the
+reading-R16 normwise bound for the reductions (cfg4a's mean/var against the
+oracle run on the kernel's own y, and end to end; cfg4b's column sums).
 """
 import numpy as np
 import pytest
@@ -17,7 +16,7 @@ import torch
 import workloads as W
 from oracle import oracle as O
 
-from harness import abs_terms_desc, assert_bitexact, assert_normwise, assert_ulp, device_tensors, to_host
+from harness import abs_terms_desc, assert_bitexact, assert_normwise, check_rowstats, device_tensors, to_host
 
 pytestmark = [pytest.mark.gpu, pytest.mark.full_size]
 
@@ -50,20 +49,19 @@ def test_every_tuning_candidate_full_size_whole_output(name):
     x = W.make_inputs(d)
     ref = O.run(d, x)
     scale = {}
-    if name == "cfg4a":
-        scale = {"mean": O.run(abs_terms_desc(d, 1), x)["mean"], "var": O.run(abs_terms_desc(d, 2), x)["var"]}
-    elif name == "cfg4b":
+    if name == "cfg4b":
         scale = {"out": O.run(abs_terms_desc(d, 0), x)["out"]}
     dev_in = device_tensors({**d, "tensors": {n: t for n, t in d["tensors"].items() if t["role"] == "in"}}, x)
     seen = set()
     for k in range(nv):
         got, kname = _run_variant(d, dev_in, k)
         seen.add(kname)
+        if name == "cfg4a":
+            check_rowstats(d, x, got)
+            continue
         for n, v in got.items():
             if n in scale:
                 assert_normwise(v, ref[n], scale[n], 1e-5, f"{name} candidate {k} ({kname}) {n}")
-            elif name == "cfg4a":
-                assert_ulp(v, ref[n], 1, f"{name} candidate {k} ({kname}) {n}")
             else:
                 assert_bitexact(v, ref[n], f"{name} candidate {k} ({kname}) {n}")
     assert len(seen) == nv, seen        # each candidate really ran its own kernel

@@ -7,7 +7,8 @@ Tolerances, each derived from the arithmetic, not measured:
   * fp32 outputs: the CUDA math library's documented maximum error plus one ulp
     for the oracle's own rounding of its double result (reading R12):
     expf 2, logf 1, tanhf 2 ulp; sigmoid = 1/(1 + expf(-v)) 2 + 1 + 1; GELU-erf
-    = v * normcdff(v), normcdff 5 ulp, + 1 for the product.  GELU-tanh keeps its
+    = v * normcdff(v), normcdff 5 ulp, + 1 for the product (below v = -13.2
+    normcdff's result is subnormal: 4 |v| 2^-149 absolute).  GELU-tanh keeps its
     MUFU form for fp32 outputs too: relative error <= (12 + 3|a|) u with
     a = v (C2 + C1 v^2) the log2-domain argument (ex2.approx 2^-22, rcp.approx,
     three roundings, and the fp32 rounding of a amplified by ln2 |a|), plus
@@ -21,7 +22,7 @@ import torch
 
 from oracle import oracle as O
 
-from harness import assert_bitexact, assert_ulp, assert_normwise, abs_terms_desc, run_gpu, ordered32
+from harness import assert_bitexact, assert_ulp, check_rowstats, ordered32, run_gpu
 
 pytestmark = pytest.mark.gpu
 
@@ -74,6 +75,15 @@ def test_transcendental_sweep_and_special_values(op, out_dtype):
             assert np.array_equal(g[~fin & ~np.isnan(r)], r[~fin & ~np.isnan(r)])
             tol = (12 + 3 * a[fin]) * 2.0 ** -24 * np.abs(r[fin]) + 16 * 2.0 ** -126   # MUFU forms flush subnormals
             assert np.all(np.abs(g[fin] - r[fin]) <= tol), np.max(np.abs(g[fin] - r[fin]) / tol)
+        elif op == "gelu_erf":
+            # v * normcdff(v): where Phi(v) < 2^-126 (v < -13.2) normcdff returns a subnormal, whose
+            # absolute error (a few units of 2^-149) the product scales by |v|
+            g, r = got["out"], ref
+            d = np.abs(ordered32(g) - ordered32(r))
+            nan = np.isnan(g) & np.isnan(r)
+            sub = np.abs(g.astype(np.float64) - r.astype(np.float64)) <= 4 * np.abs(x.astype(np.float64)) * 2.0 ** -149
+            bad = ~nan & (d > F32_ULP[op]) & ~sub
+            assert not bad.any(), (x[bad][:4], g[bad][:4], r[bad][:4])
         else:
             assert_ulp(got["out"], ref, F32_ULP[op], f"{op} {in_dtype}->f32")
 
@@ -109,10 +119,7 @@ def test_cfg4a_gelu_special_values_through_the_row_kernel():
     x["bias"][:] = 0
     got, op = run_gpu(d, x)
     assert op.info()["launches"][0]["class"] == "row_reduce"
-    ref = O.run(d, x)
-    assert_ulp(got["y"], ref["y"], 1, "y")
-    for si, n in ((1, "mean"), (2, "var")):
-        assert_normwise(got[n], ref[n], O.run(abs_terms_desc(d, si), x)[n], 1e-5, n)
+    check_rowstats(d, x, got)
 
 
 # ---------------------------------------------------------------- division
