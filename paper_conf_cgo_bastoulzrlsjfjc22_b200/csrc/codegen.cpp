@@ -57,6 +57,9 @@ thread_local bool g_approx16 = false;
 // set with it: the statement's result is fp16 (the GELU's short ftz form is
 // exact enough down to fp16's subnormals; bf16/fp32 results take the wide form)
 thread_local bool g_out_f16 = false;
+// the statement is an integer statement (its target is i32, reading R30):
+// int32 bits in the fp32 registers, integer node forms, no packed fp32x2 path
+thread_local bool g_int = false;
 // ... but only for nodes whose value reaches the output without an add or
 // subtract on the way: a ~2^-22 relative error ahead of a cancellation is no
 // longer within one 16-bit ulp (fuzz seed 21 case 294: -x2 / -1.5 + x0 + x1
@@ -65,6 +68,20 @@ bool fast_ok(const XNode& n) { return g_approx16 && n.no_addsub; }
 
 // C expression of a fused-DAG node given its operand expressions
 std::string op_expr(const XNode& n, const std::string& a, const std::string& b) {
+  if (g_int) {
+    switch (n.op) {
+      case FOP_OP_CONST: return "__int_as_float(" + std::to_string((long long)n.imm) + ")";
+      case FOP_OP_ADD: return "fop::iadd(" + a + ", " + b + ")";
+      case FOP_OP_SUB: return "fop::isub(" + a + ", " + b + ")";
+      case FOP_OP_MUL: return "fop::imul(" + a + ", " + b + ")";
+      case FOP_OP_MAX: return "fop::imax(" + a + ", " + b + ")";
+      case FOP_OP_MIN: return "fop::imin(" + a + ", " + b + ")";
+      case FOP_OP_NEG: return "fop::ineg(" + a + ")";
+      case FOP_OP_ABS: return "fop::iabs(" + a + ")";
+      case FOP_OP_RELU: return "fop::irelu(" + a + ")";
+    }
+    return "__int_as_float(0)";   // (validate() admits no other node in an integer statement)
+  }
   if (fast_ok(n)) {
     if (n.op == FOP_OP_EXP) return std::string(g_out_f16 ? "fop::exp_fast(" : "fop::exp_fast_wide(") + a + ")";
     if (n.op == FOP_OP_SIGMOID) return std::string(g_out_f16 ? "fop::sigmoid_fast(" : "fop::sigmoid_fast_wide(") + a + ")";
@@ -113,6 +130,7 @@ void decide_fast(const XStmt& x) {
   const char* e = std::getenv("FOP_APPROX16");
   g_approx16 = !(e && *e == '0') && x.kind == FOP_ASSIGN && esize(x.out_dtype) == 2 && x.out_dtype != FOP_I32;
   g_out_f16 = x.kind == FOP_ASSIGN && x.out_dtype == FOP_F16;
+  g_int = x.out_dtype == FOP_I32;
   std::vector<bool> feeds(x.nodes.size(), false);   // value reaches an add/sub
   for (int i = (int)x.nodes.size() - 1; i >= 0; i--)
     for (size_t j = i + 1; j < x.nodes.size(); j++) {
@@ -251,7 +269,7 @@ struct Sink {
 };
 thread_local bool g_packed = true;
 void emit_elems(Out& o, const XStmt& x, const std::vector<bool>& var, const DagCtx& c, int W, const Sink& s) {
-  bool packed = g_packed && W % 2 == 0 && s.pair;
+  bool packed = g_packed && W % 2 == 0 && s.pair && !g_int;
   if (!packed) {
     o.l("#pragma unroll");
     o.l("for (int " + c.ev + " = 0; " + c.ev + " < " + num(W) + "; ++" + c.ev + ") {");
@@ -283,6 +301,7 @@ void emit_elems(Out& o, const XStmt& x, const std::vector<bool>& var, const DagC
 std::string fin_expr(Out& o, const XStmt& x, const std::string& acc, const std::string& tag) {
   if (x.fin.empty()) return acc;
   g_out_f16 = x.out_dtype == FOP_F16;   // (finalize nodes never take the fast forms: no_addsub unset)
+  g_int = x.out_dtype == FOP_I32;
   for (size_t i = 0; i < x.fin.size(); i++) {
     const XNode& n = x.fin[i];
     std::string nm = "f" + num(x.stmt) + "_" + num(i) + tag;
@@ -2399,6 +2418,7 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
     g_packed = !(e && *e == '0');
     g_approx16 = false;                           // set per statement by decide_fast()
     g_out_f16 = false;
+    g_int = false;
   }
   Gen g(p, L);
   // 32-bit index arithmetic when every offset and work index fits

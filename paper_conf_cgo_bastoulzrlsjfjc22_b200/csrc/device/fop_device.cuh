@@ -428,6 +428,20 @@ __device__ __forceinline__ u64 div2_by(u64 a, float d) {
   return pk(div_by_fix(lo(q), lo(q0), lo(a), d), div_by_fix(hi(q), hi(q0), hi(a), d));
 }
 
+// ------------------------------------------------------------------ int32 (reading R30)
+// Integer statements keep int32 values as raw bits in the same 32-bit
+// registers the fp32 DAG uses (loads/stores of I32 move raw bits); their
+// nodes operate on those bits with two's-complement wrap-around (unsigned
+// arithmetic modulo 2^32 — no signed-overflow UB in the C++ source).
+__device__ __forceinline__ float iadd(float a, float b) { return __uint_as_float(__float_as_uint(a) + __float_as_uint(b)); }
+__device__ __forceinline__ float isub(float a, float b) { return __uint_as_float(__float_as_uint(a) - __float_as_uint(b)); }
+__device__ __forceinline__ float imul(float a, float b) { return __uint_as_float(__float_as_uint(a) * __float_as_uint(b)); }
+__device__ __forceinline__ float imax(float a, float b) { return __int_as_float(max(__float_as_int(a), __float_as_int(b))); }
+__device__ __forceinline__ float imin(float a, float b) { return __int_as_float(min(__float_as_int(a), __float_as_int(b))); }
+__device__ __forceinline__ float ineg(float a) { return __uint_as_float(0u - __float_as_uint(a)); }
+__device__ __forceinline__ float iabs(float a) { return __float_as_int(a) < 0 ? ineg(a) : a; }
+__device__ __forceinline__ float irelu(float a) { return __float_as_int(a) > 0 ? a : __int_as_float(0); }
+
 // GELU, tanh form: 0.5 v (1 + tanh u) == v * sigmoid(2u) = v / (1 + 2^(v * (C2 + C1 v^2)))
 // with u = sqrt(2/pi)(v + 0.044715 v^3), C2 = -2 sqrt(2/pi) log2(e), C1 = 0.044715 C2.
 // MUFU.EX2 + MUFU.RCP: relative error ~1e-6, far inside one fp16/bf16 ulp

@@ -638,6 +638,10 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     int P = 1;
     if (G == 1 && Q == 1 && !split && !L.row_peel && knob("FOP_ROW_P", 1))
       while (P < 32 && 32 / (2 * P) >= nvd) P *= 2;
+    // FOP_ROW_PFORCE: P rows per warp regardless (e.g. 2 rows of 48 32-byte vectors
+    // over 16 lanes each: 32-byte accesses without a ragged lane count)
+    if (G == 1 && Q == 1 && !split && !L.row_peel && knob("FOP_ROW_PFORCE", 0) > 1)
+      P = std::min(32, pow2_floor(knob("FOP_ROW_PFORCE", 0)));
     L.row_g = G;
     L.row_q = Q;
     L.row_p = P;

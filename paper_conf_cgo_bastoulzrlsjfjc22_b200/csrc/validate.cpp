@@ -164,7 +164,6 @@ void validate(const fop_desc& d) {
       for (int a = 1; a < st.nacc; a++)
         if (st.acc[a].tensor == st.acc[0].tensor && !affine_of(d, st.acc[a]).same(w))
           fail(FOP_E_UNSUPPORTED, where(s) + "read-modify-write statement reads its target at another index");
-      if (wt.dtype == FOP_I32) fail(FOP_E_UNSUPPORTED, where(s) + "i32 read-modify-write");
     }
     if (st.kind == FOP_ASSIGN && injective) {
       // A read of the target at another index makes the statement a
@@ -181,13 +180,39 @@ void validate(const fop_desc& d) {
     if (st.kind == FOP_REDUCE && !has_red)
       fail(FOP_E_UNSUPPORTED, where(s) + "REDUCE statement without a reduction loop (use ASSIGN)");
 
-    // i32: pure element moves only (bit-exact copies/transposes)
-    bool any_i32 = wt.dtype == FOP_I32;
-    for (int a = 1; a < st.nacc; a++) any_i32 |= d.t[st.acc[a].tensor].dtype == FOP_I32;
-    if (any_i32) {
-      bool move = st.kind == FOP_ASSIGN && st.nnodes == 1 && st.node[0].op == FOP_OP_LOAD &&
-                  d.t[st.acc[st.node[0].a].tensor].dtype == wt.dtype;
-      if (!move) fail(FOP_E_UNSUPPORTED, where(s) + "i32 tensors are supported for pure moves only");
+    // Element types (reading R30).  A pure element move copies any
+    // type.  A statement writing an i32 tensor is an INTEGER statement: it reads
+    // i32 tensors only and its DAG is + - * max min neg abs relu and integral
+    // constants on int32 values, wrapping modulo 2^32 (two's complement).  Any
+    // other statement is a float statement and reads no i32 tensor.
+    const bool move = st.kind == FOP_ASSIGN && st.nnodes == 1 && st.node[0].op == FOP_OP_LOAD &&
+                      d.t[st.acc[st.node[0].a].tensor].dtype == wt.dtype;
+    if (!move) {
+      const bool integer = wt.dtype == FOP_I32;
+      for (int a = 1; a < st.nacc; a++)
+        if ((d.t[st.acc[a].tensor].dtype == FOP_I32) != integer)
+          fail(FOP_E_INVALID, where(s) + (integer ? "integer statement reads a float tensor"
+                                                   : "float statement reads an i32 tensor"));
+      auto int_ok = [](const fop_node& q) {
+        switch (q.op) {
+          case FOP_OP_LOAD: case FOP_OP_ACC: case FOP_OP_ADD: case FOP_OP_SUB: case FOP_OP_MUL:
+          case FOP_OP_MAX: case FOP_OP_MIN: case FOP_OP_NEG: case FOP_OP_ABS: case FOP_OP_RELU: return true;
+          case FOP_OP_CONST: return q.imm == std::floor(q.imm) && q.imm >= -2147483648.0f && q.imm < 2147483648.0f;
+        }
+        return false;
+      };
+      for (int i = 0; i < st.nnodes; i++) {
+        if (integer && !int_ok(st.node[i])) fail(FOP_E_INVALID, where(s) + "operation not defined on i32");
+        if (!integer && st.node[i].op == FOP_OP_CAST && st.node[i].cvt == FOP_I32)
+          fail(FOP_E_INVALID, where(s) + "cast to i32");
+      }
+      for (int i = 0; st.kind == FOP_REDUCE && i < st.nfin; i++) {
+        if (integer && !int_ok(st.fin[i])) fail(FOP_E_INVALID, where(s) + "operation not defined on i32");
+        if (!integer && st.fin[i].op == FOP_OP_CAST && st.fin[i].cvt == FOP_I32)
+          fail(FOP_E_INVALID, where(s) + "cast to i32");
+      }
+      if (integer && st.kind == FOP_REDUCE)
+        fail(FOP_E_UNSUPPORTED, where(s) + "i32 reductions (the oracle defines them; the kernels do not yet)");
     }
   }
 }

@@ -9,6 +9,7 @@ import re
 import subprocess
 import tempfile
 
+import numpy as np
 import pytest
 
 import workloads as W
@@ -351,3 +352,48 @@ def test_fast_forms_not_ahead_of_add_or_subtract():
     e_direct = FusedOp(op([("load", 0), ("exp", 0)]), jit=0, autotune=0).source()
     e_summed = FusedOp(op([("load", 0), ("exp", 0), ("load", 1), ("add", 1, 2)]), jit=0, autotune=0).source()
     assert "fop::exp_fast(" in e_direct and "fop::exp_fast(" not in e_summed
+
+
+def _int_desc(expr, out="i32", xin="i32", kind="assign", write_idx=("i",)):
+    t = lambda dt, role, shape=(64,): {"shape": list(shape), "dtype": dt, "role": role, "init": None, "strides": None}  # noqa: E731
+    return {"name": "i", "loops": {"i": 64, "k": 4},
+            "tensors": {"a": t(xin, "in", (64, 4)), "out": t(out, "out")},
+            "stmts": [{"kind": kind, "op": "sum", "loops": ["i", "k"] if kind == "reduce" else ["i"],
+                       "write": ("out", list(write_idx)),
+                       "reads": [("a", ["i", "k"] if kind == "reduce" else ["i", 0])], "expr": expr}]}
+
+
+@pytest.mark.parametrize("desc,status", [
+    (_int_desc([("load", 0), ("const", 3.0), ("mul", 0, 1), ("neg", 2), ("abs", 3), ("relu", 4)]), None),
+    (_int_desc([("load", 0), ("const", 2.0), ("div", 0, 1)]), "FOP_E_INVALID"),          # / not defined on i32
+    (_int_desc([("load", 0), ("exp", 0)]), "FOP_E_INVALID"),
+    (_int_desc([("load", 0), ("const", 0.5), ("add", 0, 1)]), "FOP_E_INVALID"),          # non-integral constant
+    (_int_desc([("load", 0), ("const", 1.0), ("add", 0, 1)], out="f32"), "FOP_E_INVALID"),  # float stmt reads i32
+    (_int_desc([("load", 0), ("const", 1.0), ("add", 0, 1)], xin="f32"), "FOP_E_INVALID"),  # int stmt reads f32
+    (_int_desc([("load", 0)], out="f32"), "FOP_E_INVALID"),                              # not a move: a conversion
+    (_int_desc([("load", 0)]), None),                                                     # pure i32 move
+    (_int_desc([("load", 0)], kind="reduce"), "FOP_E_UNSUPPORTED"),                       # oracle-only for now
+])
+def test_integer_statement_rules_match_the_oracle(desc, status):
+    """Reading R30: the product accepts exactly the integer statements the oracle defines
+    (tests/test_oracle_ops.py), except i32 reductions, which it reports unsupported."""
+    from oracle import oracle as O
+    x = {"a": np.arange(256, dtype=np.float32 if desc["tensors"]["a"]["dtype"] == "f32" else np.int32)}
+    if status is None:
+        FusedOp(desc, jit=0)
+        O.run(desc, x)
+        return
+    with pytest.raises(FopError) as e:
+        FusedOp(desc, jit=0)
+    assert e.value.status == status
+    if status == "FOP_E_INVALID":
+        with pytest.raises(ValueError):
+            O.run(desc, x)
+
+
+def test_integer_kernels_compile_for_sm100a():
+    d = _int_desc([("load", 0), ("const", 3.0), ("mul", 0, 1), ("const", -7.0), ("max", 2, 3)])
+    op = FusedOp(d)
+    src = op.source()
+    assert "fop::imul(" in src and "fop::imax(" in src and "fop::mul2" not in src
+    assert "IMAD" in _sass(op.cubin(0)) or "IMUL" in _sass(op.cubin(0))
