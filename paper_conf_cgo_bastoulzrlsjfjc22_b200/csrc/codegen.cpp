@@ -2337,6 +2337,104 @@ struct Gen {
     if (NCH == 1) {
       exchange();
       final_store();
+    } else if (L.col_fin) {
+      // Flag-word finalize (FOP_COL_FIN=1/2, ablations; 0 = the default below):
+      // chunk blocks store their SW slab sums as 64-bit words (1 << 32 | fp32
+      // bits) — one single-copy-atomic store carries the value and its arrival,
+      // so no fence orders it — and ONE block per slab polls the words, adds
+      // them in chunk order (deterministic) and clears them (the workspace is
+      // zero again for the next run).  1: the slab's last chunk block (the last
+      // dispatched) is that block, no atomic at all; 2: the last block to
+      // arrive at a relaxed arrival counter (no fence before it).  Measured on
+      // cfg4b: 27.2 us (1) vs 25.3 us for the fence + counter scheme — the
+      // designated block is not the last to finish, so its poll loop sits on
+      // the critical path (profiles/r02/sweep_r02_colfin.log).
+      const int FM = L.col_fin;
+      const std::string OWN = FM == 1 ? "c == " + num(NCH - 1) + "u" : "false";
+      o.l("u64* partw = (u64*)(args.ws + " + num((int64_t)L.ws_off) + "ull);");
+      o.l(std::string("if (rl == 0u") + (FM == 1 ? " && chunk != " + num(NCH - 1) + "u" : "") + ") {");
+      o.l("  #pragma unroll");
+      o.l("  for (int e = 0; e < " + num(W) + "; ++e) fop::st_relaxed_gpu_u64(&partw[(chunk * " + num(slabs) +
+          "u + slab) * " + num(SW) + "u + cv * " + num(W) + "u + e], (1ull << 32) | __float_as_uint(red[cv * " + num(W) +
+          "u + e]));");
+      o.l("}");
+      if (FM == 2) {
+        size_t words = ((size_t)NCH * (size_t)slabs * (size_t)SW * 8 + 255) & ~size_t(255);
+        o.l("unsigned* cnt = (unsigned*)(args.ws + " + num((int64_t)(L.ws_off + words)) + "ull);");
+        o.l("__syncthreads();");
+        o.l("if (tid == 0u) last_flag = (atomicAdd(&cnt[slab], 1u) == " + num(NCH - 1) + "u);");
+        o.l("__syncthreads();");
+        o.l("if (last_flag) {");
+      } else {
+        o.l("if (chunk == " + num(NCH - 1) + "u) {");
+      }
+      o.ind++;
+      o.l("#pragma unroll");
+      o.l("for (int e = 0; e < " + num(W) + "; ++e) acc[e] = " + init + ";");
+      const int64_t MAXIT = (NCH + L.gr - 1) / L.gr;
+      const std::string NW_ = FM == 1 ? num(NCH - 1) : num(NCH);   // chunks whose words are read
+      // every word this thread combines is requested before the first is
+      // checked (one round trip); missing ones are re-polled as a batch
+      o.l("u64 pw_[" + num(MAXIT) + "][" + num(W) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int it = 0; it < " + num(MAXIT) + "; ++it) {");
+      o.l("  const idx_t c = rl + it * " + num(L.gr) + "u;");
+      o.l("  #pragma unroll");
+      o.l("  for (int e = 0; e < " + num(W) + "; ++e) pw_[it][e] = c < " + NW_ +
+          "u ? fop::ld_relaxed_gpu_u64(&partw[(c * " + num(slabs) + "u + slab) * " + num(SW) + "u + cv * " + num(W) +
+          "u + e]) : 0ull;");
+      o.l("}");
+      o.l("unsigned long long t0_ = 0;");
+      o.l("for (unsigned ns_ = 32u;;) {");
+      o.l("  bool all_ = true;");
+      o.l("  #pragma unroll");
+      o.l("  for (int it = 0; it < " + num(MAXIT) + "; ++it)");
+      o.l("    #pragma unroll");
+      o.l("    for (int e = 0; e < " + num(W) + "; ++e) all_ &= rl + it * " + num(L.gr) + "u >= " + NW_ +
+          "u || (unsigned)(pw_[it][e] >> 32) != 0u;");
+      o.l("  if (all_) break;");
+      o.l("  unsigned long long t_ = 0;");
+      o.l("  asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t_));");
+      o.l("  if (t0_ == 0ull) t0_ = t_;");
+      o.l("  else if (t_ - t0_ > 4000000000ull) break;   // a word that never arrives: NaN, not a hang");
+      o.l("  __nanosleep(ns_);");
+      o.l("  if (ns_ < 256u) ns_ *= 2u;");
+      o.l("  #pragma unroll");
+      o.l("  for (int it = 0; it < " + num(MAXIT) + "; ++it) {");
+      o.l("    const idx_t c = rl + it * " + num(L.gr) + "u;");
+      o.l("    #pragma unroll");
+      o.l("    for (int e = 0; e < " + num(W) + "; ++e)");
+      o.l("      if (c < " + NW_ + "u && (unsigned)(pw_[it][e] >> 32) == 0u) pw_[it][e] = "
+          "fop::ld_relaxed_gpu_u64(&partw[(c * " + num(slabs) + "u + slab) * " + num(SW) + "u + cv * " + num(W) + "u + e]);");
+      o.l("  }");
+      o.l("}");
+      o.l("#pragma unroll");
+      o.l("for (int it = 0; it < " + num(MAXIT) + "; ++it) {");
+      o.l("  const idx_t c = rl + it * " + num(L.gr) + "u;");
+      o.l("  if (c < " + num(NCH) + "u) {");
+      o.l("    #pragma unroll");
+      o.l("    for (int e = 0; e < " + num(W) + "; ++e) {");
+      o.l("      const float v_ = " + OWN + " ? red[cv * " + num(W) + "u + e] : ((unsigned)(pw_[it][e] >> 32) "
+          "? __uint_as_float((unsigned)pw_[it][e]) : __int_as_float(0x7fc00000));");
+      o.l("      acc[e] = " + comb("acc[e]", "v_") + ";");
+      o.l("    }");
+      o.l("  }");
+      o.l("}");
+      o.l("__syncthreads();   // every thread has read red[] before the tree reuses it");
+      tree();
+      exchange();
+      final_store();
+      o.l("for (int it = 0; it < " + num(MAXIT) + "; ++it) {   // leave the words zero for the next run");
+      o.l("  const idx_t c = rl + it * " + num(L.gr) + "u;");
+      o.l("  if (c < " + NW_ + "u) {");
+      o.l("    #pragma unroll");
+      o.l("    for (int e = 0; e < " + num(W) + "; ++e) fop::st_relaxed_gpu_u64(&partw[(c * " + num(slabs) + "u + slab) * " +
+          num(SW) + "u + cv * " + num(W) + "u + e], 0ull);");
+      o.l("  }");
+      o.l("}");
+      if (FM == 2) o.l("if (tid == 0u) cnt[slab] = 0u;");
+      o.ind--;
+      o.l("}");
     } else {
       size_t part = (size_t)NCH * (size_t)slabs * (size_t)SW * sizeof(float);
       part = (part + 255) & ~size_t(255);

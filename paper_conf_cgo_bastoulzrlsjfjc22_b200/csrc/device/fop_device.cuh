@@ -689,6 +689,34 @@ __device__ __forceinline__ u64 ld_relaxed_sys_u64(const u64* p) {
   asm volatile("ld.relaxed.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ void st_relaxed_gpu_u64(u64* p, u64 v) {
+  asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ u64 ld_relaxed_gpu_u64(const u64* p) {
+  u64 v;
+  asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+// COL_REDUCE flag words: (1 << 32 | fp32 bits).  Poll until the valid half is
+// set; the word carries the value, so no fence or atomic orders it.
+// A word that never arrives (a launch that broke the one-wave residency the
+// geometry guarantees) gives NaN after ~4 s instead of a hang.
+__device__ __forceinline__ float wait_flag_word(const u64* p) {
+  u64 w = ld_relaxed_gpu_u64(p);
+  if ((unsigned)(w >> 32) != 0u) return __uint_as_float((unsigned)w);
+  unsigned long long t0 = 0, t = 0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  unsigned ns = 32;
+  for (;;) {
+    __nanosleep(ns);
+    if (ns < 256) ns *= 2;
+    w = ld_relaxed_gpu_u64(p);
+    if ((unsigned)(w >> 32) != 0u) return __uint_as_float((unsigned)w);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 4000000000ull) return __int_as_float(0x7fc00000);
+  }
+}
+
 // Poll *p until its epoch half equals ep (the word lands in `w`); false after
 // ~limit_ns.  The first `spins` polls do not sleep (a peer that is about to
 // arrive costs one round trip, not a scheduler wake-up).

@@ -142,6 +142,7 @@ struct Launch {
   int row_prefetch = 0;           // ROW: prefetch the next row's streaming loads
   int col_pipe = 0;               // COL: software-pipelined row batches
   int col_il = 1;                 // COL: chunks interleave over rows (grid sweeps rows together)
+  int col_fin = 0;                // COL finalize: 0 fence + counter (default); 1/2 flag words (ablations)
   int row_hoist = 1;              // ROW: keep row-invariant loads in registers across rows
   int row_g = 1;                  // ROW: warps per row (> 1 for few long rows)
   int row_q = 1;                  // ROW: CTAs per row (a thread-block cluster) for few long rows

@@ -688,7 +688,13 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.nchunks = nch;
     L.work = rows;
     L.grid = slabs * nch;
-    if (nch > 1) {
+    // finalize: store + fence + arrival counter + last-arriving block (0, default),
+    // or flag words polled by the slab's last chunk block (1) / last arrival (2)
+    L.col_fin = knob("FOP_COL_FIN", 0);
+    if (nch > 1 && L.col_fin) {
+      L.ws_bytes = ((size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(unsigned long long) + 255) & ~size_t(255);
+      if (L.col_fin == 2) L.ws_bytes += (size_t)slabs * sizeof(unsigned);
+    } else if (nch > 1) {
       size_t part = (size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(float);
       part = (part + 255) & ~size_t(255);
       L.ws_bytes = part + (size_t)slabs * sizeof(unsigned);
