@@ -437,6 +437,9 @@ struct Gen {
         if (q.op == FOP_OP_LOAD) {
           for (size_t k = 0; k < L.kl.size(); k++)
             if (C(L.loads[q.acc], (int)k) != 0) dep[i] |= 1u << k;
+          // a flattened period launch: loop 0 is (c, r); only the period loads
+          // depend on c alone, the others on the whole flat index (pseudo-loop 30)
+          if (L.period && !L.period_load[q.acc] && (dep[i] & 1u)) dep[i] |= 1u << 30;
         } else if (q.op == X_FWD || q.op == X_SELF || q.op == X_SCALAR) {
           dep[i] = ~0u;
         } else if (q.op != FOP_OP_CONST) {
@@ -457,11 +460,12 @@ struct Gen {
         bool frontier0 = false;
         for (size_t j = i + 1; j < n; j++)
           if ((x.nodes[j].a == (int)i || x.nodes[j].b == (int)i) && (dep[j] & ~1u)) frontier0 = true;
-        const bool vec_table = dep[i] == 1u && costly[i] && frontier0 && L.kl.size() > 1 &&
-                               L.kl[0].extent % L.width == 0 && geometry_knob(L, "FOP_SMEM_TABLES_V", 1);
+        // (a flattened period launch: the cone depends on c = flat index mod period, any consumer)
+        const bool vec_table = dep[i] == 1u && costly[i] && frontier0 && geometry_knob(L, "FOP_SMEM_TABLES_V", 1) &&
+                               ((L.kl.size() > 1 && L.kl[0].extent % L.width == 0) || L.period);
         if (!vec_table && (var[i] || !costly[i] || !frontier || __builtin_popcount(dep[i]) != 1)) continue;
         int k = __builtin_ctz(dep[i]);
-        int64_t E = L.kl[k].extent;
+        int64_t E = k == 0 && L.period ? L.period : L.kl[k].extent;
         if ((k == 0 && !vec_table) || E > 8192 || bytes + E * 4 > 32 * 1024) continue;
         bytes += E * 4;
         Table t{(int)si, (int)i, k, E, "tbl" + num(x.stmt) + "_" + num(i)};
@@ -584,6 +588,13 @@ struct Gen {
       its[u].push_back({0, "iv" + t});
       decompose("r" + t, 1, (int)L.kl.size(), t, its[u]);
       if (tail) o.l("const bool full" + t + " = iv" + t + " + " + num(W) + "u <= " + num(EV) + "u;");
+      if (L.period) {   // c of each element: the flat index modulo the period (one wrap at most: W <= period)
+        o.l("unsigned PC" + t + "[" + num(W) + "];");
+        o.l("{ const unsigned c0_ = (unsigned)(iv" + t + " % " + num(L.period) + "u);");
+        o.l("  #pragma unroll");
+        o.l("  for (int e = 0; e < " + num(W) + "; ++e) PC" + t + "[e] = c0_ + e >= " + num(L.period) + "u ? c0_ + e - " +
+            num(L.period) + "u : c0_ + e; }");
+      }
       // loads
       for (size_t k = 0; k < L.loads.size(); k++) {
         if (!need[k]) continue;
@@ -602,6 +613,15 @@ struct Gen {
             o.l("  for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = fop::sload_raw<" +
                 num(es(a.tensor)) + ", " + pol(a, false) + ">(" + ptr(a.tensor, off + " + e * " + num(cv)) + ");");
           o.l("}");
+          continue;
+        }
+        if (L.period && L.period_load[k]) {   // bias[c] over the flattened (c, r): one element per lane slot
+          std::vector<std::pair<int, std::string>> rest(its[u].begin() + 1, its[u].end());
+          std::string off0 = affine(a, rest);
+          o.l("float " + nm + "[" + num(W) + "];");
+          o.l("#pragma unroll");
+          o.l("for (int e = 0; e < " + num(W) + "; ++e) " + nm + "[e] = ok" + t + " ? fop::sload<" + dt + ", " +
+              pol(a, true) + ">(" + ptr(a.tensor, off0 + " + (idx_t)PC" + t + "[e] * " + num(cv)) + ") : 0.f;");
           continue;
         }
         if (cv == 0) {
@@ -664,7 +684,9 @@ struct Gen {
           if (tb.si == (int)si)
             for (auto& kv : its[u])
               if (kv.first == tb.k) {  // slots past the end (ok false) still evaluate: keep the index in the table
-                if (tb.k == 0) {   // per element: the vector's W entries, read with 16 B shared loads
+                if (tb.k == 0 && L.period) {   // per element at c = flat index mod period
+                  ov[tb.node] = tb.name + "[PC" + t + "[$E]]";
+                } else if (tb.k == 0) {   // per element: the vector's W entries, read with 16 B shared loads
                   const std::string tv = "TV" + tb.name.substr(3) + t;
                   o.l("float " + tv + "[" + num(L.width) + "];");
                   o.l("#pragma unroll");

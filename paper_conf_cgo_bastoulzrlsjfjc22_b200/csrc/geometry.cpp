@@ -281,6 +281,45 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     collapse_into(p, acc, seg2, L.kl);
   }
 
+  // ---- EW over an innermost extent no vector divides, under a broadcast along
+  // it (bias add over 1001 columns: the bias row blocks the collapse of
+  // (c, r), and W must divide E[c]).  When every access is either contiguous
+  // across (d_v, next loop) — coef(next) == E[d_v] — or ignores the next loop
+  // (a "period" access, e.g. bias[c]), the two loops become one flat loop
+  // carrying full-width vectors; period accesses are read per element at
+  // c = flat index mod E[d_v] (vector and scalar accesses mixed).
+  L.period = 0;
+  L.period_load.assign(L.loads.size(), 0);
+  if (L.kclass == FOP_CLASS_EW && L.seq.empty() && !L.virt_vec && !L.scalar_variant && !L.force_w1 &&
+      L.kl.size() >= 2 && geometry_knob(L, "FOP_EW_PERIOD", 1)) {
+    const int64_t E0 = L.kl[0].extent;
+    int mes = 16;
+    for (const Affine* a : acc)
+      if (coef(L, *a, 0) == 1) mes = std::min(mes, esize(d.t[a->tensor].dtype));
+    const int Wf = std::max(1, vbytes / mes);
+    if (Wf > 1 && E0 % Wf != 0 && E0 >= Wf && (o.force_width <= 0 || o.force_width >= Wf)) {
+      bool ok = true;
+      int nflat = 0;
+      for (size_t k = 0; k < L.loads.size() && ok; k++) {
+        const int64_t c0 = coef(L, L.loads[k], 0), c1 = coef(L, L.loads[k], 1);
+        if (c0 == 1 && c1 == E0) nflat++;
+        else if (c1 == 0) L.period_load[k] = 1;
+        else ok = false;
+      }
+      for (const auto& x : L.stmts)
+        ok &= coef(L, x.write, 0) == 1 && coef(L, x.write, 1) == E0;
+      if (ok && nflat + (int)L.stmts.size() > 0) {
+        L.period = E0;
+        KLoop& K = L.kl[0];
+        K.members.insert(K.members.end(), L.kl[1].members.begin(), L.kl[1].members.end());
+        K.extent *= L.kl[1].extent;
+        L.kl.erase(L.kl.begin() + 1);
+      } else {
+        L.period_load.assign(L.loads.size(), 0);
+      }
+    }
+  }
+
   // ---- a4: width
   int min_es = 16;
   bool any_vec = false;
@@ -428,7 +467,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   L.load_cb.assign(L.loads.size(), 0);
   L.load_cb_r.assign(L.loads.size(), 0);
   for (size_t k = 0; k < L.loads.size(); k++) {
-    if (coef(L, L.loads[k], 0) == 1) L.load_cb[k] = vec_cb(L.loads[k], 0, W, vmax_ld);
+    if (coef(L, L.loads[k], 0) == 1 && !L.period_load[k]) L.load_cb[k] = vec_cb(L.loads[k], 0, W, vmax_ld);
     if (L.kclass == FOP_CLASS_TRANSPOSE && coef(L, L.loads[k], 0) != 1 && coef(L, L.loads[k], 1) == 1)
       L.load_cb_r[k] = vec_cb(L.loads[k], 1, L.read_width, 32);
   }
