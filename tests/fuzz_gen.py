@@ -12,7 +12,8 @@ generator:
     bit; REDUCE sums compare normwise (R16), max reductions bit for bit;
   * patterns: one ASSIGN, one REDUCE, a TEMP producer over a subset of the
     loops consumed by an ASSIGN (cfg2's shape), a row REDUCE whose value an
-    ASSIGN over the same loops consumes (softmax/LayerNorm's shape).
+    ASSIGN over the same loops consumes (softmax/LayerNorm's shape), and an
+    integer ASSIGN over i32 tensors (reading R30, bit-exact).
 """
 import numpy as np
 
@@ -20,6 +21,8 @@ EXTENTS = [1, 2, 3, 5, 7, 8, 13, 16, 24, 31, 32, 33, 48, 64, 100, 128, 257]
 DTYPES = ["f32", "f16", "bf16"]
 EXACT_UNARY = ["neg", "abs", "relu", "sqrt"]
 EXACT_BINARY = ["add", "sub", "mul", "div", "max", "min"]
+INT_UNARY = ["neg", "abs", "relu"]                       # reading R30: integer statements
+INT_BINARY = ["add", "sub", "mul", "max", "min"]
 
 
 def _loops(rng, max_elems=120_000):
@@ -81,7 +84,7 @@ def _dag(rng, nloads, nodes_max=6):
 def random_op(rng):
     loops = _loops(rng)
     names = list(loops)
-    pat = rng.choice(["assign", "reduce", "producer", "rowstat"], p=[0.4, 0.25, 0.15, 0.2])
+    pat = rng.choice(["assign", "reduce", "producer", "rowstat", "integer"], p=[0.35, 0.25, 0.12, 0.18, 0.1])
     tensors, stmts = {}, []
     seed = int(rng.integers(1000, 100000))
 
@@ -98,7 +101,33 @@ def random_op(rng):
         return reads
 
     out_dt = str(rng.choice(DTYPES))
-    if pat == "assign":
+    if pat == "integer":
+        # reading R30: i32 tensors only, wrap-around integer DAG, any layout (transposes included)
+        reads = []
+        for i in range(int(rng.integers(1, 4))):
+            sub = [n for n in names if rng.random() < 0.75] or [str(rng.choice(names))]
+            sub = list(rng.permutation(sub)) if rng.random() < 0.4 else sub
+            t = _tensor(rng, loops, sub, "i32", "in", seed + i)
+            t["init"] = ("randint", -2 ** 30, 2 ** 30, seed + i)
+            tensors[f"x{i}"] = t
+            reads.append((f"x{i}", list(sub)))
+        perm = list(rng.permutation(names)) if rng.random() < 0.5 else names
+        tensors["out"] = _tensor(rng, loops, perm, "i32", "out", 0)
+        expr = [("load", k) for k in range(len(reads))]
+        if rng.random() < 0.5:
+            expr.append(("const", float(rng.choice([3.0, -7.0, 65537.0, 0.0]))))
+        for _ in range(int(rng.integers(1, 6))):
+            n = len(expr)
+            if rng.random() < 0.3:
+                expr.append((str(rng.choice(INT_UNARY)), int(rng.integers(0, n))))
+            else:
+                expr.append((str(rng.choice(INT_BINARY)), int(rng.integers(0, n)), int(rng.integers(0, n))))
+        last = len(expr) - 1
+        for k in range(len(reads)):   # every load used
+            expr.append(("add", last, k))
+            last = len(expr) - 1
+        stmts.append({"kind": "assign", "loops": names, "write": ("out", list(perm)), "reads": reads, "expr": expr})
+    elif pat == "assign":
         reads = inputs(int(rng.integers(1, 4)))
         perm = list(rng.permutation(names)) if rng.random() < 0.5 else names
         tensors["out"] = _tensor(rng, loops, perm, out_dt, "out", 0)
