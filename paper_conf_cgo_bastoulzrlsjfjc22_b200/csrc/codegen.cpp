@@ -1317,17 +1317,34 @@ struct Gen {
     decompose("t", 2, (int)L.kl.size(), "", outer);
     std::vector<std::pair<int, std::string>> in_its = {{0, "v"}, {1, "(rb * " + num(TR) + "u + rc * " + num(WR) + "u)"}};
     in_its.insert(in_its.end(), outer.begin(), outer.end());
+    // Tile orientation.  d_v-major (OM = 0): the input vectors land as 16 B
+    // shared stores, the read-out gathers element (f mod E[d_v], f div E[d_v])
+    // with lanes 8 tile rows apart — few banks when E[d_v] is long.  Output-
+    // major (OM = 1, long E[d_v] such as C = 255): the tile IS the flat output
+    // chunk; lanes take consecutive d_v positions (32 different input rows of
+    // the same d_r vector) and scatter each vector's WR elements into
+    // consecutive 2/4-byte cells — lane-contiguous, conflict-free — and the
+    // read-out is a straight 16 B vector per thread.
+    const bool OM = L.tr_om != 0;
     o.l("__syncthreads();   // the previous tile is written out");
     o.l("#pragma unroll 4");
     o.l("for (unsigned q = threadIdx.x; q < " + num(nin) + "u; q += " + num(L.block) + "u) {");
     o.ind++;
-    o.l("const unsigned rc = q % " + num(TR / WR) + "u, v = q / " + num(TR / WR) + "u;");
+    if (OM) o.l("const unsigned v = q % " + num(EV) + "u, rc = q / " + num(EV) + "u;");
+    else o.l("const unsigned rc = q % " + num(TR / WR) + "u, v = q / " + num(TR / WR) + "u;");
     o.l("u32 w[" + num(WR * esi / 4) + "];");
     o.l("fop::vload_words<" + std::string(dtn(d.t[ta.tensor].dtype)) + ", " + num(WR) + ", " +
         num(L.load_cb_r[L.trans_load]) + ", " + pol(ta, false) + ">(w, " + ptr(ta.tensor, affine(ta, in_its)) + ");");
     o.l("#pragma unroll");
-    o.l("for (int c = 0; c < " + num(WR * esi / 4) + "; ++c) reinterpret_cast<u32*>(fop_tile + (v * " + num(TR) +
-        "u + rc * " + num(WR) + "u) * " + num(esi) + "u)[c] = w[c];");
+    if (OM && esi == 2)
+      o.l("for (int i = 0; i < " + num(WR) + "; ++i) reinterpret_cast<u16*>(fop_tile)[(rc * " + num(WR) + "u + i) * " +
+          num(EV) + "u + v] = (u16)(w[i >> 1] >> ((i & 1) * 16));");
+    else if (OM)
+      o.l("for (int i = 0; i < " + num(WR) + "; ++i) reinterpret_cast<u32*>(fop_tile)[(rc * " + num(WR) + "u + i) * " +
+          num(EV) + "u + v] = w[i];");
+    else
+      o.l("for (int c = 0; c < " + num(WR * esi / 4) + "; ++c) reinterpret_cast<u32*>(fop_tile + (v * " + num(TR) +
+          "u + rc * " + num(WR) + "u) * " + num(esi) + "u)[c] = w[c];");
     o.ind--;
     o.l("}");
     o.l("__syncthreads();");
@@ -1339,19 +1356,29 @@ struct Gen {
     o.ind++;
     std::string cell = "fop_tile + (((q * " + num(OW) + "u + e) % " + num(EV) + "u) * " + num(TR) + "u + (q * " +
                        num(OW) + "u + e) / " + num(EV) + "u) * " + num(esi) + "u";
+    if (OM) {   // the thread's OW output elements: one or two 16 B shared loads
+      const int nw = OW * esi / 4;
+      o.l("u32 tw_[" + num(nw) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int c = 0; c < " + num(nw / 4) + "; ++c) reinterpret_cast<uint4*>(tw_)[c] = "
+          "reinterpret_cast<const uint4*>(fop_tile + q * " + num(OW * esi) + "u)[c];");
+    }
+    auto elem_bits = [&](const std::string& castty) {   // raw element e (u16 or u32 bits)
+      if (!OM) return "*reinterpret_cast<const " + castty + "*>(" + cell + ")";
+      return esi == 2 ? std::string("(u16)(tw_[e >> 1] >> ((e & 1) * 16))") : std::string("tw_[e]");
+    };
     if (raw) {
       o.l("u32 O[" + num(OW) + "];");
       o.l("#pragma unroll");
-      o.l("for (int e = 0; e < " + num(OW) + "; ++e) O[e] = " +
-          std::string(esi == 2 ? "*reinterpret_cast<const u16*>(" : "*reinterpret_cast<const u32*>(") + cell + ");");
+      o.l("for (int e = 0; e < " + num(OW) + "; ++e) O[e] = " + elem_bits(esi == 2 ? "u16" : "u32") + ";");
       o.l("fop::vstore_raw<" + num(eso) + ", " + num(OW) + ", 16, " + spol() + ">(dst + q * 16u, O);");
     } else {
       std::string lt = "L" + num(L.trans_load);
       o.l("float " + lt + "[" + num(OW) + "];");
       o.l("#pragma unroll");
-      std::string rd = d.t[ta.tensor].dtype == FOP_F16    ? "fop::h2f(*reinterpret_cast<const u16*>(" + cell + "))"
-                       : d.t[ta.tensor].dtype == FOP_BF16 ? "fop::b2f(*reinterpret_cast<const u16*>(" + cell + "))"
-                                                          : "*reinterpret_cast<const float*>(" + cell + ")";
+      std::string rd = d.t[ta.tensor].dtype == FOP_F16    ? "fop::h2f(" + elem_bits("u16") + ")"
+                       : d.t[ta.tensor].dtype == FOP_BF16 ? "fop::b2f(" + elem_bits("u16") + ")"
+                                                          : "__uint_as_float(" + elem_bits("u32") + ")";
       o.l("for (int e = 0; e < " + num(OW) + "; ++e) " + lt + "[e] = " + rd + ";");
       DagCtx c;
       c.tag = "";

@@ -384,6 +384,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     while (wr > 1 && L.kl[1].extent % wr) wr /= 2;
     L.read_width = wr;
     L.tr_smem = 0;
+    L.tr_om = 0;
     if (W >= 2 && wr == 1 && !L.scalar_variant && geometry_knob(L, "FOP_TR_SMEM", 1)) {
       // d_r cannot carry vectors (odd extent, e.g. a 7x7 plane: 49), but when
       // consecutive d_v rows are adjacent in the load tensor (coef(d_v) ==
@@ -431,19 +432,29 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
         for (size_t q = 0; q < L.kl.size(); q++) ok &= coef(L, L.loads[k], (int)q) == 0;   // constants only
       }
       const int esi = esize(d.t[L.loads[L.trans_load].tensor].dtype);
-      // the input rows are read with whole vectors along d_r: every row start aligned
-      ok &= chunk_bytes(p, L, L.loads[L.trans_load], 1, wr * esi) == wr * esi;
       const int64_t rowb = EVx * std::max(esi, eso);
-      int64_t TR = 0;
       const int64_t cap = std::min<int64_t>(ER, geometry_knob(L, "FOP_TR_SMEM_BYTES", 32768) / rowb);
-      for (int64_t tr = cap - cap % wr; ok && tr >= wr; tr -= wr)
-        if (ER % tr == 0 && (tr * EVx * eso) % 16 == 0) {
-          TR = tr;
-          break;
-        }
+      // output-major tile for long d_v rows (codegen gen_transpose_smem_out): each
+      // lane reads one input row's vector, so the vector grows to a full 32 B
+      // sector (C = 255: 3.1 -> 5.4 TB/s, profiles/r02/sweep_r02_trsmem.log)
+      const bool om = EVx >= 32 && geometry_knob(L, "FOP_TR_SMEM_OM", 1);
+      auto pick = [&](int w_) -> int64_t {   // rows per tile for read vectors of w_ elements, 0 = none
+        // the input rows are read with whole vectors along d_r: every row start aligned
+        if (!ok || w_ < 2 || ER % w_ || chunk_bytes(p, L, L.loads[L.trans_load], 1, w_ * esi) != w_ * esi) return 0;
+        for (int64_t tr = cap - cap % w_; tr >= w_; tr -= w_)
+          if (ER % tr == 0 && (tr * EVx * eso) % 16 == 0) return tr;
+        return 0;
+      };
+      int64_t TR = 0;
+      if (om) {
+        const int w32 = std::min<int>(32, geometry_knob(L, "FOP_TR_WR_BYTES", 32)) / esi;
+        if ((TR = pick(w32))) wr = L.read_width = w32;
+      }
+      if (!TR) TR = pick(wr);
       if (TR) {
         L.tr_smem = 2;
         L.tr_tv = TR;
+        L.tr_om = om ? 1 : 0;
       }
     }
     if ((W == 1 || wr == 1) && !L.tr_smem) {  // degenerate tile: plain elementwise with gathers

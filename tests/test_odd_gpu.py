@@ -57,3 +57,24 @@ def test_bias_add_full_size_every_candidate():
         op.run(dev)
         torch.cuda.synchronize()
         assert_bitexact(to_host(dev["out"], "f16"), ref, f"candidate {k} {op.selected(0)[0]}")
+
+
+@pytest.mark.parametrize("dims,dtype", [((2, 255, 56, 56), "f16"), ((1, 255, 7, 8), "f32"), ((2, 129, 4, 8), "bf16"),
+                                        ((3, 33, 8, 8), "f16")])
+@pytest.mark.parametrize("om", ["1", "0"])
+def test_transpose_long_odd_channels_output_major_tile(monkeypatch, dims, dtype, om):
+    """NCHW -> NHWC with a long odd C (255): the output rows carry no store vector, so a
+    tile of whole NHWC rows is written flat; with the output-major tile (FOP_TR_SMEM_OM=1,
+    the default for C >= 32) lanes scatter consecutive channels into the tile and read it
+    out as 16 B vectors.  Both tile orientations bit-exact, NaN payloads of a pure move kept."""
+    monkeypatch.setenv("FOP_TR_SMEM_OM", om)
+    d = W.cfg3(*dims, dtype=dtype)
+    d["tensors"]["x"]["init"] = ("special", 5)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x)
+    assert op.selected(0)[0].startswith("fop_transpose_smem")
+    assert ("tw_" in op.source()) == (om == "1" and dims[1] >= 32)
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+    d["stmts"][0]["expr"] = [("load", 0)]
+    got, op = run_gpu(d, x)
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out (move)")

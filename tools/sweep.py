@@ -29,7 +29,7 @@ L2 = 126 << 20
 def main():
     name = sys.argv[1]
     variants = sys.argv[2:] or [""]
-    d = (W.CONFIGS.get(name) or W.N4.get(name) or W.N3[name])()
+    d = (W.CONFIGS.get(name) or W.N4.get(name) or W.ODD.get(name) or W.N3[name])()
     x = W.make_inputs(d)
     o = W.alloc_outputs(d, fill_nan=False)
     nbytes = W.algorithmic_bytes(d)

@@ -38,13 +38,13 @@ are defined in ``include/fop.h``.
 
 from .configs import (CONFIGS, cfg1, cfg1_bias_b, cfg2, cfg3, cfg4a, cfg4b,
                       fig2_running_example, transpose2d, nhwc_to_nchw, cfg2_nhwc, bias_add_rows, algorithmic_bytes,
-                      elem_size, N4, N3)
+                      elem_size, N4, N3, ODD)
 from .inputs import (make_inputs, alloc_outputs, tensor_span, tensor_strides,
                      contiguous_strides, NP_DTYPE)
 
 __all__ = [
     "CONFIGS", "cfg1", "cfg1_bias_b", "cfg2", "cfg3", "cfg4a", "cfg4b",
-    "fig2_running_example", "transpose2d", "nhwc_to_nchw", "cfg2_nhwc", "bias_add_rows", "algorithmic_bytes", "elem_size", "N4", "N3",
+    "fig2_running_example", "transpose2d", "nhwc_to_nchw", "cfg2_nhwc", "bias_add_rows", "algorithmic_bytes", "elem_size", "N4", "N3", "ODD",
     "make_inputs", "alloc_outputs", "tensor_span", "tensor_strides",
     "contiguous_strides", "NP_DTYPE",
 ]
