@@ -2016,7 +2016,8 @@ struct Gen {
   void gen_col() {
     const int W = L.width, U = L.unroll;
     const XStmt& x = L.stmts[0];
-    const int64_t NVD = L.kl[0].extent / W;
+    const int64_t EV0 = L.kl[0].extent;
+    const int64_t NVD = L.col_shift ? (EV0 + W - 1) / W : EV0 / W;   // col_shift: a partial last vector
     const int64_t SVN = (NVD + L.gv - 1) / L.gv;
     int64_t slabs = SVN;
     for (int k = 1; k < L.nsplit; k++) slabs *= L.kl[k].extent;
@@ -2111,6 +2112,47 @@ struct Gen {
         for (size_t k = 0; k < L.loads.size(); k++) {
           if (!wpv[k]) continue;
           const Affine& a = L.loads[k];
+          if (L.col_shift) {
+            // the row's W elements from the two aligned 16 B chunks around them,
+            // funnel-shifted by the row's misalignment m_ (elements); a second
+            // chunk past the tensor's end is read element-wise
+            const int esk = es(a.tensor), epw = 4 / esk;
+            const std::string B = buf + num(k) + "_" + num(u);
+            const int64_t span = tensor_bytes(a.tensor) / esk;
+            o.l("{");
+            o.l("  const idx_t o_ = " + affine(a, bits) + ";");
+            o.l("  const unsigned m_ = (unsigned)(((u64)T" + num(a.tensor) + " + (u64)o_ * " + num(esk) + "u) & 15u) / " +
+                num(esk) + "u;");
+            o.l("  const idx_t a_ = o_ - m_;");
+            // (the second chunk could come from the next lane's first by a shuffle:
+            // measured slower, 2978 vs 3888 GB/s on [65536,1001] — the shuffle waits
+            // for each row's load, serialising the batch's latency)
+            o.l("  u32 V_[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};");
+            o.l("  if (okc && rr < r1) {");
+            o.l("    fop::ldraw<16, " + pol(a, false) + ">(V_, T" + num(a.tensor) + " + (u64)a_ * " + num(esk) + "u);");
+            o.l("    if (m_ != 0u) {");
+            o.l("      if (a_ + " + num(2 * W) + "u <= (idx_t)" + num(span) + "ull) fop::ldraw<16, " + pol(a, false) +
+                ">(V_ + 4, T" + num(a.tensor) + " + (u64)(a_ + " + num(W) + "u) * " + num(esk) + "u);");
+            if (esk == 2)
+              o.l("      else for (int e = 0; e < " + num(W) + "; ++e) if (a_ + " + num(W) + "u + e < (idx_t)" + num(span) +
+                  "ull) V_[4 + (e >> 1)] |= (u32)fop::ld16<" + pol(a, false) + ">(T" + num(a.tensor) + " + (u64)(a_ + " +
+                  num(W) + "u + e) * 2u) << ((e & 1) * 16);");
+            else
+              o.l("      else for (int e = 0; e < " + num(W) + "; ++e) if (a_ + " + num(W) + "u + e < (idx_t)" + num(span) +
+                  "ull) fop::ldraw<4, " + pol(a, false) + ">(V_ + 4 + e, T" + num(a.tensor) + " + (u64)(a_ + " + num(W) +
+                  "u + e) * 4u);");
+            o.l("    }");
+            o.l("  }");
+            o.l("  const unsigned t_ = m_ / " + num(epw) + "u, s_ = (m_ % " + num(epw) + "u) * " + num(esk * 8) + "u;");
+            o.l("  #pragma unroll");
+            o.l("  for (int q = 0; q < 4; ++q) {   // word q of the window: V_[t_ + q .. t_ + q + 1] >> s_");
+            o.l("    const u32 lo_ = t_ == 0u ? V_[q] : t_ == 1u ? V_[q + 1] : t_ == 2u ? V_[q + 2] : V_[q + 3];");
+            o.l("    const u32 hi_ = t_ == 0u ? V_[q + 1] : t_ == 1u ? V_[q + 2] : t_ == 2u ? V_[q + 3] : V_[q + 4];");
+            o.l("    " + B + "[q] = __funnelshift_r(lo_, hi_, s_);");
+            o.l("  }");
+            o.l("}");
+            continue;
+          }
           o.l("if (okc && rr < r1) fop::vload_words<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + num(W) + ", " +
               num(L.load_cb[k]) + ", " + pol(a, false) + ">(" + buf + num(k) + "_" + num(u) + ", " +
               ptr(a.tensor, affine(a, bits)) + ");");
@@ -2374,7 +2416,12 @@ struct Gen {
       std::string off = affine(x.write, cits);
       int64_t cw = C(x.write, 0);
       std::string dt = dtn(x.out_dtype);
-      if (cw == 1 && L.store_cb[0])
+      if (cw == 1 && L.store_cb[0] && L.col_shift && EV0 % W) {   // the last vector is partial
+        o.l("if (iv + " + num(W) + "u <= " + num(EV0) + "u) fop::vstore<" + dt + ", " + num(W) + ", " +
+            num(L.store_cb[0]) + ", fop::ST_DEFAULT>(" + ptr(x.write.tensor, off) + ", res);");
+        o.l("else for (int e = 0; e < " + num(W) + "; ++e) if (iv + e < " + num(EV0) + "u) fop::sstore<" + dt + ">(" +
+            ptr(x.write.tensor, off + " + e") + ", res[e]);");
+      } else if (cw == 1 && L.store_cb[0])
         o.l("fop::vstore<" + dt + ", " + num(W) + ", " + num(L.store_cb[0]) + ", fop::ST_DEFAULT>(" +
             ptr(x.write.tensor, off) + ", res);");
       else

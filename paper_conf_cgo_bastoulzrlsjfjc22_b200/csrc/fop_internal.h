@@ -177,6 +177,7 @@ struct Launch {
   size_t ws_off = 0, ws_bytes = 0;  // COL_REDUCE partials + counters
   std::vector<int> align;         // per tensor: byte alignment the vector variant assumes
   bool scalar_variant = false;    // this launch is the narrow (W=1) variant
+  int col_shift = 0;              // COL: full-width vectors over odd rows via per-row funnel shifts of aligned chunks
   int tr_om = 0;                  // TRANSPOSE smem (tr_smem 2): output-major tile (lane-contiguous scatter, vector read-out)
   int64_t period = 0;             // EW: kl[0] is (d_v x next loop) flattened; period accesses use c = flat % period
   std::vector<char> period_load;  // per load: read per element at c = flat index mod period (bias[c] over odd c)

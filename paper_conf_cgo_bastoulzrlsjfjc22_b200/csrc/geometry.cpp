@@ -367,9 +367,24 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     }
     if (ok && ref) L.row_peel = 1;
   }
+  // COL_REDUCE over rows no vector divides (column sums over 1001 columns): keep
+  // the full width; each lane loads the two aligned 16 B chunks around its W
+  // columns of the row and funnel-shifts them by the row's misalignment (the
+  // same for every lane of the row), so the loads stay 16 B vectors whatever
+  // the row pitch; the last vector's columns past E[d_v] are never stored.
+  L.col_shift = 0;
+  if (L.kclass == FOP_CLASS_COL_REDUCE && W > 1 && EV % W != 0 && EV >= W && L.nsplit == 1 && !L.scalar_variant &&
+      L.stmts.size() == 1 && geometry_knob(L, "FOP_COL_SHIFT", 1)) {
+    bool ok = coef(L, L.stmts[0].write, 0) == 1;
+    for (const auto& a : L.loads) {
+      const int64_t c0 = coef(L, a, 0);
+      ok &= c0 == 0 || (c0 == 1 && W * esize(d.t[a.tensor].dtype) == 16);
+    }
+    if (ok) L.col_shift = 1;
+  }
   if (tail_ok) {
     if (EV < W) W = pow2_floor(EV);
-  } else if (!L.row_peel) {
+  } else if (!L.row_peel && !L.col_shift) {
     while (W > 1 && EV % W) W /= 2;
   }
   L.width = W;
@@ -485,6 +500,9 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   L.store_cb.assign(L.stmts.size(), 0);
   for (size_t k = 0; k < L.stmts.size(); k++)
     if (coef(L, L.stmts[k].write, 0) == 1) L.store_cb[k] = vec_cb(L.stmts[k].write, 0, W, vmax);
+  if (L.col_shift)   // aligned 16 B chunks around each row's window (the base must be 16 B aligned)
+    for (size_t k = 0; k < L.loads.size(); k++)
+      if (coef(L, L.loads[k], 0) == 1) L.load_cb[k] = 16;
   if (L.row_peel) {   // alignment comes from the per-row shift, not from the static coefficients
     for (size_t k = 0; k < L.loads.size(); k++) {
       if (coef(L, L.loads[k], 0) != 1) continue;
@@ -713,7 +731,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
                                                        (int64_t)knob("FOP_ROW_CLUSTERS", 1 << 30)})) * Q;
     L.unroll = 1;
   } else {  // COL_REDUCE
-    int64_t nvd = EV / W;
+    int64_t nvd = L.col_shift ? (EV + W - 1) / W : EV / W;   // col_shift: a partial last vector
     const Affine* big = nullptr;
     for (const auto& a : L.loads)
       if (coef(L, a, 0) == 1) big = &a;

@@ -78,3 +78,49 @@ def test_transpose_long_odd_channels_output_major_tile(monkeypatch, dims, dtype,
     d["stmts"][0]["expr"] = [("load", 0)]
     got, op = run_gpu(d, x)
     assert_bitexact(got["out"], O.run(d, x)["out"], "out (move)")
+
+
+def _colred(R, C, dtype="f16", op="sum", expr=None):
+    return {"name": "colred", "loops": {"r": R, "c": C},
+            "tensors": {"x": {"shape": [R, C], "dtype": dtype, "role": "in", "init": ("normal", 0.0, 1.0, 71),
+                              "strides": None},
+                        "out": {"shape": [C], "dtype": "f32", "role": "out", "init": None, "strides": None}},
+            "stmts": [{"kind": "reduce", "op": op, "loops": ["r", "c"], "write": ("out", ["c"]),
+                       "reads": [("x", ["r", "c"])], "expr": expr or [("load", 0)]}]}
+
+
+@pytest.mark.parametrize("R,C,dtype,op", [(65536, 1001, "f16", "sum"), (777, 1001, "f16", "sum"), (300, 13, "f16", "sum"),
+                                          (5000, 37, "f32", "sum"), (2000, 257, "bf16", "sum"), (3001, 1001, "f16", "max"),
+                                          (64, 9, "f16", "sum")])
+@pytest.mark.parametrize("offset", [0, 1])
+def test_column_reduction_over_odd_rows(R, C, dtype, op, offset):
+    """Column sums / maxima over rows of odd length: full-width vectors, each row's window
+    funnel-shifted out of two aligned 16 B chunks; the partial last vector's extra
+    columns are never stored.  Misaligned base pointers take the narrow variant."""
+    from harness import abs_terms_desc, assert_normwise
+    d = _colred(R, C, dtype, op)
+    x = W.make_inputs(d)
+    got, o = run_gpu(d, x, offset=offset)
+    if offset == 0:
+        assert "__funnelshift_r" in o.source(), o.info()["launches"][0]
+    ref = O.run(d, x)["out"]
+    if op == "max":
+        assert_bitexact(got["out"], ref, "out")
+    else:
+        assert_normwise(got["out"], ref, O.run(abs_terms_desc(d, 0), x)["out"], 1e-5, "out")
+
+
+def test_column_sum_of_squares_odd_rows_every_candidate():
+    from harness import abs_terms_desc, assert_normwise, device_tensors, to_host
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    d = _colred(65536, 1001, "f16", "sum", [("load", 0), ("mul", 0, 0)])
+    x = W.make_inputs(d)
+    ref = O.run(d, x)["out"]
+    scale = O.run(abs_terms_desc(d, 0), x)["out"]
+    nv = FusedOp(d).info()["launches"][0]["nvariants"]
+    for k in range(nv):
+        op = FusedOp(d, variant=k)
+        dev = device_tensors(d, x)
+        op.run(dev)
+        torch.cuda.synchronize()
+        assert_normwise(to_host(dev["out"], "f32"), ref, scale, 1e-5, f"candidate {k}")
