@@ -43,6 +43,7 @@ def test_nhwc_bn_odd_channels(dims):
     assert_bitexact(got["y"], O.run(d, x)["y"], "y")
 
 
+@pytest.mark.full_size
 def test_bias_add_full_size_every_candidate():
     """[65536, 1001] f16 (a 1001-class classifier's logits over 65536 tokens), every tuning candidate."""
     from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
@@ -110,6 +111,7 @@ def test_column_reduction_over_odd_rows(R, C, dtype, op, offset):
         assert_normwise(got["out"], ref, O.run(abs_terms_desc(d, 0), x)["out"], 1e-5, "out")
 
 
+@pytest.mark.full_size
 def test_column_sum_of_squares_odd_rows_every_candidate():
     from harness import abs_terms_desc, assert_normwise, device_tensors, to_host
     from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp

@@ -7,7 +7,7 @@
 set -x
 export PYTHONUNBUFFERED=1
 K='not full_size and not past_2p31 and not absent_rank and not two_processes and not run_host'
-T="tests/test_parity_gpu.py tests/test_n4_ops.py tests/test_n3_recurrence.py tests/test_peer.py tests/test_repeat_runs.py tests/test_run_many.py tests/test_edge_cases.py"
+T="tests/test_parity_gpu.py tests/test_n4_ops.py tests/test_n3_recurrence.py tests/test_peer.py tests/test_repeat_runs.py tests/test_run_many.py tests/test_edge_cases.py tests/test_odd_gpu.py tests/test_int_gpu.py tests/test_transcendental_gpu.py"
 # racecheck and synccheck serialise kernels: the simulated multi-rank peer
 # tests (W kernels on W streams waiting for each other's pushes) then report
 # their time-out flag by design, so those run under memcheck/initcheck only
