@@ -50,6 +50,14 @@ OPS = [("cfg2", W.cfg2, "ew"), ("cfg3", W.cfg3, "transpose"), ("cfg4a", W.cfg4a,
 GLOBAL = {"cfg2": (lambda w: W.cfg2(N=128 * w), "n"), "cfg3": (lambda w: W.cfg3(N=256 * w), "n"),
           "cfg4a": (lambda w: W.cfg4a(B=64 * w), "b"), "cfg4b": (lambda w: W.cfg4b(R=65536 * w), "r")}
 STRONG_SCALE = 4              # BASELINE.json configs[4]: "4x the above batch"
+# the paper's own headline, quoted beside the B200 numbers (context, not a target: another
+# metric — whole-network fused-operator time vs isl scheduling — on another GPU)
+PAPER_CONTEXT = {"claim": "1.7x geomean improvement of fused-operator time over state-of-the-art (isl) "
+                          "scheduling, fused operators of 7 networks (1.78x recomputed from Table II)",
+                 "gpu": "NVIDIA Tesla V100 PCIe 16 GB @1245 MHz, CUDA 10.1, MindSpore r1.1 + AKG",
+                 "source": "PAPER.md P:28 (Sec. I), P:361-365 (Sec. VI platform), P:397-403 (Table II)",
+                 "b200_bar": "BASELINE.json north_star: >= 80% of 8 TB/s per fused op (6.4 TB/s); "
+                             "per-op fractions of 8 TB/s and of the measured copy are in config.per_op"}
 FALLBACK_HBM = 6650.0
 L2_BYTES = 126 << 20          # B200 L2 (public figure), for the steady-state copies
 METRIC = "achieved HBM GB/s (fused-op suite; per-op GB/s and % of peak in config.per_op)"
@@ -593,6 +601,7 @@ def run_fop(args):
                     "ms_per_step": e2e_ms, "path": "fop_run_host_many (pinned host -> HBM -> kernels -> host, copies pipelined both ways)"},
             "clocks": clk.summary(),
             "gpu_launches": args.steps * sum(o["launches"] for o in ops),
+            "paper_context": PAPER_CONTEXT,
         }
         print(json.dumps(line), flush=True)
     torch.cuda.synchronize()

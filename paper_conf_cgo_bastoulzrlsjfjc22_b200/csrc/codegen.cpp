@@ -1755,11 +1755,15 @@ struct Gen {
       // over few vectors) use compensated (Kahan) accumulation: the error of
       // a plain running sum grows with the count (R16's bound assumes a
       // short per-lane chain), Kahan's stays ~2u * sum|t| whatever the length.
-      const bool kahan = red && x.redop == FOP_RED_SUM && (SPL ? (NRO + SPL - 1) / SPL : NRO) * K * W > 128;
+      // integer reductions (R30): exact wrap-around, no Kahan, no packed fp32 pairs
+      const bool ired = red && x.out_dtype == FOP_I32;
+      const bool kahan = red && !ired && x.redop == FOP_RED_SUM && (SPL ? (NRO + SPL - 1) / SPL : NRO) * K * W > 128;
+      const std::string RADD = ired ? "fop::iadd(" : "__fadd_rn(", RMAX = ired ? "fop::imax(" : "fop::op_max(";
       if (red) {
         o.l(std::string("float acc") + num(x.stmt) + " = " +
-            (x.redop == FOP_RED_MAX ? "__uint_as_float(0xff800000u)" : "0.f") + ";");
-        if (x.redop == FOP_RED_SUM) o.l("u64 acc" + num(x.stmt) + "p = fop::pk1(0.f);");
+            (x.redop == FOP_RED_MAX ? (ired ? "__int_as_float(0x80000000)" : "__uint_as_float(0xff800000u)")
+                                    : (ired ? "__int_as_float(0)" : "0.f")) + ";");
+        if (x.redop == FOP_RED_SUM && !ired) o.l("u64 acc" + num(x.stmt) + "p = fop::pk1(0.f);");
         if (kahan) o.l("float acc" + num(x.stmt) + "c = 0.f; u64 acc" + num(x.stmt) + "cp = fop::pk1(0.f);");
       }
       if (x.kind == FOP_ASSIGN && x.fwd && regmode)
@@ -1910,8 +1914,8 @@ struct Gen {
           Sink sk;
           if (red) {
             bool mx = x.redop == FOP_RED_MAX;
-            sk.scalar = [&, A, mx](const std::string& v) {
-              o.l(A + " = " + (mx ? "fop::op_max(" : "__fadd_rn(") + A + ", " + v + ");");
+            sk.scalar = [&, A, mx, RADD, RMAX](const std::string& v) {
+              o.l(A + " = " + (mx ? RMAX : RADD) + A + ", " + v + ");");
             };
             if (kahan) {   // y = v - c; t = s + y; c = (t - s) - y; s = t
               sk.scalar = [&, A](const std::string& v) {
@@ -1926,7 +1930,7 @@ struct Gen {
                 o.l("{ const u64 y_ = fop::sub2(fop::mul2(" + a + ", " + b + "), " + A + "cp); const u64 t_ = fop::add2(" + A +
                     "p, y_); " + A + "cp = fop::sub2(fop::sub2(t_, " + A + "p), y_); " + A + "p = t_; }");
               };
-            } else if (!mx) {
+            } else if (!mx && !ired) {
               sk.pair = [&, A](const std::string& v, const std::string&) { o.l(A + "p = fop::add2(" + A + "p, " + v + ");"); };
               sk.pair_fma = [&, A](const std::string& a, const std::string& b, const std::string&) {
                 o.l(A + "p = fop::fma2(" + a + ", " + b + ", " + A + "p);");
@@ -1973,13 +1977,15 @@ struct Gen {
         if (kahan)   // each running sum minus its compensation, then combined
           o.l(a + " = __fadd_rn(__fsub_rn(" + a + ", " + a + "c), __fadd_rn(__fsub_rn(fop::lo(" + a + "p), fop::lo(" + a +
               "cp)), __fsub_rn(fop::hi(" + a + "p), fop::hi(" + a + "cp))));");
-        else if (x.redop == FOP_RED_SUM)
+        else if (x.redop == FOP_RED_SUM && !ired)
           o.l(a + " = __fadd_rn(" + a + ", __fadd_rn(fop::lo(" + a + "p), fop::hi(" + a + "p)));");
+        const std::string I = ired ? "i" : "";
         if (P > 1)
-          o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::group_max<" : "fop::group_sum<") + num(LN) + ">(" +
-              a + ");");
+          o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::group_" + I + "max<" : "fop::group_" + I + "sum<") +
+              num(LN) + ">(" + a + ");");
         else
-          o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::warp_max(" : "fop::warp_sum(") + a + ");");
+          o.l(a + " = " + std::string(x.redop == FOP_RED_MAX ? "fop::warp_" + I + "max(" : "fop::warp_" + I + "sum(") + a +
+              ");");
         if (G > 1) {   // the row's G warp partials, combined in warp order
           std::string rs = "RS" + num(x.stmt);
           o.l("if ((threadIdx.x & 31u) == 0u) " + rs + "[threadIdx.x >> 5] = " + a + ";");
@@ -1987,7 +1993,7 @@ struct Gen {
           o.l(a + " = " + rs + "[grp * " + num(G) + "u];");
           o.l("#pragma unroll");
           o.l("for (int g_ = 1; g_ < " + num(G) + "; ++g_) " + a + " = " +
-              (x.redop == FOP_RED_MAX ? "fop::op_max(" : "__fadd_rn(") + a + ", " + rs + "[grp * " + num(G) + "u + g_]);");
+              (x.redop == FOP_RED_MAX ? RMAX : RADD) + a + ", " + rs + "[grp * " + num(G) + "u + g_]);");
           o.l("__syncthreads();");
         }
         if (Q > 1) {   // the cluster's Q block partials, read from every CTA's shared memory in rank order
@@ -1997,7 +2003,7 @@ struct Gen {
           o.l(a + " = fop::ld_dsmem(&" + rq + ", 0u);");
           o.l("#pragma unroll");
           o.l("for (unsigned q_ = 1; q_ < " + num(Q) + "u; ++q_) " + a + " = " +
-              (x.redop == FOP_RED_MAX ? "fop::op_max(" : "__fadd_rn(") + a + ", fop::ld_dsmem(&" + rq + ", q_));");
+              (x.redop == FOP_RED_MAX ? RMAX : RADD) + a + ", fop::ld_dsmem(&" + rq + ", q_));");
           o.l("fop::cluster_sync();");
         }
         std::string res = fin_expr(o, x, a, "");
@@ -2026,8 +2032,11 @@ struct Gen {
     const int64_t RPC = (ROWS + NCH - 1) / NCH;
     const int SW = L.gv * W;
     bool isMax = x.redop == FOP_RED_MAX;
-    std::string init = isMax ? "__uint_as_float(0xff800000u)" : "0.f";
+    const bool ired = x.out_dtype == FOP_I32;   // integer reduction (R30): exact, any order
+    std::string init = isMax ? (ired ? "__int_as_float(0x80000000)" : "__uint_as_float(0xff800000u)")
+                             : (ired ? "__int_as_float(0)" : "0.f");
     auto comb = [&](const std::string& a, const std::string& b) {
+      if (ired) return (isMax ? "fop::imax(" : "fop::iadd(") + a + ", " + b + ")";
       return isMax ? "fop::op_max(" + a + ", " + b + ")" : "__fadd_rn(" + a + ", " + b + ")";
     };
     header("COL_REDUCE (slab of gv x W columns, row chunks, fixed-order trees)", 1);
@@ -2065,11 +2074,11 @@ struct Gen {
       o.l("const idx_t r1 = (r0 + " + num(RPC) + "u < " + num(ROWS) + "u) ? r0 + " + num(RPC) + "u : " + num(ROWS) +
           "u;");
     }
-    const bool packed = !isMax && W % 2 == 0 && g_packed;
+    const bool packed = !isMax && !ired && W % 2 == 0 && g_packed;
     // rows one lane accumulates in sequence; a long chain is summed with
     // compensation (Kahan), as in ROW_REDUCE
     const int64_t chain = (ROWS + NCH * (int64_t)L.gr - 1) / (NCH * (int64_t)L.gr);
-    const bool kahan = !isMax && chain > 128;
+    const bool kahan = !isMax && !ired && chain > 128;
     o.l("float acc[" + num(W) + "];");
     o.l("#pragma unroll");
     o.l("for (int e = 0; e < " + num(W) + "; ++e) acc[e] = " + init + ";");

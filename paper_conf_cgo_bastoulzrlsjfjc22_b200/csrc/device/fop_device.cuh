@@ -552,6 +552,30 @@ __device__ __forceinline__ float warp_max(float v) {
   for (int o = 16; o > 0; o >>= 1) v = op_max(v, __shfl_xor_sync(0xffffffffu, v, o));
   return v;
 }
+// int32 reductions (reading R30): wrap-around sums are exactly associative,
+// so every association order gives the oracle's bits
+__device__ __forceinline__ float warp_isum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = iadd(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ float warp_imax(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = imax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+template <int LN>
+__device__ __forceinline__ float group_isum(float v) {
+#pragma unroll
+  for (int o = LN / 2; o > 0; o >>= 1) v = iadd(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+template <int LN>
+__device__ __forceinline__ float group_imax(float v) {
+#pragma unroll
+  for (int o = LN / 2; o > 0; o >>= 1) v = imax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
 // butterflies over aligned groups of LN lanes (LN rows of a short-row kernel
 // share a warp: the xor offsets < LN never leave the group)
 template <int LN>

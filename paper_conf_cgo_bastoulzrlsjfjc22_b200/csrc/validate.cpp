@@ -211,8 +211,6 @@ void validate(const fop_desc& d) {
         if (!integer && st.fin[i].op == FOP_OP_CAST && st.fin[i].cvt == FOP_I32)
           fail(FOP_E_INVALID, where(s) + "cast to i32");
       }
-      if (integer && st.kind == FOP_REDUCE)
-        fail(FOP_E_UNSUPPORTED, where(s) + "i32 reductions (the oracle defines them; the kernels do not yet)");
     }
   }
 }

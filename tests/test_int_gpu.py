@@ -2,7 +2,9 @@
 neg abs relu and integral constants, wrap-around modulo 2^32 — bit-exact
 against the oracle (BASELINE.json north_star: "bit-exact for ... integer
 ops"), through every EW path: vector loop with broadcast, narrow (misaligned)
-variant, transposes, read-modify-write (Fig. 2's Y) and recurrences.
+variant, transposes, read-modify-write (Fig. 2's Y) and recurrences, and through
+the row and column reduction kernels (sums modulo 2^32 are exactly associative:
+every tuning candidate must give the oracle's bits).
 
 The statement model is the paper's (statements over tensors with affine
 accesses); the DAG's integer semantics are this
@@ -111,3 +113,41 @@ def test_int_recurrence_prefix_sum():
     got, op = run_gpu(d, x)
     assert op.info()["launches"][0]["seq"] == ["t"]
     assert_bitexact(got["y"], O.run(d, x)["y"], "y")
+
+
+def _ired(R, C, op, axis, expr=None):
+    return {"name": "ired", "loops": {"r": R, "c": C},
+            "tensors": {"x": _t([R, C]), "out": _t([C] if axis == "col" else [R], role="out")},
+            "stmts": [{"kind": "reduce", "op": op, "loops": ["r", "c"],
+                       "write": ("out", ["c"] if axis == "col" else ["r"]), "reads": [("x", ["r", "c"])],
+                       "expr": expr or [("load", 0), ("const", 3.0), ("mul", 0, 1)]}]}
+
+
+@pytest.mark.parametrize("R,C", [(65536, 1024), (1000, 13), (7, 40000), (100000, 8), (3, 5)])
+@pytest.mark.parametrize("op", ["sum", "max"])
+@pytest.mark.parametrize("axis", ["col", "row"])
+def test_int_reductions_bit_exact_every_candidate(R, C, op, axis):
+    """i32 REDUCE (R30): sums modulo 2^32 are exactly associative, so the row and column
+    kernels' butterflies, cross-warp / cluster / cross-chunk combines give the oracle's bits
+    in any order — checked for every auto-tuning candidate (different association orders)."""
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    d = _ired(R, C, op, axis)
+    x = {"x": _rand(R * C, 12)}
+    ref = O.run(d, x)["out"]
+    nv = FusedOp(d).info()["launches"][0]["nvariants"]
+    for k in range(nv):
+        got, op_ = run_gpu(d, x, variant=k)
+        assert_bitexact(got["out"], ref, f"candidate {k} {op_.selected(0)[0]}")
+    with np.errstate(over="ignore"):
+        m = x["x"].reshape(R, C).astype(np.int64) * 3
+        red = m.sum(0 if axis == "col" else 1) if op == "sum" else m.max(0 if axis == "col" else 1)
+    if op == "max":                                   # numpy: max of the wrapped products
+        red = ((x["x"].reshape(R, C) * np.int32(3)).astype(np.int32)).max(0 if axis == "col" else 1)
+    assert np.array_equal(got["out"], ((red + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(I32))
+
+
+def test_int_column_sum_misaligned_uses_the_narrow_variant():
+    d = _ired(777, 1001, "sum", "col", [("load", 0)])
+    x = {"x": _rand(777 * 1001, 13)}
+    got, op = run_gpu(d, x, offset=1)
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")

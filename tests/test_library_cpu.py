@@ -372,11 +372,11 @@ def _int_desc(expr, out="i32", xin="i32", kind="assign", write_idx=("i",)):
     (_int_desc([("load", 0), ("const", 1.0), ("add", 0, 1)], xin="f32"), "FOP_E_INVALID"),  # int stmt reads f32
     (_int_desc([("load", 0)], out="f32"), "FOP_E_INVALID"),                              # not a move: a conversion
     (_int_desc([("load", 0)]), None),                                                     # pure i32 move
-    (_int_desc([("load", 0)], kind="reduce"), "FOP_E_UNSUPPORTED"),                       # oracle-only for now
+    (_int_desc([("load", 0)], kind="reduce"), None),                                      # i32 column sum
 ])
 def test_integer_statement_rules_match_the_oracle(desc, status):
     """Reading R30: the product accepts exactly the integer statements the oracle defines
-    (tests/test_oracle_ops.py), except i32 reductions, which it reports unsupported."""
+    (tests/test_oracle_ops.py), reductions included."""
     from oracle import oracle as O
     x = {"a": np.arange(256, dtype=np.float32 if desc["tensors"]["a"]["dtype"] == "f32" else np.int32)}
     if status is None:

@@ -32,6 +32,31 @@ def _ulp16(a, b):
     return np.abs(ordered16(a) - ordered16(b))
 
 
+def _assert_lstm(d, x, got, ref):
+    """LSTM cell, fp32 outputs of transcendental compositions.  With u = 2^-24
+    and the CUDA math library's documented bounds (expf, tanhf <= 2 ulp = 4u relative):
+      sigmoid = 1/(1 + expf(-v)): <= 4u (expf, damped by e/(1+e)) + u (add) + u (rcp) = 6u;
+      A = sigmoid(f) c_prev: 7u;  B = sigmoid(i) tanh(g): 6u + 4u + u = 11u;
+      the oracle rounds each transcendental once (u) and each product (u): A 2u, B 3u;
+      c = A + B: |gpu - ref| <= 9u|A| + 14u|B| + 2u|c| <= 16u (|A| + |B|)  (no absolute floor:
+      the bound is normwise in the two products, which is where cancellation can hide);
+      h = sigmoid(o) tanh(c) reads each side's OWN stored c, |d tanh| <= |dc|:
+      |gpu - ref| <= 16u (|A| + |B|) + 16u |h| + 2^-149."""
+    u = 2.0 ** -24
+    B_, H = d["loops"]["b"], d["loops"]["h"]
+    g = x["g"].astype(np.float64).reshape(B_, 4 * H)
+    gi, gf, gg = g[:, :H], g[:, H:2 * H], g[:, 2 * H:3 * H]
+    sig = lambda t: 1.0 / (1.0 + np.exp(-t))  # noqa: E731
+    A = np.abs(sig(gf) * x["c_prev"].astype(np.float64).reshape(B_, H))
+    Bm = np.abs(sig(gi) * np.tanh(gg))
+    tol_c = (16 * u * (A + Bm)).reshape(-1)
+    gc, rc = got["c"].astype(np.float64), ref["c"].astype(np.float64)
+    assert np.all(np.abs(gc - rc) <= tol_c), float(np.max(np.abs(gc - rc) / tol_c))
+    gh, rh = got["h_out"].astype(np.float64), ref["h_out"].astype(np.float64)
+    tol_h = tol_c + 16 * u * np.abs(rh) + 2.0 ** -149
+    assert np.all(np.abs(gh - rh) <= tol_h), float(np.max(np.abs(gh - rh) / tol_h))
+
+
 def _assert_layernorm(d, x, got, ref):
     """y = t*gamma + beta with t = (x - mean)*rstd: mean and var are
     reductions (R16), so y may differ by 1 f16 ulp plus 1e-5 of the magnitudes
@@ -163,8 +188,8 @@ def test_n4_gpu_vs_oracle(name, full):
     ref = O.run(d, x)
     for n, v in got.items():
         if name == "lstm_cell":
-            err = np.abs(v.astype(np.float64) - ref[n].astype(np.float64))
-            assert np.all(err <= 4e-6 * np.abs(ref[n].astype(np.float64)) + 4e-6), (n, err.max())
+            _assert_lstm(d, x, got, ref)
+            break
         elif name in ("bert_layernorm", "wide_layernorm"):
             _assert_layernorm(d, x, v, ref[n])
         elif name in ("bert_softmax", "vocab_softmax"):
