@@ -143,6 +143,7 @@ def test_int_reductions_bit_exact_every_candidate(R, C, op, axis):
         red = m.sum(0 if axis == "col" else 1) if op == "sum" else m.max(0 if axis == "col" else 1)
     if op == "max":                                   # numpy: max of the wrapped products
         red = ((x["x"].reshape(R, C) * np.int32(3)).astype(np.int32)).max(0 if axis == "col" else 1)
+    red = red.astype(np.int64)
     assert np.array_equal(got["out"], ((red + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(I32))
 
 
