@@ -430,7 +430,10 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     // (a long odd d_v, e.g. C = 255, puts the read-out's consecutive lanes 8
     // tile rows apart, on few shared-memory banks: 1104 GB/s, still above the
     // gathering elementwise kernel's 958 — profiles/odd_variety_r01.log)
-    if (W == 1 && wr >= 2 && !L.scalar_variant && L.kl[0].extent <= geometry_knob(L, "FOP_TR_SMEM_MAXV", 1 << 30) &&
+    // (FOP_TR_SMEM_OUT=1 takes this path even when d_v could carry store vectors: an ablation/tuning
+    // candidate for ordinary transposes such as cfg3)
+    if ((W == 1 || geometry_knob(L, "FOP_TR_SMEM_OUT", 0)) && wr >= 2 && !L.scalar_variant &&
+        L.kl[0].extent <= geometry_knob(L, "FOP_TR_SMEM_MAXV", 1 << 30) &&
         geometry_knob(L, "FOP_TR_SMEM", 1)) {
       // the mirror case: d_v rows too short/odd for store vectors (an input
       // layer's C = 3; NHWC -> NCHW of a 7x7 plane), but the output rows are
