@@ -1,5 +1,12 @@
 python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
-timeout 900 python -m pytest tests/test_odd_gpu.py -q -x -k "column" > gpurun_out/pytest_colodd.log 2>&1; echo pytest=$?
+timeout 900 python -m pytest tests/test_odd_gpu.py tests/test_int_gpu.py -q -x -k "column or reduction" > gpurun_out/pytest_colodd.log 2>&1; echo pytest=$?
 tail -3 gpurun_out/pytest_colodd.log
-timeout 600 python tools/odd_variety.py > gpurun_out/odd_variety_r02.log 2>&1; echo odd=$?
-head -3 gpurun_out/odd_variety_r02.log
+S="timeout 600 python tools/sweep.py"
+A="opt:autotune=0"
+for op in colsum_1001; do $S $op "$A" "$A,FOP_COL_XCHG=0" "$A,FOP_COL_U=8,FOP_COL_MINB=4" "$A,FOP_COL_U=2,FOP_COL_MINB=8" "$A,FOP_COL_U=4,FOP_COL_MINB=4"; done > gpurun_out/sweep_colx.log 2>&1
+grep "^{" gpurun_out/sweep_colx.log | python -c "
+import sys, json
+for l in sys.stdin:
+    j=json.loads(l)
+    print(j['op'], j['variant'][:80].ljust(80), '%.0f' % j.get('GBs_median',0), '%.1f' % j.get('us_median',0), j.get('grid'), j.get('error','')[:200])
+"
