@@ -126,7 +126,16 @@ def random_op(rng):
         for k in range(len(reads)):   # every load used
             expr.append(("add", last, k))
             last = len(expr) - 1
-        stmts.append({"kind": "assign", "loops": names, "write": ("out", list(perm)), "reads": reads, "expr": expr})
+        if rng.random() < 0.35 and len(names) > 1:   # an integer REDUCE over some loops (wrap-around, exact)
+            red = [n for n in names if rng.random() < 0.5] or [names[-1]]
+            keep = [n for n in names if n not in red] or [names[0]]
+            red = [n for n in names if n not in keep]
+            tensors["out"] = _tensor(rng, loops, keep, "i32", "out", 0, pad=False)
+            stmts.append({"kind": "reduce", "op": "max" if rng.random() < 0.3 else "sum", "loops": names,
+                          "write": ("out", list(keep)), "reads": reads, "expr": expr})
+        else:
+            stmts.append({"kind": "assign", "loops": names, "write": ("out", list(perm)), "reads": reads,
+                          "expr": expr})
     elif pat == "assign":
         reads = inputs(int(rng.integers(1, 4)))
         perm = list(rng.permutation(names)) if rng.random() < 0.5 else names

@@ -48,7 +48,7 @@ def compare(d, x, got, ref):
             continue
         from_sum = any(q["kind"] == "reduce" and q.get("op", "sum") == "sum" and
                        any(r[0] == q["write"][0] for r in st["reads"]) for q in d["stmts"][:si])
-        if st["kind"] == "reduce" and st.get("op", "sum") == "sum":
+        if st["kind"] == "reduce" and st.get("op", "sum") == "sum" and t["dtype"] != "i32":   # (i32: exact)
             assert_normwise(got[n], ref[n], O.run(abs_terms_desc(d, si), x)[n], 1e-5, n)
         elif from_sum and t["dtype"] == "f32":
             g, r = got[n].astype(np.float64), ref[n].astype(np.float64)
