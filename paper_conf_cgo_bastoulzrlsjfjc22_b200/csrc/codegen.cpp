@@ -1185,6 +1185,174 @@ struct Gen {
     footer();
   }
 
+  // ------------------------------------------------------------ TRANSPOSE, software-pipelined
+  // The register transpose with the NEXT grid-stride iteration's tile loads
+  // issued before the current tiles are converted and stored (FOP_TR_PIPE=1):
+  // the thread's loads never drain between iterations.  Two register sets
+  // (current / next) of raw words; same tiles, same arithmetic, same bits.
+  bool transpose_pipe_ok() const {
+    const XStmt& x = L.stmts[0];
+    if (x.move || !geometry_knob(L, "FOP_TR_PIPE", 0)) return false;
+    for (const auto& a : L.loads) {
+      int64_t cv = C(a, 0), cr = C(a, 1);
+      int cb = cv == 1 ? 0 : 0;
+      (void)cb;
+      if (cv == 1 || cr == 1) {
+        const int n_in = cv == 1 ? L.width : L.read_width;
+        const int c_ = cv == 1 ? -1 : -2;
+        (void)c_;
+        if (n_in * es(a.tensor) < 4) return false;
+      } else if (!(cv == 0 && cr == 0)) {
+        return false;   // gathers: not pipelined
+      }
+    }
+    return true;
+  }
+  void gen_transpose_pipe() {
+    const int W = L.width, WR = L.read_width;
+    const int U = std::max(1, L.unroll);
+    const int64_t NTV = L.kl[0].extent / W, NTR = L.kl[1].extent / WR;
+    const int64_t TVH = (NTV + L.gv - 1) / L.gv;
+    const int64_t TRH = (NTR + (int64_t)L.gr * U - 1) / ((int64_t)L.gr * U);
+    const int64_t STRIDE = L.grid * L.block;
+    const XStmt& x = L.stmts[0];
+    header("TRANSPOSE (register tiles W x WR, U per thread, next iteration's loads in flight)", 1);
+    const int NO = (int)L.kl.size() - 2;   // outer kernel loops
+    std::vector<char> kind(L.loads.size(), 'S');
+    std::vector<int> wpv(L.loads.size(), 0), n_in(L.loads.size(), 0), n_out(L.loads.size(), 0);
+    for (size_t k = 0; k < L.loads.size(); k++) {
+      const int64_t cv = C(L.loads[k], 0), cr = C(L.loads[k], 1);
+      if (cv == 1 || cr == 1) {
+        kind[k] = cv == 1 ? 'A' : 'B';
+        n_in[k] = cv == 1 ? W : WR;
+        n_out[k] = cv == 1 ? WR : W;
+        wpv[k] = n_in[k] * es(L.loads[k].tensor) / 4;
+      }
+    }
+    // state of one fetched iteration: iv, outer iterators, per u: ir, ok, the raw words
+    for (const std::string S : {"_c", "_n"}) {
+      o.l("idx_t iv" + S + " = 0;");
+      for (int q = 0; q < NO; q++) o.l("idx_t i" + num(q + 2) + S + " = 0;");
+      for (int u = 0; u < U; u++) {
+        o.l("idx_t ir_" + num(u) + S + " = 0; bool ok_" + num(u) + S + " = false;");
+        for (size_t k = 0; k < L.loads.size(); k++)
+          if (wpv[k]) o.l("u32 WL" + num(k) + "_" + num(u) + S + "[" + num(n_out[k]) + "][" + num(wpv[k]) + "];");
+      }
+    }
+    auto fetch = [&](const std::string& g, const std::string& S) {
+      o.l("{");
+      o.ind++;
+      o.l("idx_t t = " + g + ";");
+      o.l("const idx_t tv_lo = t % " + num(L.gv) + "u; t /= " + num(L.gv) + "u;");
+      o.l("const idx_t tr_lo = t % " + num(L.gr) + "u; t /= " + num(L.gr) + "u;");
+      o.l("const idx_t tv_hi = t % " + num(TVH) + "u; t /= " + num(TVH) + "u;");
+      if (NO > 0) o.l("const idx_t tr_hi = t % " + num(TRH) + "u; t /= " + num(TRH) + "u;");
+      else o.l("const idx_t tr_hi = t;");
+      o.l("const idx_t tv = tv_hi * " + num(L.gv) + "u + tv_lo;");
+      o.l("const bool okv = " + g + " < (idx_t)" + num(L.work) + "ull && tv < " + num(NTV) + "u;");
+      o.l("iv" + S + " = tv * " + num(W) + "u;");
+      for (int q = 0; q < NO; q++) {
+        if (q == NO - 1) o.l("i" + num(q + 2) + S + " = t;");
+        else o.l("i" + num(q + 2) + S + " = t % " + num(L.kl[q + 2].extent) + "u; t /= " + num(L.kl[q + 2].extent) + "u;");
+      }
+      for (int u = 0; u < U; u++) {
+        const std::string us = "_" + num(u) + S;
+        o.l("{ const idx_t tr = tr_hi * " + num((int64_t)L.gr * U) + "u + " + num((int64_t)u * L.gr) + "u + tr_lo;");
+        o.l("  ok" + us + " = okv && tr < " + num(NTR) + "u; ir" + us + " = tr * " + num(WR) + "u; }");
+        std::vector<std::pair<int, std::string>> its = {{0, "iv" + S}, {1, "ir" + us}};
+        for (int q = 0; q < NO; q++) its.push_back({q + 2, "i" + num(q + 2) + S});
+        for (size_t k = 0; k < L.loads.size(); k++) {
+          if (!wpv[k]) continue;
+          const Affine& a = L.loads[k];
+          const bool A = kind[k] == 'A';
+          const int cb = A ? L.load_cb[k] : L.load_cb_r[k];
+          const int64_t step = A ? C(a, 1) : C(a, 0);
+          const std::string vl = A ? "b" : "a";
+          o.l("#pragma unroll");
+          o.l("for (int " + vl + " = 0; " + vl + " < " + num(n_out[k]) + "; ++" + vl + ") if (ok" + us +
+              ") fop::vload_words<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + num(n_in[k]) + ", " + num(cb) +
+              ", " + pol(a, false) + ">(WL" + num(k) + us + "[" + vl + "], " +
+              ptr(a.tensor, affine(a, its) + " + " + vl + " * " + num(step)) + ");");
+        }
+      }
+      o.ind--;
+      o.l("}");
+    };
+    o.l("const idx_t tid = (idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x;");
+    fetch("tid", "_c");
+    o.l("#pragma unroll 1");
+    o.l("for (idx_t g = tid; g < (idx_t)" + num(L.work) + "ull; g += (idx_t)" + num(STRIDE) + "ull) {");
+    o.ind++;
+    fetch("(g + (idx_t)" + num(STRIDE) + "ull)", "_n");
+    int64_t cwr = C(x.write, 1);
+    std::string dto = dtn(x.out_dtype);
+    for (int u = 0; u < U; u++) {
+      const std::string t = "_" + num(u) + "_c";
+      std::vector<std::pair<int, std::string>> its = {{0, "iv_c"}, {1, "ir" + t}};
+      for (int q = 0; q < NO; q++) its.push_back({q + 2, "i" + num(q + 2) + "_c"});
+      o.l("if (ok" + t + ") {");
+      o.ind++;
+      for (size_t k = 0; k < L.loads.size(); k++) {
+        const std::string nm = "L" + num(k) + t;
+        if (wpv[k]) {
+          o.l("float " + nm + "[" + num(n_out[k]) + "][" + num(n_in[k]) + "];");
+          o.l("#pragma unroll");
+          o.l("for (int q = 0; q < " + num(n_out[k]) + "; ++q) fop::cvt_words<" +
+              std::string(dtn(d.t[L.loads[k].tensor].dtype)) + ", " + num(n_in[k]) + ">(" + nm + "[q], W" + nm + "[q]);");
+        } else {   // a scalar (constant over the tile)
+          o.l("const float " + nm + " = fop::sload<" + std::string(dtn(d.t[L.loads[k].tensor].dtype)) + ", " +
+              pol(L.loads[k], true) + ">(" + ptr(L.loads[k].tensor, affine(L.loads[k], its)) + ");");
+        }
+      }
+      DagCtx c;
+      c.tag = t;
+      c.ev = "a";
+      c.load_varies = [&](int k) { return kind[k] != 'S'; };
+      c.load = [&, t](int k, const std::string& e) {
+        std::string nm = "L" + num(k) + t;
+        switch (kind[k]) {
+          case 'A': return nm + "[b][" + e + "]";
+          case 'S': return nm;
+          default: return nm + "[" + e + "][b]";
+        }
+      };
+      c.fwd = [&](int, const std::string&) { return std::string("0.f"); };
+      c.scalar = [&](int) { return std::string("0.f"); };
+      auto var = varies(x, c);
+      emit_nodes(o, x, var, false, c);
+      o.l("float O[" + num(WR) + "][" + num(W) + "];");
+      o.l("#pragma unroll");
+      o.l("for (int b = 0; b < " + num(WR) + "; ++b) {");
+      o.ind++;
+      Sink sk;
+      sk.scalar = [&](const std::string& v) { o.l("O[b][a] = " + v + ";"); };
+      sk.pair = [&](const std::string& v, const std::string& p) {
+        o.l("fop::upk(" + v + ", O[b][2 * " + p + "], O[b][2 * " + p + " + 1]);");
+      };
+      emit_elems(o, x, var, c, W, sk);
+      o.ind--;
+      o.l("}");
+      o.l("#pragma unroll");
+      o.l("for (int b = 0; b < " + num(WR) + "; ++b) fop::vstore<" + dto + ", " + num(W) + ", " + num(L.store_cb[0]) +
+          ", " + spol() + ">(" + ptr(x.write.tensor, affine(x.write, its) + " + b * " + num(cwr)) + ", O[b]);");
+      o.ind--;
+      o.l("}");
+    }
+    // the next iteration becomes the current one
+    o.l("iv_c = iv_n;");
+    for (int q = 0; q < NO; q++) o.l("i" + num(q + 2) + "_c = i" + num(q + 2) + "_n;");
+    for (int u = 0; u < U; u++) {
+      o.l("ir_" + num(u) + "_c = ir_" + num(u) + "_n; ok_" + num(u) + "_c = ok_" + num(u) + "_n;");
+      for (size_t k = 0; k < L.loads.size(); k++)
+        if (wpv[k])
+          o.l("#pragma unroll\nfor (int q = 0; q < " + num(n_out[k]) + "; ++q)\n#pragma unroll\nfor (int w = 0; w < " +
+              num(wpv[k]) + "; ++w) WL" + num(k) + "_" + num(u) + "_c[q][w] = WL" + num(k) + "_" + num(u) + "_n[q][w];");
+    }
+    o.ind--;
+    o.l("}");
+    footer();
+  }
+
   // ------------------------------------------------------------ TRANSPOSE via shared memory
   // For d_r rows too short or odd to carry vectors (a 7x7 plane: 49
   // elements, 98 B rows) whose d_v rows are adjacent in the load tensor: a
@@ -2638,6 +2806,7 @@ std::string generate(const Plan& p, Launch& L, int launch_index) {
     case FOP_CLASS_TRANSPOSE:
       if (L.tma) g.gen_transpose_tma();
       else if (L.tr_smem) g.gen_transpose_smem();
+      else if (g.transpose_pipe_ok()) g.gen_transpose_pipe();
       else g.gen_transpose();
       break;
     case FOP_CLASS_ROW_REDUCE: g.gen_row(); break;

@@ -126,3 +126,19 @@ def test_column_sum_of_squares_odd_rows_every_candidate():
         op.run(dev)
         torch.cuda.synchronize()
         assert_normwise(to_host(dev["out"], "f32"), ref, scale, 1e-5, f"candidate {k}")
+
+
+@pytest.mark.parametrize("dims,dtype", [((2, 256, 56, 56), "f16"), ((1, 40, 9, 16), "f32"), ((3, 64, 8, 8), "bf16")])
+@pytest.mark.parametrize("knobs", ["FOP_TR_PIPE=1", "FOP_TR_PIPE=1,FOP_TR_U=1", "FOP_TR_PIPE=1,FOP_TR_U=1,FOP_TR_MINB=2"])
+def test_transpose_software_pipelined_bitexact(monkeypatch, dims, dtype, knobs):
+    """The register transpose with the next grid-stride iteration's loads issued before the
+    current tiles are stored (FOP_TR_PIPE): same tiles, same arithmetic, same bits."""
+    for kv in knobs.split(","):
+        k, v = kv.split("=")
+        monkeypatch.setenv(k, v)
+    d = W.cfg3(*dims, dtype=dtype)
+    d["tensors"]["x"]["init"] = ("special", 9)
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x, autotune=0)
+    assert "next iteration's loads in flight" in op.source()
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")
