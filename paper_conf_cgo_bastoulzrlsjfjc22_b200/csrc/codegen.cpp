@@ -1194,14 +1194,9 @@ struct Gen {
     const XStmt& x = L.stmts[0];
     if (x.move || !geometry_knob(L, "FOP_TR_PIPE", 0)) return false;
     for (const auto& a : L.loads) {
-      int64_t cv = C(a, 0), cr = C(a, 1);
-      int cb = cv == 1 ? 0 : 0;
-      (void)cb;
+      const int64_t cv = C(a, 0), cr = C(a, 1);
       if (cv == 1 || cr == 1) {
-        const int n_in = cv == 1 ? L.width : L.read_width;
-        const int c_ = cv == 1 ? -1 : -2;
-        (void)c_;
-        if (n_in * es(a.tensor) < 4) return false;
+        if ((cv == 1 ? L.width : L.read_width) * es(a.tensor) < 4) return false;   // raw words need >= 4 B
       } else if (!(cv == 0 && cr == 0)) {
         return false;   // gathers: not pipelined
       }
