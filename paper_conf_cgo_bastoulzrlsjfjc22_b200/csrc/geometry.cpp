@@ -303,8 +303,8 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       for (size_t k = 0; k < L.loads.size() && ok; k++) {
         const int64_t c0 = coef(L, L.loads[k], 0), c1 = coef(L, L.loads[k], 1);
         if (c0 == 1 && c1 == E0) nflat++;
-        else if (c1 == 0) L.period_load[k] = 1;
-        else ok = false;
+        else if (c1 == 0 && c0 != 0) L.period_load[k] = 1;   // varies with c only: read at flat mod E[c]
+        else if (c1 != 0 || c0 != 0) ok = false;              // (c0 == c1 == 0: a scalar along both, kept)
       }
       for (const auto& x : L.stmts)
         ok &= coef(L, x.write, 0) == 1 && coef(L, x.write, 1) == E0;

@@ -426,6 +426,12 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
     if (footprint < (int64_t)kTuneColdBytes && !std::getenv("FOP_TUNE_HOT")) {
       flush = l2_flush_fn(l);
       if (flush && c.mem_alloc(&scratch, kTuneScratchBytes) != 0) scratch = 0;   // no room: time L2-hot
+      // defined contents: the flush kernel only reads it to evict L2, but compute-sanitizer's
+      // initcheck (rightly) reports reads of never-written memory
+      if (scratch && c.memset8(scratch, 0, kTuneScratchBytes) != 0) {
+        c.mem_free(scratch);
+        scratch = 0;
+      }
     }
     // steady state of a pipeline: the inputs are not in L2 and the previous
     // launch's outputs are still dirty in it (written back during this one)

@@ -143,3 +143,31 @@ def test_fuzz_regressions():
                 else:
                     os.environ[k] = v
         assert_normwise(got["out"], O.run(d, x)["out"], O.run(abs_terms_desc(d, 0), x)["out"], 1e-5, "out")
+
+
+def _regression_descs():
+    import glob
+    import json
+    import os
+    here = os.path.join(os.path.dirname(os.path.abspath(__file__)), "fuzz_regressions")
+    return [(os.path.basename(p), json.load(open(p))) for p in sorted(glob.glob(os.path.join(here, "*.json")))]
+
+
+@pytest.mark.parametrize("name,d", _regression_descs())
+def test_fuzz_regression_descriptors_compile(name, d):
+    """Operators a fuzz campaign broke (JSON under tests/fuzz_regressions/): they plan and compile
+    for sm_100a.  period_scalar_*: an EW statement flattened over an odd innermost extent that also
+    reads a tensor constant along both flattened loops (round 2, seeds 35 and 37: the scalar was
+    emitted as a per-element array)."""
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    FusedOp(d)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("name,d", _regression_descs())
+def test_fuzz_regression_descriptors_match_oracle(name, d):
+    import sys
+    import os
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools"))
+    from fuzz_campaign import check
+    check(d, repeat=True)
