@@ -2301,7 +2301,16 @@ struct Gen {
             // for each row's load, serialising the batch's latency)
             o.l("  u32 V_[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};");
             o.l("  if (okc && rr < r1) {");
-            o.l("    fop::ldraw<16, " + pol(a, false) + ">(V_, T" + num(a.tensor) + " + (u64)a_ * " + num(esk) + "u);");
+            // (the last row's last window may end past the tensor: read only its elements)
+            o.l("    if (a_ + " + num(W) + "u <= (idx_t)" + num(span) + "ull) fop::ldraw<16, " + pol(a, false) +
+                ">(V_, T" + num(a.tensor) + " + (u64)a_ * " + num(esk) + "u);");
+            if (esk == 2)
+              o.l("    else for (int e = 0; e < " + num(W) + "; ++e) if (a_ + e < (idx_t)" + num(span) +
+                  "ull) V_[e >> 1] |= (u32)fop::ld16<" + pol(a, false) + ">(T" + num(a.tensor) + " + (u64)(a_ + e) * 2u) << "
+                  "((e & 1) * 16);");
+            else
+              o.l("    else for (int e = 0; e < " + num(W) + "; ++e) if (a_ + e < (idx_t)" + num(span) + "ull) fop::ldraw<4, " +
+                  pol(a, false) + ">(V_ + e, T" + num(a.tensor) + " + (u64)(a_ + e) * 4u);");
             o.l("    if (m_ != 0u) {");
             o.l("      if (a_ + " + num(2 * W) + "u <= (idx_t)" + num(span) + "ull) fop::ldraw<16, " + pol(a, false) +
                 ">(V_ + 4, T" + num(a.tensor) + " + (u64)(a_ + " + num(W) + "u) * " + num(esk) + "u);");
