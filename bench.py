@@ -271,6 +271,33 @@ def to_device(buf, dtype, device):
     return torch.from_numpy(np.ascontiguousarray(buf)).to(device)
 
 
+def _peer_self_test(dist, world, rank, dev):
+    """One fused-exchange column sum on a small sharded problem; (ok, why)."""
+    import torch
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc, PeerExchange
+    px = None
+    try:
+        d, _ = shard_desc(W.cfg4b(R=2048 * world, C=1024), "r", rank, world, fused=True)
+        op = FusedOp(d, peer_world=world, peer_loop="r", peer_timeout_ms=2000)
+        px = PeerExchange(op.peer_bytes)
+        x = torch.ones(2048 * 1024, dtype=torch.float16, device=dev)
+        out = torch.zeros(1024, dtype=torch.float32, device=dev)
+        op.run({"x": x, "out": out}, peers=px.peers)
+        torch.cuda.synchronize()
+        if not bool((out == float(2048 * world)).all()):
+            return False, f"column sums {out[:4].tolist()} != {2048 * world}"
+        return True, ""
+    except Exception as e:  # noqa: BLE001 — reported in the bench line, never silent
+        return False, f"{type(e).__name__}: {e}"[:200]
+    finally:
+        if px is not None:
+            try:
+                px.close()
+            except Exception:  # noqa: BLE001
+                pass
+
+
 def run_fop(args):
     import torch
     import torch.distributed as dist
@@ -294,6 +321,20 @@ def run_fop(args):
 
     from paper_conf_cgo_bastoulzrlsjfjc22_b200.dist import shard_desc, allreduce_partials, PeerExchange
     peer = world > 1 and args.exchange == "peer"
+    exchange_note = None
+    if peer:
+        # The fused cross-GPU exchange has only ever run between ranks sharing one GPU (the build boxes
+        # have one): before timing, every rank runs it once on a small sharded column sum with a 2 s
+        # bound on the device wait and checks the result; if any rank fails (IPC mapping, peer access,
+        # a wait that times out), all ranks time the NCCL all-reduce path instead and the line says why.
+        ok, why = _peer_self_test(dist, world, rank, dev)
+        flag = torch.tensor([1 if ok else 0], dtype=torch.int32, device=dev)
+        flag = flag.cpu() if dist.get_backend() == "gloo" else flag
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if int(flag.item()) == 0:
+            peer = False
+            exchange_note = "nccl: the in-kernel peer exchange failed its self-test on some rank" + \
+                            (f" (rank {rank}: {why})" if why else "")
     ops = []
     order = args.op_order.split(",")
     if sorted(order) != sorted(n for n, _, _ in OPS):
@@ -577,6 +618,7 @@ def run_fop(args):
                 "workload": WORKLOAD if args.scaling == "weak" else WORKLOAD_STRONG,
                 "global_batch_scale": gscale,
                 "exchange_check": exchange_check,
+                "exchange_note": exchange_note,
                 "op_order": [o["name"] for o in ops],
                 "parallelism": ("dp%d (batch-sharded; " % world) + (
                     "no exchange)" if world == 1 else
