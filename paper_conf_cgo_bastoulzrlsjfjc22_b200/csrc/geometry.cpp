@@ -167,11 +167,13 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
         v.push_back({{"FOP_TR_SMEM_BYTES", 16384}, {"FOP_TR_SMEM_MINB", 8}});
         break;
       }
-      v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 2}});
-      v.push_back({{"FOP_TR_U", 2}, {"FOP_TR_MINB", 2}});
-      v.push_back({{"FOP_TR_U", 1}, {"FOP_TR_MINB", 3}});
-      // 32-byte stores along d_v over 16-byte loads along d_r (cfg3 5986 -> 6028 GB/s)
-      v.push_back({{"FOP_VEC_BYTES", 32}, {"FOP_TR_WR_BYTES", 16}, {"FOP_TR_U", 1}, {"FOP_TR_MINB", 1}});
+      v.push_back({{"FOP_BLOCK", 256}, {"FOP_TR_MINB", 1}});                       // round 1's default
+      v.push_back({{"FOP_BLOCK", 128}, {"FOP_TR_MINB", 2}});
+      v.push_back({{"FOP_BLOCK", 256}, {"FOP_TR_U", 1}, {"FOP_TR_MINB", 2}});
+      v.push_back({{"FOP_BLOCK", 32}, {"FOP_TR_MINB", 8}});
+      // 32-byte stores along d_v over 16-byte loads along d_r (cfg3 6088 GB/s at 2 x 128 threads)
+      v.push_back({{"FOP_VEC_BYTES", 32}, {"FOP_TR_WR_BYTES", 16}, {"FOP_TR_U", 1}, {"FOP_BLOCK", 128},
+                   {"FOP_TR_MINB", 2}});
       break;
     case FOP_CLASS_ROW_REDUCE:
       if (L.row_g > 1) {   // few long rows: neighbouring warps-per-row counts
@@ -607,7 +609,11 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       tvh = (tvh + BV - 1) / BV * BV;
     }
     L.work = (int64_t)gv * L.gr * tvh * trh * prod_rest;
-    L.minblocks = knob("FOP_TR_MINB", L.unroll >= 2 ? 1 : 2);
+    // 8 warps per SM (16 at U = 1) in small CTAs: 64-thread CTAs x 4 per SM measured +1.4 % over
+    // one 256-thread CTA on cfg3 (6097 vs 6013 GB/s, profiles/r02/sweep_r02_trblock.log) — CTAs
+    // retire independently, so the grid's tail is finer
+    L.block = knob("FOP_BLOCK", 64);
+    L.minblocks = knob("FOP_TR_MINB", std::max(1, (L.unroll >= 2 ? 8 : 16) * 32 / L.block));
     int64_t need = (L.work + L.block - 1) / L.block;
     L.grid = std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * L.minblocks));
 
