@@ -169,8 +169,11 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       }
       v.push_back({{"FOP_BLOCK", 256}, {"FOP_TR_MINB", 1}});                       // round 1's default
       v.push_back({{"FOP_BLOCK", 128}, {"FOP_TR_MINB", 2}});
-      v.push_back({{"FOP_BLOCK", 256}, {"FOP_TR_U", 1}, {"FOP_TR_MINB", 2}});
       v.push_back({{"FOP_BLOCK", 32}, {"FOP_TR_MINB", 8}});
+      // round 1's candidates (more warps per SM: f32 data, 2-D transposes, C = 96)
+      v.push_back({{"FOP_BLOCK", 256}, {"FOP_TR_U", 1}, {"FOP_TR_MINB", 2}});
+      v.push_back({{"FOP_BLOCK", 256}, {"FOP_TR_U", 2}, {"FOP_TR_MINB", 2}});
+      v.push_back({{"FOP_BLOCK", 256}, {"FOP_TR_U", 1}, {"FOP_TR_MINB", 3}});
       // 32-byte stores along d_v over 16-byte loads along d_r (cfg3 6088 GB/s at 2 x 128 threads)
       v.push_back({{"FOP_VEC_BYTES", 32}, {"FOP_TR_WR_BYTES", 16}, {"FOP_TR_U", 1}, {"FOP_BLOCK", 128},
                    {"FOP_TR_MINB", 2}});
