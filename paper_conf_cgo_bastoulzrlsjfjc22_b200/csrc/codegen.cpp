@@ -2228,10 +2228,15 @@ struct Gen {
     // contiguous: chunk c owns rows [c*RPC, (c+1)*RPC).  Both are fixed
     // assignments, so the summation order is fixed run to run.
     const bool il = L.col_il && NCH > 1;
-    const int64_t RSTEP = il ? NCH * (int64_t)L.gr : (int64_t)L.gr;   // between the U rows of a batch
+    // FOP_COL_FIN=3: the slab's last chunk block streams no rows — it only waits for the others'
+    // flag words and combines them, so the combine starts as soon as the slowest partial lands
+    const bool pure_fin = L.col_fin == 3 && NCH > 2;
+    const int64_t NCS = pure_fin ? NCH - 1 : NCH;   // chunks that stream rows
+    const int64_t RSTEP = il ? NCS * (int64_t)L.gr : (int64_t)L.gr;   // between the U rows of a batch
     if (il) {
       o.l("const idx_t r0 = chunk * " + num(L.gr) + "u;");
-      o.l("const idx_t r1 = " + num(ROWS) + "u;");
+      o.l(std::string("const idx_t r1 = ") + (pure_fin ? "chunk == " + num(NCH - 1) + "u ? 0u : " : "") + num(ROWS) +
+          "u;");
     } else {
       o.l("const idx_t r0 = chunk * " + num(RPC) + "u;");
       o.l("const idx_t r1 = (r0 + " + num(RPC) + "u < " + num(ROWS) + "u) ? r0 + " + num(RPC) + "u : " + num(ROWS) +
@@ -2240,7 +2245,7 @@ struct Gen {
     const bool packed = !isMax && !ired && W % 2 == 0 && g_packed;
     // rows one lane accumulates in sequence; a long chain is summed with
     // compensation (Kahan), as in ROW_REDUCE
-    const int64_t chain = (ROWS + NCH * (int64_t)L.gr - 1) / (NCH * (int64_t)L.gr);
+    const int64_t chain = (ROWS + NCS * (int64_t)L.gr - 1) / (NCS * (int64_t)L.gr);
     const bool kahan = !isMax && !ired && chain > 128;
     o.l("float acc[" + num(W) + "];");
     o.l("#pragma unroll");
@@ -2626,7 +2631,7 @@ struct Gen {
       // cfg4b: 27.2 us (1) vs 25.3 us for the fence + counter scheme — the
       // designated block is not the last to finish, so its poll loop sits on
       // the critical path (profiles/r02/sweep_r02_colfin.log).
-      const int FM = L.col_fin;
+      const int FM = L.col_fin == 3 ? 1 : L.col_fin;   // 3: mode 1 with a pure finalizer (no rows of its own)
       const std::string OWN = FM == 1 ? "c == " + num(NCH - 1) + "u" : "false";
       o.l("u64* partw = (u64*)(args.ws + " + num((int64_t)L.ws_off) + "ull);");
       o.l(std::string("if (rl == 0u") + (FM == 1 ? " && chunk != " + num(NCH - 1) + "u" : "") + ") {");
@@ -2674,7 +2679,7 @@ struct Gen {
       o.l("  asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t_));");
       o.l("  if (t0_ == 0ull) t0_ = t_;");
       o.l("  else if (t_ - t0_ > 4000000000ull) break;   // a word that never arrives: NaN, not a hang");
-      o.l("  __nanosleep(ns_);");
+      if (!geometry_knob(L, "FOP_COL_SPIN", 0)) o.l("  __nanosleep(ns_);");   // (1: spin without sleeping)
       o.l("  if (ns_ < 256u) ns_ *= 2u;");
       o.l("  #pragma unroll");
       o.l("  for (int it = 0; it < " + num(MAXIT) + "; ++it) {");

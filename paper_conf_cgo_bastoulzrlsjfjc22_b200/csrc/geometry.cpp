@@ -774,6 +774,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     if (nch > 1 && L.col_fin) {
       L.ws_bytes = ((size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(unsigned long long) + 255) & ~size_t(255);
       if (L.col_fin == 2) L.ws_bytes += (size_t)slabs * sizeof(unsigned);
+      if (L.col_fin == 3 && !L.col_il) L.col_fin = 1;   // the pure finalizer needs interleaved chunks
     } else if (nch > 1) {
       size_t part = (size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(float);
       part = (part + 255) & ~size_t(255);
