@@ -2277,6 +2277,15 @@ struct Gen {
       else if (cv != 0) pipe = false;
     }
     const int64_t BSTEP = RSTEP * U;
+    // col_shift with the second chunk taken from the neighbouring lane (FOP_COL_SHFL=1, ablation): every
+    // row's own chunk is loaded first, the whole batch in flight, then each row's window is assembled by
+    // a shuffle inside the row's gv-lane segment; only the segment's last lane and a lane whose neighbour
+    // has no vector load a second chunk.  Measured 1.7-3.4 TB/s on [65536,1001] f16 vs 3.2-3.9 for two
+    // chunk loads per lane (the per-row window registers cost occupancy): off by default
+    const bool shfl = L.col_shift && !pipe && L.gv > 1 && geometry_knob(L, "FOP_COL_SHFL", 0);
+    if (shfl)
+      o.l("const unsigned smask_ = " + std::string(L.gv == 32 ? "0xffffffffu" : "(" + num((1u << L.gv) - 1) +
+          "u << ((threadIdx.x & 31u) & ~" + num(L.gv - 1) + "u))") + ";");
     auto batch_loads = [&](const std::string& rbase, const std::string& buf, const std::string& tg) {
       for (int u = 0; u < U; u++) {
         std::string t = tg + num(u);
@@ -2289,6 +2298,40 @@ struct Gen {
         for (size_t k = 0; k < L.loads.size(); k++) {
           if (!wpv[k]) continue;
           const Affine& a = L.loads[k];
+          if (shfl) {
+            const int esk = es(a.tensor);
+            const std::string B = buf + num(k) + "_" + num(u), X = "X" + num(k) + "_" + num(u) + tg,
+                              M = "M" + num(k) + "_" + num(u) + tg;
+            const int64_t span = tensor_bytes(a.tensor) / esk;
+            auto elementwise = [&](const std::string& dst, const std::string& from) {
+              if (esk == 2)
+                return "for (int e = 0; e < " + num(W) + "; ++e) if (" + from + " + e < (idx_t)" + num(span) + "ull) " +
+                       dst + "[e >> 1] |= (u32)fop::ld16<" + pol(a, false) + ">(T" + num(a.tensor) + " + (u64)(" + from +
+                       " + e) * 2u) << ((e & 1) * 16);";
+              return "for (int e = 0; e < " + num(W) + "; ++e) if (" + from + " + e < (idx_t)" + num(span) +
+                     "ull) fop::ldraw<4, " + pol(a, false) + ">(" + dst + " + e, T" + num(a.tensor) + " + (u64)(" + from +
+                     " + e) * 4u);";
+            };
+            o.l("{");
+            o.l("  const idx_t o_ = " + affine(a, bits) + ";");
+            o.l("  " + M + " = (unsigned)(((u64)T" + num(a.tensor) + " + (u64)o_ * " + num(esk) + "u) & 15u) / " +
+                num(esk) + "u;");
+            o.l("  const idx_t a_ = o_ - " + M + ";");
+            o.l("  #pragma unroll");
+            o.l("  for (int w_ = 0; w_ < 4; ++w_) { " + B + "[w_] = 0u; " + X + "[w_] = 0u; }");
+            o.l("  if (rr < r1) {");
+            o.l("    if (a_ + " + num(W) + "u <= (idx_t)" + num(span) + "ull) fop::ldraw<16, " + pol(a, false) + ">(" + B +
+                ", T" + num(a.tensor) + " + (u64)a_ * " + num(esk) + "u);");
+            o.l("    else " + elementwise(B, "a_"));
+            o.l("    if (" + M + " != 0u && (cv == " + num(L.gv - 1) + "u || j + 1u >= " + num(NVD) + "u)) {");
+            o.l("      if (a_ + " + num(2 * W) + "u <= (idx_t)" + num(span) + "ull) fop::ldraw<16, " + pol(a, false) + ">(" +
+                X + ", T" + num(a.tensor) + " + (u64)(a_ + " + num(W) + "u) * " + num(esk) + "u);");
+            o.l("      else " + elementwise(X, "a_ + " + num(W) + "u"));
+            o.l("    }");
+            o.l("  }");
+            o.l("}");
+            continue;
+          }
           if (L.col_shift) {
             // the row's W elements from the two aligned 16 B chunks around them,
             // funnel-shifted by the row's misalignment m_ (elements); a second
@@ -2367,7 +2410,38 @@ struct Gen {
       for (int u = 0; u < U; u++)
         for (size_t k = 0; k < L.loads.size(); k++)
           if (wpv[k]) o.l("u32 A" + num(k) + "_" + num(u) + "[" + num(wpv[k]) + "];");
+      if (shfl)
+        for (int u = 0; u < U; u++)
+          for (size_t k = 0; k < L.loads.size(); k++)
+            if (wpv[k]) o.l("unsigned M" + num(k) + "_" + num(u) + "_a; u32 X" + num(k) + "_" + num(u) + "_a[4];");
       batch_loads("r", "A", "_a");
+      if (shfl) {   // the batch is in flight: now each row's window (its own chunk + the neighbour's)
+        for (int u = 0; u < U; u++)
+          for (size_t k = 0; k < L.loads.size(); k++) {
+            if (!wpv[k]) continue;
+            const int esk = es(L.loads[k].tensor), epw = 4 / esk;
+            const std::string A = "A" + num(k) + "_" + num(u), M = "M" + num(k) + "_" + num(u) + "_a",
+                              X = "X" + num(k) + "_" + num(u) + "_a";
+            o.l("{");
+            o.l("  u32 V_[8];");
+            o.l("  #pragma unroll");
+            o.l("  for (int w_ = 0; w_ < 4; ++w_) { V_[w_] = " + A + "[w_]; V_[4 + w_] = __shfl_down_sync(smask_, " + A +
+                "[w_], 1, " + num(L.gv) + "); }");
+            o.l("  if (cv == " + num(L.gv - 1) + "u || j + 1u >= " + num(NVD) + "u) {");
+            o.l("    #pragma unroll");
+            o.l("    for (int w_ = 0; w_ < 4; ++w_) V_[4 + w_] = " + X + "[w_];");
+            o.l("  }");
+            o.l("  const unsigned t_ = " + M + " / " + num(epw) + "u, s_ = (" + M + " % " + num(epw) + "u) * " +
+                num(esk * 8) + "u;");
+            o.l("  #pragma unroll");
+            o.l("  for (int q = 0; q < 4; ++q) {");
+            o.l("    const u32 lo_ = t_ == 0u ? V_[q] : t_ == 1u ? V_[q + 1] : t_ == 2u ? V_[q + 2] : V_[q + 3];");
+            o.l("    const u32 hi_ = t_ == 0u ? V_[q + 1] : t_ == 1u ? V_[q + 2] : t_ == 2u ? V_[q + 3] : V_[q + 4];");
+            o.l("    " + A + "[q] = __funnelshift_r(lo_, hi_, s_);");
+            o.l("  }");
+            o.l("}");
+          }
+      }
     }
     std::vector<std::vector<std::pair<int, std::string>>> its(U);
     for (int u = 0; u < U; u++) {

@@ -94,11 +94,13 @@ def _colred(R, C, dtype="f16", op="sum", expr=None):
                                           (5000, 37, "f32", "sum"), (2000, 257, "bf16", "sum"), (3001, 1001, "f16", "max"),
                                           (64, 9, "f16", "sum")])
 @pytest.mark.parametrize("offset", [0, 1])
-def test_column_reduction_over_odd_rows(R, C, dtype, op, offset):
+@pytest.mark.parametrize("shfl", ["0", "1"])
+def test_column_reduction_over_odd_rows(monkeypatch, R, C, dtype, op, offset, shfl):
     """Column sums / maxima over rows of odd length: full-width vectors, each row's window
     funnel-shifted out of two aligned 16 B chunks; the partial last vector's extra
     columns are never stored.  Misaligned base pointers take the narrow variant."""
     from harness import abs_terms_desc, assert_normwise
+    monkeypatch.setenv("FOP_COL_SHFL", shfl)     # second chunk: loaded (0, default) or shuffled from the neighbour (1)
     d = _colred(R, C, dtype, op)
     x = W.make_inputs(d)
     got, o = run_gpu(d, x, offset=offset)
