@@ -24,7 +24,18 @@
  * which the write access does not depend) of the DAG value, then applies the
  * finalize DAG (e.g. /768 for a mean); a later statement reads the STORED
  * (rounded) values.  Arithmetic nodes are fp32; add/sub/mul/div/sqrt are IEEE
- * correctly rounded and never contracted.
+ * correctly rounded and never contracted (divisions too: the kernels' fast form
+ * for a loop-invariant divisor returns the correctly rounded quotient).
+ *
+ * Integer statements (reading R30): a statement whose write tensor is
+ * FOP_I32 (and that is not a pure element move) computes on int32 values — it
+ * reads i32 tensors only, its DAG uses ADD SUB MUL MAX MIN NEG ABS RELU and
+ * CONST with an integral immediate, every result wraps modulo 2^32 (two's
+ * complement), REDUCE SUM is the sum modulo 2^32 (any association order gives
+ * the same bits) and MAX the maximum.  A float statement reads no i32 tensor.
+ * Anything else on i32 (DIV, SQRT, transcendentals, CAST to i32, a fractional
+ * immediate, mixing i32 and float tensors) is FOP_E_INVALID.  A pure move
+ * copies any dtype bit for bit.
  *
  * Ownership: the caller owns every buffer (host descriptors, device tensors,
  * workspace).  fop_plan copies the descriptor; a plan is immutable after
@@ -86,7 +97,7 @@ typedef enum { FOP_RED_SUM = 0, FOP_RED_MAX = 1 } fop_reduce_op;
 
 typedef enum {
   FOP_OP_LOAD = 0,      /* a = read access index (1..nacc-1) */
-  FOP_OP_CONST = 1,     /* imm (fp32) */
+  FOP_OP_CONST = 1,     /* imm (fp32; an integral value in int32 range in an integer statement) */
   FOP_OP_ACC = 2,       /* finalize DAG only: the reduced value */
   FOP_OP_ADD = 3, FOP_OP_SUB = 4, FOP_OP_MUL = 5, FOP_OP_DIV = 6,
   FOP_OP_MAX = 7, FOP_OP_MIN = 8,          /* fmaxf/fminf semantics */
