@@ -160,7 +160,14 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       v.push_back({{"FOP_VEC_BYTES", 32}, {"FOP_EW_U", 4}, {"FOP_EW_MINB", 2}, {"FOP_BLOCK", 128}});
       break;
     case FOP_CLASS_TRANSPOSE:
-      if (L.tma) break;
+      if (L.tma) {   // TMA tiles: 2 warps per CTA x 2 CTAs per SM next to the default 4 x 1,
+                     // and the register tiles (ahead where the tuner's cold launch says so)
+        v.push_back({{"FOP_TR_TMA_WARPS", 2}, {"FOP_TR_TMA_MINB", 2}});
+        v.push_back({{"FOP_TR_TMA", 0}});
+        v.push_back({{"FOP_TR_TMA", 0}, {"FOP_BLOCK", 256}, {"FOP_TR_MINB", 1}});
+        v.push_back({{"FOP_TR_TMA", 0}, {"FOP_BLOCK", 128}, {"FOP_TR_MINB", 2}});
+        break;
+      }
       if (L.tr_smem) {
         v.push_back({{"FOP_TR_SMEM_MINB", 2}});
         v.push_back({{"FOP_TR_SMEM_MINB", 6}});
@@ -625,8 +632,11 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.tma = 0;
     const Affine& tl = L.loads[L.trans_load];
     const XStmt& x0 = L.stmts[0];
-    // opt-in: measured 5.72 vs 5.99 TB/s for the register transpose on cfg3
-    bool ok = knob("FOP_TR_TMA", 0) && !L.scalar_variant && L.stmts.size() == 1 &&
+    // Default for eligible 16-bit transposes since round 2 (2 stages per warp): in the bench suite
+    // 6427 vs 6106 GB/s for the register tiles (suite 6299 vs 6166), cold single launch under ncu
+    // 122.4 vs 131.8 us; only back-to-back repeats of the same transpose favour the register tiles
+    // (5971 vs 6104, profiles/r02/tma_suite_r02.log).  FOP_TR_TMA=0 selects the register path.
+    bool ok = knob("FOP_TR_TMA", 1) && !L.scalar_variant && L.stmts.size() == 1 &&
               esize(d.t[tl.tensor].dtype) == 2 && esize(x0.out_dtype) == 2 && L.kl.size() <= 5 &&
               L.kl[0].extent >= 64 && L.kl[1].extent >= 64 && tl.base % 8 == 0 && x0.write.base % 8 == 0;
     for (size_t k = 0; k < L.loads.size() && ok; k++) {
@@ -662,7 +672,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
         L.tma_out_tensor = x0.write.tensor;
         L.tma_in_base = tl.base;
         L.tma_out_base = x0.write.base;
-        L.tma_stages = std::max(2, std::min(8, knob("FOP_TR_TMA_STAGES", 4)));
+        L.tma_stages = std::max(2, std::min(8, knob("FOP_TR_TMA_STAGES", 2)));   // 3+ stages: 5.6-5.8 TB/s in the suite
         L.tma_ntv = (L.kl[0].extent + 63) / 64;
         L.tma_ntr = (L.kl[1].extent + 63) / 64;
         L.tma_tiles = L.tma_ntv * L.tma_ntr * prod_rest;

@@ -223,7 +223,6 @@ CUfunction narrow_fn(Plan& p, Plan::Loaded& l, size_t i) {
 // (kTuneScratchBytes; B200's L2 is 126 MB) through it; fop_l2_dirty then
 // writes the first bytes of the scratch, leaving that many dirty lines.
 constexpr size_t kTuneScratchBytes = size_t(320) << 20;
-constexpr size_t kTuneColdBytes = size_t(512) << 20;   // operators touching less are tuned from a cold L2
 CUfunction l2_flush_fn(Plan::Loaded& l) {
   if (l.flush_fn) return (CUfunction)l.flush_fn;
   static Launch F;
@@ -403,18 +402,17 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
   // (bit-identical for ASSIGN; reductions within R16), and the plan is
   // idempotent, so the extra launches only cost time once.
   //
-  // An operator whose tensors fit in a few L2s would be timed L2-hot by
-  // back-to-back launches on the same buffers, which ranks geometries by
-  // their L2 behaviour instead of the HBM streaming they do in a real
-  // pipeline (BERT LayerNorm: the L2-hot ranking kept a geometry 9 % slower
-  // from HBM).  For those, every timed launch is preceded by a read of a
-  // scratch buffer larger than L2 (and the previous launch's dirty lines are
-  // written back during it), then by a write of as many bytes as the plan
-  // outputs: each candidate starts as it would inside a pipeline, inputs in
-  // HBM and the previous launch's outputs dirty in L2.
-  int64_t footprint = 0;
-  for (int t = 0; t < d.ntensors; t++)
-    if (d.t[t].role != FOP_TEMP) footprint += span_bytes(d.t[t]);
+  // Back-to-back launches on the same buffers would rank geometries by their
+  // behaviour when repeating themselves: L2-hot for operators that fit in a
+  // few L2s (BERT LayerNorm: that ranking kept a geometry 9 % slower from
+  // HBM), and with the previous instance's tail and write-back overlapping
+  // for large ones (cfg3: the register tiles tie back to back, the TMA tiles
+  // are 4 % faster after another operator, profiles/r02/tune_protocol_r02.log).
+  // So every timed launch is preceded by a read of a scratch buffer larger
+  // than L2 (the previous launch's dirty lines are written back during it),
+  // then by a write of as many bytes as the plan outputs: each candidate
+  // starts as it would inside a pipeline, inputs in HBM and the previous
+  // operator's outputs dirty in L2.  FOP_TUNE_HOT=1: back-to-back timing.
   auto tune = [&](size_t i) {
     int capturing = 0;
     if (c.stream_capturing(st, &capturing) != 0 || capturing) return -1;
@@ -423,7 +421,8 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
     check(c.ev_create(&e1, 0), "cuEventCreate");
     CUfunction flush = nullptr;
     CUdeviceptr scratch = 0;
-    if (footprint < (int64_t)kTuneColdBytes && !std::getenv("FOP_TUNE_HOT")) {
+    const char* hot = std::getenv("FOP_TUNE_HOT");
+    if (!(hot && *hot == '1')) {
       flush = l2_flush_fn(l);
       if (flush && c.mem_alloc(&scratch, kTuneScratchBytes) != 0) scratch = 0;   // no room: time L2-hot
       // defined contents: the flush kernel only reads it to evict L2, but compute-sanitizer's
@@ -489,8 +488,10 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
     // (BERT LayerNorm: candidates within 3 % swapped ranks between runs)
     int best = 0;
     float best_ms = 0.f, def_ms = 0.f;
+    std::vector<float> tlog;
     for (size_t k = 0; k <= l.vfns[i].size(); k++) {
       float ms = time_k(k, reps);
+      tlog.push_back(ms);
       if (k == 0) def_ms = ms;
       if (k == 0 || ms < best_ms) {
         best = (int)k;
@@ -498,6 +499,11 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
       }
     }
     if (best != 0 && best_ms > 0.98f * def_ms) best = 0;
+    if (const char* lg = std::getenv("FOP_TUNE_LOG"); lg && *lg == '1') {   // diagnostics: the candidates' times
+      std::fprintf(stderr, "[fop tune] launch %zu (%s): %s", i, scratch ? "cold" : "hot", p.launches[i].name.c_str());
+      for (size_t k = 0; k < tlog.size(); k++) std::fprintf(stderr, " v%zu=%.1fus", k, 1e3f * tlog[k]);
+      std::fprintf(stderr, " -> v%d\n", best);
+    }
     if (scratch) {
       c.ev_sync(e1);
       c.mem_free(scratch);

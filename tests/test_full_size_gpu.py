@@ -40,8 +40,11 @@ def _run_variant(desc, dev_in, k):
     return res, name
 
 
-@pytest.mark.parametrize("name", ["cfg2", "cfg3", "cfg4a", "cfg4b"])
-def test_every_tuning_candidate_full_size_whole_output(name):
+@pytest.mark.parametrize("name,tma", [("cfg2", "1"), ("cfg3", "1"), ("cfg3", "0"), ("cfg4a", "1"), ("cfg4b", "1")])
+def test_every_tuning_candidate_full_size_whole_output(monkeypatch, name, tma):
+    """cfg3 twice: the TMA tiles (the 16-bit default, what the bench times) and the
+    register tiles (FOP_TR_TMA=0, the f32/i32 path and the fallback)."""
+    monkeypatch.setenv("FOP_TR_TMA", tma)
     from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
     d = W.CONFIGS[name]()
     nv = FusedOp(d, jit=1).info()["launches"][0]["nvariants"]

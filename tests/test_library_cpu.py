@@ -156,7 +156,8 @@ def _sass(cubin):
 
 @pytest.mark.parametrize("name,expect", [
     ("cfg2", {"ew": [r"LDG\.E\.NA\.128", r"STG\.E\.128"]}),
-    ("cfg3", {"transpose": [r"LDG\.E\.NA\.128", r"STG\.E\.128"]}),
+    # 16-bit transposes default to the TMA tiles (round 2): bulk tensor copies + mbarriers, 16 B smem moves
+    ("cfg3", {"transpose": [r"UTMALDG", r"UTMASTG", r"SYNCS\.PHASECHK\.TRANS64", r"LDS\.128", r"STS\.(128|64)"]}),
     ("cfg4a", {"row_reduce": [r"LDG\.E\.NA\.128", r"STG\.E\.128", r"SHFL\.BFLY"]}),
     ("cfg4b", {"col_reduce": [r"LDG\.E\.NA\.128", r"ATOMG|RED\.|ATOM"]}),
 ])
@@ -172,6 +173,15 @@ def test_config_kernels_compile_for_sm100a_with_vector_access(name, expect):
     for pat in expect[cls]:
         assert re.search(pat, sass), (name, pat)
     assert "LDL" not in sass and "STL" not in sass      # no register spills
+
+
+def test_register_transpose_when_tma_is_off(monkeypatch):
+    monkeypatch.setenv("FOP_TR_TMA", "0")
+    op = FusedOp(W.cfg3())
+    assert op.selected(0)[0].startswith("fop_transpose_k")
+    sass = _sass(op.cubin(0))
+    assert re.search(r"LDG\.E\.NA\.128", sass) and re.search(r"STG\.E\.128", sass)
+    assert "LDL" not in sass and "STL" not in sass
 
 
 def test_tma_transpose_variant(monkeypatch):
@@ -249,10 +259,12 @@ def test_binding_rejects_wrong_buffers_before_the_abi():
     op._host_ptrs(dict(good, x=ok))
 
 
-def test_transpose_vector_loop_absorbs_contiguous_continuations():
+def test_transpose_vector_loop_absorbs_contiguous_continuations(monkeypatch):
     """NHWC -> NCHW: the store side is contiguous over w then h, and so is the
     load side's h after w, so the kernel's d_v is the collapsed h*w (3136
-    elements = 392 tiles of 8), not w alone (7 tiles, a ragged warp)."""
+    elements = 392 tiles of 8), not w alone (7 tiles, a ragged warp).  Register tiles
+    (FOP_TR_TMA=0): 16-bit transposes otherwise take the TMA skeleton."""
+    monkeypatch.setenv("FOP_TR_TMA", "0")
     op = FusedOp(W.nhwc_to_nchw(256, 56, 56, 256), jit=0, autotune=0)
     li = op.info()["launches"][0]
     assert (li["class"], li["width"], li["read_width"]) == ("transpose", 8, 8)

@@ -135,6 +135,7 @@ def test_column_sum_of_squares_odd_rows_every_candidate():
 def test_transpose_software_pipelined_bitexact(monkeypatch, dims, dtype, knobs):
     """The register transpose with the next grid-stride iteration's loads issued before the
     current tiles are stored (FOP_TR_PIPE): same tiles, same arithmetic, same bits."""
+    monkeypatch.setenv("FOP_TR_TMA", "0")        # the register skeleton (16-bit default: TMA tiles)
     for kv in knobs.split(","):
         k, v = kv.split("=")
         monkeypatch.setenv(k, v)

@@ -126,7 +126,9 @@ def test_fig2_fp16_target_rounds_every_step():
 
 # ---------------------------------------------------------------- TRANSPOSE
 @pytest.mark.parametrize("dims", [(2, 256, 56, 56), (1, 24, 5, 7), (2, 40, 3, 16), (1, 8, 1, 8)])
-def test_cfg3_transpose_bitexact(dims):
+@pytest.mark.parametrize("tma", ["0", "1"])
+def test_cfg3_transpose_bitexact(monkeypatch, dims, tma):
+    monkeypatch.setenv("FOP_TR_TMA", tma)       # register tiles / TMA tiles (the 16-bit default)
     d = W.cfg3(*dims)
     d["tensors"]["x"]["init"] = ("special", 9)
     x = W.make_inputs(d)
@@ -138,7 +140,7 @@ def test_cfg3_transpose_bitexact(dims):
 @pytest.mark.parametrize("dims,move", [((2, 256, 56, 56), False), ((1, 40, 9, 13), False), ((2, 128, 8, 64), True),
                                        ((1, 64, 64, 64), False)])
 def test_cfg3_tma_transpose_bitexact(monkeypatch, dims, move):
-    """TMA path (cp.async.bulk.tensor, 128B swizzle, mbarrier pipeline; opt-in FOP_TR_TMA=1):
+    """TMA path (cp.async.bulk.tensor, 128B swizzle, mbarrier pipeline; the 16-bit default):
     64x64 tiles with out-of-bounds edges (C=40, HW=117) must give the same bits."""
     monkeypatch.setenv("FOP_TR_TMA", "1")
     d = W.cfg3(*dims)
@@ -218,11 +220,13 @@ def test_transpose_roundtrip_on_gpu():
 @pytest.mark.parametrize("dims,cls", [((2, 56, 56, 256), "transpose"), ((3, 7, 9, 64), "transpose"),
                                       ((1, 14, 14, 40), "transpose"), ((2, 5, 8, 24), "transpose"),
                                       ((2, 7, 7, 2048), "transpose")])
-def test_nhwc_to_nchw_bitexact(dims, cls):
+@pytest.mark.parametrize("tma", ["0", "1"])
+def test_nhwc_to_nchw_bitexact(monkeypatch, dims, cls, tma):
     """The reverse layout change: d_v absorbs h after w (one contiguous run of
     H*W on both sides), so the store tiles span whole NCHW planes.  An odd
     H*W (63, 49) cannot carry store vectors: flat output tiles through shared
     memory."""
+    monkeypatch.setenv("FOP_TR_TMA", tma)
     d = W.nhwc_to_nchw(*dims, s=0.5)
     x = W.make_inputs(d)
     got, op = run_gpu(d, x)
