@@ -2186,7 +2186,8 @@ struct Gen {
     const int W = L.width, U = L.unroll;
     const XStmt& x = L.stmts[0];
     const int64_t EV0 = L.kl[0].extent;
-    const int64_t NVD = L.col_shift ? (EV0 + W - 1) / W : EV0 / W;   // col_shift: a partial last vector
+    const int64_t FP = L.col_fold;   // > 0: P-row groups of dense odd rows, read as [R/P, P*E] (geometry.cpp)
+    const int64_t NVD = L.col_shift ? (EV0 + W - 1) / W : FP ? FP * EV0 / W : EV0 / W;   // col_shift: a partial last vector
     const int64_t SVN = (NVD + L.gv - 1) / L.gv;
     int64_t slabs = SVN;
     for (int k = 1; k < L.nsplit; k++) slabs *= L.kl[k].extent;
@@ -2205,6 +2206,7 @@ struct Gen {
     header("COL_REDUCE (slab of gv x W columns, row chunks, fixed-order trees)", 1);
     o.l("__shared__ float red[" + num(L.block * W) + "];");
     o.l("__shared__ unsigned last_flag;");
+    if (FP) o.l("__shared__ unsigned fold_flag;");
     o.l("const unsigned tid = threadIdx.x, cv = tid % " + num(L.gv) + "u, rl = tid / " + num(L.gv) + "u;");
     o.l("const idx_t slab = blockIdx.x % " + num(slabs) + "u, chunk = blockIdx.x / " + num(slabs) + "u;");
     // peer exchange: the slab's run counter, read in the epilogue (FOP_PEER_EP=0, default) or at kernel
@@ -2268,7 +2270,7 @@ struct Gen {
     // Software pipeline (default): the U row loads of batch i+1 are issued as
     // raw words before batch i is converted and accumulated, so HBM requests
     // stay in flight across the accumulation instead of draining each batch.
-    bool pipe = L.col_pipe;
+    bool pipe = L.col_pipe && !FP;
     std::vector<int> wpv(L.loads.size(), 0);
     for (size_t k = 0; k < L.loads.size(); k++) {
       int64_t cv = C(L.loads[k], 0);
@@ -2292,7 +2294,7 @@ struct Gen {
         o.l("{");
         o.ind++;
         o.l("const idx_t rr = " + rbase + " + " + num(RSTEP * u) + "u;");
-        o.l("idx_t q = rr;");
+        o.l(FP ? "idx_t q = rr * " + num(FP) + "u;" : "idx_t q = rr;");   // fold: the group's first row
         std::vector<std::pair<int, std::string>> bits = cits;
         decompose("q", L.nsplit, (int)L.kl.size(), t, bits);
         for (size_t k = 0; k < L.loads.size(); k++) {
@@ -2448,7 +2450,7 @@ struct Gen {
       std::string t = "_" + num(u);
       o.l("const idx_t rr" + t + " = r + " + num(RSTEP * u) + "u;");
       o.l("const bool ok" + t + " = okc && rr" + t + " < r1;");
-      o.l("idx_t q" + t + " = rr" + t + ";");
+      o.l("idx_t q" + t + " = rr" + t + (FP ? " * " + num(FP) + "u;" : ";"));
       its[u] = cits;
       decompose("q" + t, L.nsplit, (int)L.kl.size(), t, its[u]);
       for (size_t k = 0; k < L.loads.size(); k++) {
@@ -2690,9 +2692,47 @@ struct Gen {
       o.ind--;
       o.l("}");
     };
+    // fold (col_fold = P): the slab's sums of wide columns iv + e go to F in
+    // the workspace; the last slab to arrive adds, for each output column c,
+    // F[g * E + c] over the P group rows g in order (fixed, deterministic) and
+    // stores the E results element-wise
+    auto fold_store = [&]() {
+      const size_t FB = ((size_t)FP * (size_t)EV0 * sizeof(float) + 255) & ~size_t(255);
+      o.l("{");
+      o.ind++;
+      o.l("float* F_ = (float*)(args.ws + " + num((int64_t)L.fold_off) + "ull);");
+      o.l("unsigned* fc_ = (unsigned*)(args.ws + " + num((int64_t)(L.fold_off + FB)) + "ull);");
+      o.l("if (rl == 0u && okc) {");
+      o.l("  #pragma unroll");
+      o.l("  for (int e = 0; e < " + num(W) + "; ++e) F_[iv + e] = red[cv * " + num(W) + "u + e];");
+      o.l("}");
+      o.l("__threadfence();");
+      o.l("__syncthreads();");
+      o.l("if (tid == 0u) fold_flag = (atomicAdd(fc_, 1u) == " + num(SVN - 1) + "u);");
+      o.l("__syncthreads();");
+      o.l("if (fold_flag) {");
+      o.ind++;
+      o.l("__threadfence();");
+      o.l("for (unsigned c_ = tid; c_ < " + num(EV0) + "u; c_ += " + num(L.block) + "u) {");
+      o.ind++;
+      o.l("float a_ = " + init + ";");
+      o.l("#pragma unroll");
+      o.l("for (int g = 0; g < " + num(FP) + "; ++g) a_ = " + comb("a_", "__ldcg(&F_[g * " + num(EV0) + "u + c_])") + ";");
+      std::string r = fin_expr(o, x, "a_", "");
+      std::vector<std::pair<int, std::string>> fc = {{0, "(idx_t)c_"}};
+      o.l("fop::sstore<" + std::string(dtn(x.out_dtype)) + ">(" + ptr(x.write.tensor, affine(x.write, fc)) + ", " + r + ");");
+      o.ind--;
+      o.l("}");
+      o.l("if (tid == 0u) *fc_ = 0u;");
+      o.ind--;
+      o.l("}");
+      o.ind--;
+      o.l("}");
+    };
     if (NCH == 1) {
       exchange();
-      final_store();
+      if (FP) fold_store();
+      else final_store();
     } else if (L.col_fin) {
       // Flag-word finalize (FOP_COL_FIN=1/2, ablations; 0 = the default below):
       // chunk blocks store their SW slab sums as 64-bit words (1 << 32 | fp32
@@ -2846,7 +2886,8 @@ struct Gen {
       o.l("__syncthreads();");
       tree();
       exchange();
-      final_store();
+      if (FP) fold_store();
+      else final_store();
       o.l("if (tid == 0u) cnt[slab] = 0u;");
       o.ind--;
       o.l("}");

@@ -177,6 +177,8 @@ struct Launch {
   size_t ws_off = 0, ws_bytes = 0;  // COL_REDUCE partials + counters
   std::vector<int> align;         // per tensor: byte alignment the vector variant assumes
   bool scalar_variant = false;    // this launch is the narrow (W=1) variant
+  int col_fold = 0;               // COL: dense odd rows read as [R/P, P*E] (P rows per aligned group), folded at the end
+  size_t fold_off = 0;            // COL fold: wide-column sums + counter, offset inside the launch's workspace
   int col_shift = 0;              // COL: full-width vectors over odd rows via per-row funnel shifts of aligned chunks
   int tr_om = 0;                  // TRANSPOSE smem (tr_smem 2): output-major tile (lane-contiguous scatter, vector read-out)
   int64_t period = 0;             // EW: kl[0] is (d_v x next loop) flattened; period accesses use c = flat % period

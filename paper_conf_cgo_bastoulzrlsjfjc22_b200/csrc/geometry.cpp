@@ -19,6 +19,7 @@
 // access are collapsed (a B200 step beyond the paper).
 #include <algorithm>
 #include <cstdlib>
+#include <numeric>
 #include <string>
 
 #include "fop_internal.h"
@@ -394,9 +395,30 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     }
     if (ok) L.col_shift = 1;
   }
+  // ... and when the rows are dense (pitch E[d_v]) and P = W / gcd(E, W)
+  // divides the row count, P consecutive rows are P*E elements: a whole
+  // number of aligned W-vectors.  Read the matrix as [R/P, P*E] — full-width
+  // aligned vectors, no shifts — where lane j's element e always falls on
+  // column (j*W + e) mod E (of row (j*W + e) div E inside the group); the last
+  // block to finish folds the P*E wide-column sums into the E outputs, P
+  // terms each in group-row order (the vector access is kept whole).
+  L.col_fold = 0;
+  if (L.kclass == FOP_CLASS_COL_REDUCE && W > 1 && EV % W != 0 && L.nsplit == 1 && L.kl.size() == 2 &&
+      !L.scalar_variant && L.stmts.size() == 1 && p.opts.peer_world < 1 && geometry_knob(L, "FOP_COL_FOLD", 1)) {
+    const int64_t P = W / std::gcd<int64_t>(EV, W);
+    bool ok = L.kl[1].extent % P == 0 && coef(L, L.stmts[0].write, 0) == 1 && coef(L, L.stmts[0].write, 1) == 0;
+    for (const auto& a : L.loads) {
+      const int es_a = esize(d.t[a.tensor].dtype);
+      ok &= coef(L, a, 0) == 1 && coef(L, a, 1) == EV && W * es_a == 16 && a.base * es_a % 16 == 0;
+    }
+    if (ok) {
+      L.col_fold = (int)P;
+      L.col_shift = 0;
+    }
+  }
   if (tail_ok) {
     if (EV < W) W = pow2_floor(EV);
-  } else if (!L.row_peel && !L.col_shift) {
+  } else if (!L.row_peel && !L.col_shift && !L.col_fold) {
     while (W > 1 && EV % W) W /= 2;
   }
   L.width = W;
@@ -518,6 +540,10 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
   if (L.col_shift)   // aligned 16 B chunks around each row's window (the base must be 16 B aligned)
     for (size_t k = 0; k < L.loads.size(); k++)
       if (coef(L, L.loads[k], 0) == 1) L.load_cb[k] = 16;
+  if (L.col_fold) {   // aligned 16 B vectors of the [R/P, P*E] view; the E outputs are stored element-wise
+    for (size_t k = 0; k < L.loads.size(); k++) L.load_cb[k] = 16;
+    L.store_cb[0] = 0;
+  }
   if (L.row_peel) {   // alignment comes from the per-row shift, not from the static coefficients
     for (size_t k = 0; k < L.loads.size(); k++) {
       if (coef(L, L.loads[k], 0) != 1) continue;
@@ -753,7 +779,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
                                                        (int64_t)knob("FOP_ROW_CLUSTERS", 1 << 30)})) * Q;
     L.unroll = 1;
   } else {  // COL_REDUCE
-    int64_t nvd = L.col_shift ? (EV + W - 1) / W : EV / W;   // col_shift: a partial last vector
+    int64_t nvd = L.col_shift ? (EV + W - 1) / W : L.col_fold ? L.col_fold * EV / W : EV / W;   // col_shift: a partial last vector
     const Affine* big = nullptr;
     for (const auto& a : L.loads)
       if (coef(L, a, 0) == 1) big = &a;
@@ -766,6 +792,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     for (int k = 1; k < L.nsplit; k++) slabs *= L.kl[k].extent;
     int64_t rows = 1;
     for (size_t k = L.nsplit; k < L.kl.size(); k++) rows *= L.kl[k].extent;
+    if (L.col_fold) rows /= L.col_fold;   // groups of P rows
     L.col_pipe = knob("FOP_COL_PIPE", 0);   // measured: no gain over plain batches (sweep_r01_4)
     L.col_il = knob("FOP_COL_IL", 1);
     // 6 blocks/SM x 4 rows in flight: the column-sum probe and the sweep
@@ -780,7 +807,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     L.grid = slabs * nch;
     // finalize: store + fence + arrival counter + last-arriving block (0, default),
     // or flag words polled by the slab's last chunk block (1) / last arrival (2)
-    L.col_fin = knob("FOP_COL_FIN", 0);
+    L.col_fin = L.col_fold ? 0 : knob("FOP_COL_FIN", 0);
     if (nch > 1 && L.col_fin) {
       L.ws_bytes = ((size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(unsigned long long) + 255) & ~size_t(255);
       if (L.col_fin == 2) L.ws_bytes += (size_t)slabs * sizeof(unsigned);
@@ -789,6 +816,10 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
       size_t part = (size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(float);
       part = (part + 255) & ~size_t(255);
       L.ws_bytes = part + (size_t)slabs * sizeof(unsigned);
+    }
+    if (L.col_fold) {   // the wide-column sums and the arrival counter of the fold
+      L.fold_off = (L.ws_bytes + 255) & ~size_t(255);
+      L.ws_bytes = L.fold_off + (((size_t)L.col_fold * (size_t)EV * sizeof(float) + 255) & ~size_t(255)) + 16;
     }
     L.smem = (size_t)L.block * W * sizeof(float) + 16;
   }

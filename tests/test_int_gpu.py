@@ -123,7 +123,7 @@ def _ired(R, C, op, axis, expr=None):
                        "expr": expr or [("load", 0), ("const", 3.0), ("mul", 0, 1)]}]}
 
 
-@pytest.mark.parametrize("R,C", [(65536, 1024), (1000, 13), (7, 40000), (100000, 8), (3, 5)])
+@pytest.mark.parametrize("R,C", [(65536, 1024), (1000, 13), (7, 40000), (100000, 8), (3, 5), (4096, 1001), (4098, 1002)])
 @pytest.mark.parametrize("op", ["sum", "max"])
 @pytest.mark.parametrize("axis", ["col", "row"])
 def test_int_reductions_bit_exact_every_candidate(R, C, op, axis):

@@ -92,20 +92,29 @@ def _colred(R, C, dtype="f16", op="sum", expr=None):
 
 @pytest.mark.parametrize("R,C,dtype,op", [(65536, 1001, "f16", "sum"), (777, 1001, "f16", "sum"), (300, 13, "f16", "sum"),
                                           (5000, 37, "f32", "sum"), (2000, 257, "bf16", "sum"), (3001, 1001, "f16", "max"),
-                                          (64, 9, "f16", "sum")])
+                                          (64, 9, "f16", "sum"), (4096, 1002, "f16", "sum"), (1000, 1004, "bf16", "max"),
+                                          (8, 1001, "f16", "sum"), (40000, 3, "f16", "sum"), (6, 1001, "f32", "max")])
 @pytest.mark.parametrize("offset", [0, 1])
-@pytest.mark.parametrize("shfl", ["0", "1"])
-def test_column_reduction_over_odd_rows(monkeypatch, R, C, dtype, op, offset, shfl):
-    """Column sums / maxima over rows of odd length: full-width vectors, each row's window
-    funnel-shifted out of two aligned 16 B chunks; the partial last vector's extra
-    columns are never stored.  Misaligned base pointers take the narrow variant."""
+@pytest.mark.parametrize("mode", ["fold", "shift", "shfl"])
+def test_column_reduction_over_odd_rows(monkeypatch, R, C, dtype, op, offset, mode):
+    """Column sums / maxima over rows of odd length, full-width vectors either way:
+    fold (default when P = W / gcd(C, W) divides R): the matrix read as [R/P, P*C] with
+    aligned vectors, the P*C wide-column sums folded into the C outputs by the last slab;
+    shift: each row's window funnel-shifted out of two aligned 16 B chunks (the partial
+    last vector's extra columns never stored); shfl: the second chunk shuffled from the
+    neighbour lane.  Misaligned base pointers take the narrow variant."""
+    import math
     from harness import abs_terms_desc, assert_normwise
-    monkeypatch.setenv("FOP_COL_SHFL", shfl)     # second chunk: loaded (0, default) or shuffled from the neighbour (1)
+    monkeypatch.setenv("FOP_COL_FOLD", "1" if mode == "fold" else "0")
+    monkeypatch.setenv("FOP_COL_SHFL", "1" if mode == "shfl" else "0")
     d = _colred(R, C, dtype, op)
     x = W.make_inputs(d)
     got, o = run_gpu(d, x, offset=offset)
     if offset == 0:
-        assert "__funnelshift_r" in o.source(), o.info()["launches"][0]
+        Wd = 16 // (4 if dtype == "f32" else 2)
+        fold = mode == "fold" and R % (Wd // math.gcd(C, Wd)) == 0
+        assert ("fold_flag" in o.source()) == fold, o.info()["launches"][0]
+        assert ("__funnelshift_r" in o.source()) == (not fold and C >= Wd), o.info()["launches"][0]
     ref = O.run(d, x)["out"]
     if op == "max":
         assert_bitexact(got["out"], ref, "out")

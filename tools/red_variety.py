@@ -58,16 +58,29 @@ CASES = [
 
 
 def time_op(run, sets, n=20, reps=5):
+    """Median per-launch ms over `reps` batches of `n` launches rotating over `sets`.
+    The batch is captured once in a CUDA graph and replayed, so a small operator is
+    timed on the device rather than by the host's per-call launch cost (eager
+    launches if the capture fails)."""
     import statistics
     for i in range(3):
         run(sets[i % len(sets)])
     torch.cuda.synchronize()
+    batch = lambda: [run(sets[i % len(sets)]) for i in range(n)]  # noqa: E731
+    try:
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            batch()
+        g.replay()
+        torch.cuda.synchronize()
+        batch = g.replay
+    except Exception:   # not capturable: eager launches
+        torch.cuda.synchronize()
     per = []
     for _ in range(reps):
         s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         s.record()
-        for i in range(n):
-            run(sets[i % len(sets)])
+        batch()
         e.record()
         torch.cuda.synchronize()
         per.append(s.elapsed_time(e) / n)

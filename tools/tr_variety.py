@@ -7,7 +7,6 @@ the same bytes.  Prints one JSON line per case.
 """
 import json
 import os
-import statistics
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -34,23 +33,17 @@ CASES = [
     ("NHWC->NCHW f16 7x7 [256,7,7,2048]", lambda: W.nhwc_to_nchw(256, 7, 7, 2048)),
     ("2-D f32 [16384,16384]", lambda: W.transpose2d(16384, 16384, "f32")),
     ("2-D f16 [8192,24576]", lambda: W.transpose2d(8192, 24576, "f16")),
+    ("NHWC->NCHW f16 [256,7,9,64] (H*W=63)", lambda: W.nhwc_to_nchw(256, 7, 9, 64)),
 ]
 
 
 def time_op(run, sets, n=20, reps=5):
-    for i in range(3):
-        run(sets[i % len(sets)])
-    torch.cuda.synchronize()
-    per = []
-    for _ in range(reps):
-        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        s.record()
-        for i in range(n):
-            run(sets[i % len(sets)])
-        e.record()
-        torch.cuda.synchronize()
-        per.append(s.elapsed_time(e) / n)
-    return statistics.median(per)
+    """Graph-replayed batches, as in tools/red_variety.py (one timing method for every sweep)."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("red_variety", os.path.join(ROOT, "tools", "red_variety.py"))
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    return m.time_op(run, sets, n, reps)
 
 
 def main():
