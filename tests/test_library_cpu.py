@@ -409,3 +409,26 @@ def test_integer_kernels_compile_for_sm100a():
     src = op.source()
     assert "fop::imul(" in src and "fop::imax(" in src and "fop::mul2" not in src
     assert "IMAD" in _sass(op.cubin(0)) or "IMUL" in _sass(op.cubin(0))
+
+
+@pytest.mark.parametrize("R,C,dtype,fold", [(65536, 1001, "f16", True), (777, 1001, "f16", False), (40000, 3, "f16", True),
+                                            (5000, 37, "f32", True), (4098, 1002, "f16", False), (4096, 1002, "f16", True),
+                                            (65536, 1000, "f16", False)])
+def test_column_reduction_over_odd_rows_folds_groups_of_rows(R, C, dtype, fold):
+    """COL_REDUCE over dense rows no vector divides: when P = W / gcd(C, W) divides R the
+    kernel reads [R/P, P*C] with aligned full vectors and folds P wide columns per output
+    (workspace holds the P*C sums); otherwise (or for C divisible by W) no fold."""
+    import math
+    d = {"name": "colred", "loops": {"r": R, "c": C},
+         "tensors": {"x": {"shape": [R, C], "dtype": dtype, "role": "in", "init": ("normal", 0.0, 1.0, 71), "strides": None},
+                     "out": {"shape": [C], "dtype": "f32", "role": "out", "init": None, "strides": None}},
+         "stmts": [{"kind": "reduce", "op": "sum", "loops": ["r", "c"], "write": ("out", ["c"]),
+                    "reads": [("x", ["r", "c"])], "expr": [("load", 0)]}]}
+    op = FusedOp(d, jit=0, autotune=0)
+    src, li = op.source(), op.info()["launches"][0]
+    assert li["class"] == "col_reduce" and li["width"] == 16 // (4 if dtype == "f32" else 2)
+    assert ("fold_flag" in src) == fold
+    if fold:
+        P = li["width"] // math.gcd(C, li["width"])
+        assert f"q = rr * {P}u" in src and f"c_ < {C}u" in src
+        assert op.info()["workspace_bytes"] >= P * C * 4
