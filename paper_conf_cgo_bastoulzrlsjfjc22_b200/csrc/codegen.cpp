@@ -2706,13 +2706,14 @@ struct Gen {
       o.l("  #pragma unroll");
       o.l("  for (int e = 0; e < " + num(W) + "; ++e) F_[iv + e] = red[cv * " + num(W) + "u + e];");
       o.l("}");
-      o.l("__threadfence();");
+      if (!L.col_acqrel) o.l("__threadfence();");
       o.l("__syncthreads();");
-      o.l("if (tid == 0u) fold_flag = (atomicAdd(fc_, 1u) == " + num(SVN - 1) + "u);");
+      o.l(std::string("if (tid == 0u) fold_flag = (") + (L.col_acqrel ? "fop::atom_add_acq_rel_gpu" : "atomicAdd") +
+          "(fc_, 1u) == " + num(SVN - 1) + "u);");
       o.l("__syncthreads();");
       o.l("if (fold_flag) {");
       o.ind++;
-      o.l("__threadfence();");
+      if (!L.col_acqrel) o.l("__threadfence();");
       o.l("for (unsigned c_ = tid; c_ < " + num(EV0) + "u; c_ += " + num(L.block) + "u) {");
       o.ind++;
       o.l("float a_ = " + init + ";");
@@ -2841,13 +2842,17 @@ struct Gen {
       o.l("  for (int e = 0; e < " + num(W) + "; ++e) part[(chunk * " + num(slabs) + "u + slab) * " + num(SW) +
           "u + cv * " + num(W) + "u + e] = red[cv * " + num(W) + "u + e];");
       o.l("}");
-      o.l("__threadfence();");
+      // arrival: membar.gl in every thread + relaxed atomic (default), or one
+      // acq_rel atomic after the barrier (FOP_COL_ACQREL=1, default)
+      const bool acqrel = L.col_acqrel;
+      if (!acqrel) o.l("__threadfence();");
       o.l("__syncthreads();");
-      o.l("if (tid == 0u) last_flag = (atomicAdd(&cnt[slab], 1u) == " + num(NCH - 1) + "u);");
+      o.l(std::string("if (tid == 0u) last_flag = (") + (acqrel ? "fop::atom_add_acq_rel_gpu" : "atomicAdd") +
+          "(&cnt[slab], 1u) == " + num(NCH - 1) + "u);");
       o.l("__syncthreads();");
       o.l("if (last_flag) {");
       o.ind++;
-      o.l("__threadfence();");
+      if (!acqrel) o.l("__threadfence();");
       o.l("#pragma unroll");
       o.l("for (int e = 0; e < " + num(W) + "; ++e) acc[e] = " + init + ";");
       // every partial this thread combines is requested before the first is

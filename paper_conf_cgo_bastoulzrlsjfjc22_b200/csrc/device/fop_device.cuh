@@ -616,6 +616,15 @@ __device__ __forceinline__ void mbar_wait(u64* bar, u32 phase) {
   while (!mbar_try(bar, phase)) {
   }
 }
+// Arrival counter with acquire-release semantics at GPU scope: one
+// atomic carries the release of the CTA's partial stores (ordered before it by
+// bar.sync, release is cumulative) and the acquire of the other CTAs' (for the
+// last arrival), instead of membar.gl in every thread plus a relaxed atomic.
+__device__ __forceinline__ unsigned atom_add_acq_rel_gpu(unsigned* p, unsigned v) {
+  unsigned old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
 __device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 template <int N>

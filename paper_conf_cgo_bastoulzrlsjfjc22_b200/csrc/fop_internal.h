@@ -177,6 +177,7 @@ struct Launch {
   size_t ws_off = 0, ws_bytes = 0;  // COL_REDUCE partials + counters
   std::vector<int> align;         // per tensor: byte alignment the vector variant assumes
   bool scalar_variant = false;    // this launch is the narrow (W=1) variant
+  int col_acqrel = 0;             // COL finalize: one acq_rel arrival atomic instead of membar.gl + relaxed atomic
   int col_fold = 0;               // COL: dense odd rows read as [R/P, P*E] (P rows per aligned group), folded at the end
   size_t fold_off = 0;            // COL fold: wide-column sums + counter, offset inside the launch's workspace
   int col_shift = 0;              // COL: full-width vectors over odd rows via per-row funnel shifts of aligned chunks

@@ -808,6 +808,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     // finalize: store + fence + arrival counter + last-arriving block (0, default),
     // or flag words polled by the slab's last chunk block (1) / last arrival (2)
     L.col_fin = L.col_fold ? 0 : knob("FOP_COL_FIN", 0);
+    L.col_acqrel = knob("FOP_COL_ACQREL", 1);   // measured: cfg4b 25.07 -> 25.00 us, odd fold 27.36 -> 26.97 (profiles/r02/sweep_r02_acqrel.log)
     if (nch > 1 && L.col_fin) {
       L.ws_bytes = ((size_t)nch * (size_t)slabs * (size_t)(gv * W) * sizeof(unsigned long long) + 255) & ~size_t(255);
       if (L.col_fin == 2) L.ws_bytes += (size_t)slabs * sizeof(unsigned);
