@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -358,6 +358,37 @@ zf)
   grep "fop tune" gpurun_out/bench_zf.err | grep col
   tail -1 gpurun_out/bench_zf.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),round(d['roofline']['frac'],3),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
   done
+  ;;
+col_fold)
+  # COL over odd rows: parity of the fold/shift/shfl modes + integer reductions, then the odd-extent sweep
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  timeout 1500 python -m pytest tests/test_odd_gpu.py tests/test_int_gpu.py -q -x -m gpu > gpurun_out/pytest_col.log 2>&1; echo pytest=$?
+  tail -3 gpurun_out/pytest_col.log
+  timeout 600 python tools/odd_variety.py > gpurun_out/odd_variety_fold.log 2>&1; echo odd=$?
+  cut -c1-200 gpurun_out/odd_variety_fold.log
+  ;;
+acqrel)
+  # COL finalize: acq_rel arrival atomic vs membar.gl + relaxed atomic (cfg4b, odd fold), parity under it
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  S="timeout 300 python tools/sweep.py"
+  A="opt:autotune=0"
+  for i in 1 2; do
+  $S cfg4b "$A" "$A,FOP_COL_ACQREL=1" "$A,FOP_COL_U=2,FOP_COL_MINB=8" "$A,FOP_COL_U=2,FOP_COL_MINB=8,FOP_COL_ACQREL=1" 2>&1 | cut -c1-160
+  $S colsum_1001 "$A" "$A,FOP_COL_ACQREL=1" "$A,FOP_COL_FOLD=0" 2>&1 | cut -c1-160
+  done
+  FOP_COL_ACQREL=1 timeout 1200 python -m pytest tests/test_parity_gpu.py tests/test_repeat_runs.py tests/test_odd_gpu.py tests/test_full_size_gpu.py -q -x -k "col or colsum or cfg4b or repeat or reduce or odd" > gpurun_out/pytest_acqrel.log 2>&1; echo pytest=$?
+  tail -1 gpurun_out/pytest_acqrel.log
+  ;;
+final)
+  # Round-2 closing evidence on HEAD: variety sweeps (graph-timed), bench line, smoke
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  timeout 900 python tools/odd_variety.py > gpurun_out/odd_variety_final.log 2>&1; echo odd=$?
+  timeout 900 python tools/tr_variety.py > gpurun_out/tr_variety_final.log 2>&1; echo tr=$?
+  timeout 900 python tools/red_variety.py > gpurun_out/red_variety_final.log 2>&1; echo red=$?
+  timeout 900 python bench.py > gpurun_out/bench_final.log 2>&1; echo bench=$?
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
