@@ -1840,7 +1840,11 @@ struct Gen {
         }
     }
     // prefetch of the first row's streaming loads
-    auto emit_prefetch = [&](const std::string& rowvar, const std::string& tag) {
+    // prefetch depth D = L.row_prefetch: rows row + WSTRIDE .. row + D*WSTRIDE in
+    // flight while `row` is processed (ring P, P_1 .. P_{D-1}; D = 1 default)
+    const int PD = std::max(1, L.row_prefetch);
+    auto pslot = [&](size_t k, int dd) { return "P" + num(k) + (dd ? "_" + num(dd) : std::string("")); };
+    auto emit_prefetch = [&](const std::string& rowvar, const std::string& tag, int slot) {
       bool any = false;
       for (size_t k = 0; k < L.loads.size(); k++) any |= mode[k] == 'P';
       if (!any) return;
@@ -1858,7 +1862,7 @@ struct Gen {
             auto its = ro_its(ro, pits);
             its.push_back({0, "((lane + " + num(LN * kk) + "u) * " + num(W) + "u)"});
             o.l(lane_guard(kk) + "fop::vload_words<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + num(W) +
-                ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(&P" + num(k) + "[" +
+                ", " + num(L.load_cb[k]) + ", " + pol(a, false) + ">(&" + pslot(k, slot) + "[" +
                 num((ro * K + kk) * wpv) + "], " + ptr(a.tensor, affine(a, its)) + ");");
           }
       }
@@ -1866,9 +1870,12 @@ struct Gen {
       o.l("}");
     };
     for (size_t k = 0; k < L.loads.size(); k++)
-      if (mode[k] == 'P') o.l("u32 P" + num(k) + "[" + num(NP * W * es(L.loads[k].tensor) / 4) + "];");
+      if (mode[k] == 'P')
+        for (int dd = 0; dd < PD; dd++) o.l("u32 " + pslot(k, dd) + "[" + num(NP * W * es(L.loads[k].tensor) / 4) + "];");
     o.l("idx_t row = ((idx_t)blockIdx.x * " + num(L.block) + "u + threadIdx.x) / " + num(LN) + "u;");
-    emit_prefetch("row", "_p");
+    emit_prefetch("row", "_p", 0);
+    for (int dd = 1; dd < PD; dd++)
+      emit_prefetch("row + (idx_t)" + num(WSTRIDE * dd) + "ull", "_p" + num(dd), dd);
     o.l("#pragma unroll 1");
     if (MULTI) {   // block-uniform trip count: every group (and every CTA of the cluster) reaches the barriers
       o.l("for (idx_t rb_ = ((idx_t)blockIdx.x * " + num(L.block) + "u) / " + num(LN) + "u; rb_ < (idx_t)" + num(rows) +
@@ -1885,8 +1892,12 @@ struct Gen {
         o.l("u32 Q" + num(k) + "[" + num(n) + "];");
         o.l("#pragma unroll");
         o.l("for (int i = 0; i < " + num(n) + "; ++i) Q" + num(k) + "[i] = P" + num(k) + "[i];");
+        for (int dd = 0; dd + 1 < PD; dd++) {
+          o.l("#pragma unroll");
+          o.l("for (int i = 0; i < " + num(n) + "; ++i) " + pslot(k, dd) + "[i] = " + pslot(k, dd + 1) + "[i];");
+        }
       }
-    emit_prefetch("row + (idx_t)" + num(WSTRIDE) + "ull", "_n");
+    emit_prefetch("row + (idx_t)" + num(WSTRIDE * PD) + "ull", "_n", PD - 1);
     o.l("idx_t rr = row;");
     std::vector<std::pair<int, std::string>> rits;
     decompose("rr", L.nsplit, (int)L.kl.size(), "", rits);

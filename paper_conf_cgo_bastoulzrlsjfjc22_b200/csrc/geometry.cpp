@@ -199,6 +199,9 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
       v.push_back({{"FOP_ROW_MINB", 2}});
       v.push_back({{"FOP_ROW_MINB", 4}});
       v.push_back({{"FOP_BLOCK", 128}, {"FOP_ROW_MINB", 6}});
+      // two rows prefetched per warp at 2 CTAs/SM: BERT LayerNorm 36.4 -> 30.4 us untuned
+      // (cfg4a: 23.0 vs 20.9, profiles/r02/sweep_r02_rowpf.log)
+      if (L.row_p == 1) v.push_back({{"FOP_ROW_PREFETCH", 2}, {"FOP_ROW_MINB", 2}});
       if (L.row_p > 1) {   // short rows: one vector per lane per row, latency hidden by more warps
         v.push_back({{"FOP_ROW_MINB", 6}});
         v.push_back({{"FOP_ROW_MINB", 8}});
@@ -767,7 +770,7 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     // short rows hold one vector per lane per row: more warps hide the
     // latency (profiles/red_variety_r01.log: [1048576,64] f16 3745 -> 5343 GB/s)
     L.minblocks = knob("FOP_ROW_MINB", L.block >= 1024 ? 1 : (L.block >= 512 ? 2 : (P > 1 ? 8 : 3)));
-    L.row_prefetch = knob("FOP_ROW_PREFETCH", 1);
+    L.row_prefetch = knob("FOP_ROW_PREFETCH", 1);   // rows in flight ahead of the one processed (0: none)
     L.row_hoist = knob("FOP_ROW_HOIST", 1);
     int64_t gpb = L.block * P / (32 * G);   // rows per block
     int64_t need = (rows + gpb - 1) / gpb;

@@ -484,8 +484,10 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
       reps = reps < 3 ? 3 : (reps > 40 ? 40 : reps);
     }
     // the default geometry is the rule the sweeps settled on: a candidate
-    // replaces it only when it is clearly faster (> 2 %), not on timing noise
-    // (BERT LayerNorm: candidates within 3 % swapped ranks between runs)
+    // replaces it only when it is clearly faster (> 1.5 %), not on timing noise
+    // (BERT LayerNorm: candidates within 3 % swapped ranks between runs; at 2 %
+    // cfg2's 32-byte geometry, 2.0-3.0 % ahead in every cold timing and 6.5 %
+    // in steady state, lost to the default in one bench run of three)
     int best = 0;
     float best_ms = 0.f, def_ms = 0.f;
     std::vector<float> tlog;
@@ -498,7 +500,7 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
         best_ms = ms;
       }
     }
-    if (best != 0 && best_ms > 0.98f * def_ms) best = 0;
+    if (best != 0 && best_ms > 0.985f * def_ms) best = 0;
     if (const char* lg = std::getenv("FOP_TUNE_LOG"); lg && *lg == '1') {   // diagnostics: the candidates' times
       std::fprintf(stderr, "[fop tune] launch %zu (%s): %s", i, scratch ? "cold" : "hot", p.launches[i].name.c_str());
       for (size_t k = 0; k < tlog.size(); k++) std::fprintf(stderr, " v%zu=%.1fus", k, 1e3f * tlog[k]);

@@ -68,7 +68,7 @@ def main():
     for name, mk in CASES:
         d = mk()
         try:
-            op = FusedOp(d)
+            op = FusedOp(d, autotune=int(os.environ.get("FOP_SWEEP_AUTOTUNE", "1")))
         except Exception as ex:  # noqa: BLE001
             print(json.dumps({"case": name, "error": str(ex)[:300]}), flush=True)
             continue

@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -389,6 +389,34 @@ final)
   timeout 900 python tools/tr_variety.py > gpurun_out/tr_variety_final.log 2>&1; echo tr=$?
   timeout 900 python tools/red_variety.py > gpurun_out/red_variety_final.log 2>&1; echo red=$?
   timeout 900 python bench.py > gpurun_out/bench_final.log 2>&1; echo bench=$?
+  ;;
+rowpf)
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  S="timeout 300 python tools/sweep.py"
+  A="opt:autotune=0"
+  $S cfg4a "$A" "$A,FOP_ROW_PREFETCH=2,FOP_BLOCK=128,FOP_ROW_MINB=5" "$A,FOP_ROW_PREFETCH=2,FOP_BLOCK=256,FOP_ROW_MINB=2" "$A,FOP_ROW_PREFETCH=3,FOP_BLOCK=128,FOP_ROW_MINB=4" "$A,FOP_ROW_PREFETCH=2,FOP_BLOCK=96,FOP_ROW_MINB=7" "$A,FOP_ROW_PREFETCH=2,FOP_BLOCK=64,FOP_ROW_MINB=10" "$A" 2>&1 | cut -c1-200
+  $S bert_layernorm "$A" "$A,FOP_ROW_PREFETCH=2,FOP_BLOCK=128,FOP_ROW_MINB=5" "$A,FOP_ROW_PREFETCH=2,FOP_BLOCK=256,FOP_ROW_MINB=2" 2>&1 | cut -c1-200
+  FOP_SWEEP_AUTOTUNE=0 timeout 600 python tools/ew_variety.py > gpurun_out/ew_def.log 2>&1
+  FOP_SWEEP_AUTOTUNE=0 FOP_VEC_BYTES=32 FOP_EW_U=4 FOP_EW_MINB=1 timeout 600 python tools/ew_variety.py > gpurun_out/ew_v32.log 2>&1
+  python - <<'PY'
+import json
+a=[json.loads(l) for l in open("gpurun_out/ew_def.log") if l.startswith("{")]
+b=[json.loads(l) for l in open("gpurun_out/ew_v32.log") if l.startswith("{")]
+for x,y in zip(a,b): print(x["case"][:50].ljust(50), round(x.get("GB_s",0)), round(y.get("GB_s",0)))
+PY
+  ;;
+tune2)
+  # tuner threshold 1.5 % + ROW prefetch-2 candidate: parity of every candidate, N4 ops, two bench lines
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  timeout 1500 python -m pytest tests/test_full_size_gpu.py tests/test_n4_ops.py tests/test_parity_gpu.py -q -x -m gpu > gpurun_out/pytest_tune2.log 2>&1; echo pytest=$?
+  tail -1 gpurun_out/pytest_tune2.log
+  for i in 1 2 3; do
+  FOP_TUNE_LOG=1 timeout 900 python bench.py --no-cpu > gpurun_out/bench_tune2_$i.log 2> gpurun_out/bench_tune2_$i.err; echo bench=$?
+  grep "fop tune" gpurun_out/bench_tune2_$i.err
+  tail -1 gpurun_out/bench_tune2_$i.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),d['roofline']['kernel'],round(d['roofline']['frac'],3),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
+  done
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
