@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -417,6 +417,15 @@ tune2)
   grep "fop tune" gpurun_out/bench_tune2_$i.err
   tail -1 gpurun_out/bench_tune2_$i.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),d['roofline']['kernel'],round(d['roofline']['frac'],3),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
   done
+  ;;
+rowhoist)
+  # cfg4a: bias reloaded per row (FOP_ROW_HOIST=0) to fit 64 registers and 32 warps/SM
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  S="timeout 300 python tools/sweep.py"
+  A="opt:autotune=0"
+  $S cfg4a "$A" "$A,FOP_ROW_HOIST=0" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=4" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=5,FOP_BLOCK=192" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=8,FOP_BLOCK=128" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=16,FOP_BLOCK=64" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=4,FOP_ROW_PREFETCH=0" "$A" 2>&1 | cut -c1-220
+  $S bert_layernorm "$A" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=4" 2>&1 | cut -c1-220
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
