@@ -154,3 +154,40 @@ def test_transpose_software_pipelined_bitexact(monkeypatch, dims, dtype, knobs):
     got, op = run_gpu(d, x, autotune=0)
     assert "next iteration's loads in flight" in op.source()
     assert_bitexact(got["out"], O.run(d, x)["out"], "out")
+
+
+@pytest.mark.parametrize("seed", list(range(12)))
+def test_column_reduction_fold_random_shapes(seed):
+    """Random dense odd-row column reductions on the fold path (P = W/gcd(C, W) rows per
+    aligned group, R a multiple of P, 1-3 groups per chunk up to thousands): f16/bf16/f32
+    sums of x, x*x or relu(x) (normwise, R16), maxima (bit-exact), i32 wrap-around sums
+    (bit-exact); every auto-tuning candidate."""
+    import math
+    from harness import abs_terms_desc, assert_normwise
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    rng = np.random.default_rng(1000 + seed)
+    dtype = ["f16", "bf16", "f32", "i32"][seed % 4]
+    Wd = 16 // (4 if dtype in ("f32", "i32") else 2)
+    C = int(rng.choice([3, 5, 7, 9, 13, 37, 99, 255, 1001, 1003, 2047, 6]))
+    if C % Wd == 0:
+        C += 1
+    P = Wd // math.gcd(C, Wd)
+    R = P * [1, 2, 17, 128, 1000, 4099, 3, 9000, 64, 257, 5000, 31][seed]
+    op = "max" if seed % 3 == 2 else "sum"
+    expr = [("load", 0)] if op == "max" or dtype == "i32" else \
+        [[("load", 0)], [("load", 0), ("mul", 0, 0)], [("load", 0), ("relu", 0)]][seed % 3]
+    d = _colred(R, C, dtype, op, expr)
+    if dtype == "i32":
+        d["tensors"]["x"]["init"] = ("randint", -2 ** 30, 2 ** 30, 500 + seed)
+        d["tensors"]["out"]["dtype"] = "i32"
+    x = W.make_inputs(d)
+    ref = O.run(d, x)["out"]
+    assert "fold_flag" in FusedOp(d).source(), (R, C, dtype)
+    nv = FusedOp(d).info()["launches"][0]["nvariants"]
+    for k in range(nv):
+        got, o = run_gpu(d, x, variant=k)
+        tag = f"R={R} C={C} {dtype} {op} candidate {k}"
+        if op == "max" or dtype == "i32":
+            assert_bitexact(got["out"], ref, tag)
+        else:
+            assert_normwise(got["out"], ref, O.run(abs_terms_desc(d, 0), x)["out"], 1e-5, tag)
