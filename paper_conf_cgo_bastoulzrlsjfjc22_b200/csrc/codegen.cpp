@@ -2217,6 +2217,7 @@ struct Gen {
     header("COL_REDUCE (slab of gv x W columns, row chunks, fixed-order trees)", 1);
     o.l("__shared__ float red[" + num(L.block * W) + "];");
     o.l("__shared__ unsigned last_flag;");
+    o.l("(void)last_flag;   // (used by multi-chunk finalizes only)");
     if (FP) o.l("__shared__ unsigned fold_flag;");
     o.l("const unsigned tid = threadIdx.x, cv = tid % " + num(L.gv) + "u, rl = tid / " + num(L.gv) + "u;");
     o.l("const idx_t slab = blockIdx.x % " + num(slabs) + "u, chunk = blockIdx.x / " + num(slabs) + "u;");
@@ -2730,6 +2731,33 @@ struct Gen {
       o.l("float a_ = " + init + ";");
       o.l("#pragma unroll");
       o.l("for (int g = 0; g < " + num(FP) + "; ++g) a_ = " + comb("a_", "__ldcg(&F_[g * " + num(EV0) + "u + c_])") + ";");
+      // the R mod P rows after the last whole group, element-wise, in row order
+      const int64_t RT = L.kl[1].extent, R0 = RT - RT % FP;
+      if (R0 < RT) {
+        o.l("#pragma unroll 1");
+        o.l("for (unsigned tr_ = " + num(R0) + "u; tr_ < " + num(RT) + "u; ++tr_) {");
+        o.ind++;
+        const std::vector<std::pair<int, std::string>> tits = {{0, "(idx_t)c_"}, {1, "(idx_t)tr_"}};
+        for (size_t k = 0; k < L.loads.size(); k++) {
+          const Affine& a = L.loads[k];
+          o.l("float L" + num(k) + "_t[1];");
+          o.l("L" + num(k) + "_t[0] = fop::sload<" + std::string(dtn(d.t[a.tensor].dtype)) + ", " + pol(a, true) + ">(" +
+              ptr(a.tensor, affine(a, tits)) + ");");
+        }
+        DagCtx tc;
+        tc.tag = "_t";
+        tc.load_varies = [](int) { return true; };
+        tc.load = [&](int k, const std::string& e) { return "L" + num(k) + "_t[" + e + "]"; };
+        tc.fwd = [&](int, const std::string&) { return std::string("0.f"); };
+        tc.scalar = [&](int) { return std::string("0.f"); };
+        auto tvar = varies(x, tc);
+        emit_nodes(o, x, tvar, false, tc);
+        Sink tsk;
+        tsk.scalar = [&](const std::string& v) { o.l("a_ = " + comb("a_", v) + ";"); };
+        emit_elems(o, x, tvar, tc, 1, tsk);
+        o.ind--;
+        o.l("}");
+      }
       std::string r = fin_expr(o, x, "a_", "");
       std::vector<std::pair<int, std::string>> fc = {{0, "(idx_t)c_"}};
       o.l("fop::sstore<" + std::string(dtn(x.out_dtype)) + ">(" + ptr(x.write.tensor, affine(x.write, fc)) + ", " + r + ");");

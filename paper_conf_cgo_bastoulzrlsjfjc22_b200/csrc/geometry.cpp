@@ -218,6 +218,11 @@ std::vector<std::vector<std::pair<std::string, int>>> tuning_variants(const Laun
 static int knob_w_cap(const Launch& L) { return geometry_knob(L, "FOP_SEQ_W", 1 << 20); }
 
 void finalize_launch_geometry(const Plan& p, Launch& L) {
+  // variants start as copies of the planned launch: a flag one class sets must
+  // not survive into a copy that ends in another class (the narrow variant of a
+  // transpose becomes EW with gathers; a stale tma = 1 sent misaligned pointers
+  // to cuTensorMapEncodeTiled — fuzz seed 41, tests/fuzz_regressions/)
+  L.tma = 0;
   const fop_desc& d = p.desc;
   const fop_plan_opts& o = p.opts;
   auto acc = all_accesses(L);
@@ -398,18 +403,19 @@ void finalize_launch_geometry(const Plan& p, Launch& L) {
     }
     if (ok) L.col_shift = 1;
   }
-  // ... and when the rows are dense (pitch E[d_v]) and P = W / gcd(E, W)
-  // divides the row count, P consecutive rows are P*E elements: a whole
-  // number of aligned W-vectors.  Read the matrix as [R/P, P*E] — full-width
-  // aligned vectors, no shifts — where lane j's element e always falls on
-  // column (j*W + e) mod E (of row (j*W + e) div E inside the group); the last
-  // block to finish folds the P*E wide-column sums into the E outputs, P
-  // terms each in group-row order (the vector access is kept whole).
+  // ... and when the rows are dense (pitch E[d_v]), with P = W / gcd(E, W),
+  // P consecutive rows are P*E elements: a whole number of aligned W-vectors.
+  // Read the first R - R mod P rows as [R/P, P*E] — full-width aligned
+  // vectors, no shifts — where lane j's element e always falls on column
+  // (j*W + e) mod E (of row (j*W + e) div E inside the group); the last block
+  // to finish folds the P*E wide-column sums into the E outputs, P terms each
+  // in group-row order, then adds the R mod P remaining rows element-wise
+  // (the vector access is kept whole, scalar accesses mixed in).
   L.col_fold = 0;
   if (L.kclass == FOP_CLASS_COL_REDUCE && W > 1 && EV % W != 0 && L.nsplit == 1 && L.kl.size() == 2 &&
       !L.scalar_variant && L.stmts.size() == 1 && p.opts.peer_world < 1 && geometry_knob(L, "FOP_COL_FOLD", 1)) {
     const int64_t P = W / std::gcd<int64_t>(EV, W);
-    bool ok = L.kl[1].extent % P == 0 && coef(L, L.stmts[0].write, 0) == 1 && coef(L, L.stmts[0].write, 1) == 0;
+    bool ok = L.kl[1].extent >= P && coef(L, L.stmts[0].write, 0) == 1 && coef(L, L.stmts[0].write, 1) == 0;
     for (const auto& a : L.loads) {
       const int es_a = esize(d.t[a.tensor].dtype);
       ok &= coef(L, a, 0) == 1 && coef(L, a, 1) == EV && W * es_a == 16 && a.base * es_a % 16 == 0;

@@ -171,3 +171,20 @@ def test_fuzz_regression_descriptors_match_oracle(name, d):
     sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools"))
     from fuzz_campaign import check
     check(d, repeat=True)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("name,d", _regression_descs())
+def test_fuzz_regression_descriptors_run(name, d):
+    """Every fuzz regression through the campaign's own sequence: a first (tuning) run, then
+    aligned, misaligned (narrow variant) and aligned runs of the same plan, all against the
+    oracle.  tma_seed41_case273: a 128x128 bf16 transpose on the TMA tiles (round 2's
+    default) failed cuTensorMapEncodeTiled on one of the repeat runs."""
+    import importlib.util
+    import os
+    spec = importlib.util.spec_from_file_location(
+        "fuzz_campaign", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools",
+                                      "fuzz_campaign.py"))
+    fc = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(fc)
+    fc.check(d, repeat=True)

@@ -411,13 +411,14 @@ def test_integer_kernels_compile_for_sm100a():
     assert "IMAD" in _sass(op.cubin(0)) or "IMUL" in _sass(op.cubin(0))
 
 
-@pytest.mark.parametrize("R,C,dtype,fold", [(65536, 1001, "f16", True), (777, 1001, "f16", False), (40000, 3, "f16", True),
-                                            (5000, 37, "f32", True), (4098, 1002, "f16", False), (4096, 1002, "f16", True),
-                                            (65536, 1000, "f16", False)])
+@pytest.mark.parametrize("R,C,dtype,fold", [(65536, 1001, "f16", True), (777, 1001, "f16", True), (40000, 3, "f16", True),
+                                            (5000, 37, "f32", True), (4098, 1002, "f16", True), (4096, 1002, "f16", True),
+                                            (65536, 1000, "f16", False), (7, 1001, "f16", False), (3, 1002, "f16", False)])
 def test_column_reduction_over_odd_rows_folds_groups_of_rows(R, C, dtype, fold):
-    """COL_REDUCE over dense rows no vector divides: when P = W / gcd(C, W) divides R the
-    kernel reads [R/P, P*C] with aligned full vectors and folds P wide columns per output
-    (workspace holds the P*C sums); otherwise (or for C divisible by W) no fold."""
+    """COL_REDUCE over dense rows no vector divides: with R >= P = W / gcd(C, W) the kernel
+    reads the first R - R mod P rows as [R/P, P*C] with aligned full vectors and folds P wide
+    columns per output (workspace holds the P*C sums), the R mod P tail rows added
+    element-wise by the folding block; fewer rows than P (or C divisible by W): no fold."""
     import math
     d = {"name": "colred", "loops": {"r": R, "c": C},
          "tensors": {"x": {"shape": [R, C], "dtype": dtype, "role": "in", "init": ("normal", 0.0, 1.0, 71), "strides": None},
@@ -431,4 +432,5 @@ def test_column_reduction_over_odd_rows_folds_groups_of_rows(R, C, dtype, fold):
     if fold:
         P = li["width"] // math.gcd(C, li["width"])
         assert f"q = rr * {P}u" in src and f"c_ < {C}u" in src
+        assert ("tr_ < " in src) == (R % P != 0)
         assert op.info()["workspace_bytes"] >= P * C * 4

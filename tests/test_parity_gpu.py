@@ -609,3 +609,24 @@ def test_cuda_graph_capture_and_replay(warm):
                     assert_normwise(got, ref[n], scale, 1e-5, n)
                 else:
                     assert_bitexact(got, ref[n], f"{d['name']} {n}")
+
+
+@pytest.mark.parametrize("mk", [lambda: W.cfg3(2, 64, 8, 8), lambda: W.transpose2d(128, 192, "bf16"),
+                                lambda: W.nhwc_to_nchw(2, 8, 8, 64)])
+@pytest.mark.parametrize("offset", [1, 4, 8])
+def test_tma_transpose_misaligned_pointers_take_the_narrow_variant(mk, offset):
+    """16-bit transposes plan onto TMA tiles (16 B-aligned tensor-map base addresses):
+    pointers off that alignment must run the narrow variant (an EW kernel with gathers),
+    never the tensor-map path; aligned runs of the same plan before and after stay exact."""
+    from harness import device_tensors, to_host
+    d = mk()
+    x = W.make_inputs(d)
+    ref = O.run(d, x)["out"]
+    got, op = run_gpu(d, x)
+    assert "cp.async.bulk.tensor" in op.source() or "tma" in op.selected(0)[0], op.selected(0)
+    assert_bitexact(got["out"], ref, "aligned")
+    for off in (offset, 0):
+        dev = device_tensors(d, x, offset=off)
+        op.run(dev)
+        torch.cuda.synchronize()
+        assert_bitexact(to_host(dev["out"], d["tensors"]["out"]["dtype"]), ref, f"offset {off}")

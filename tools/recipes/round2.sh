@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -426,6 +426,14 @@ rowhoist)
   A="opt:autotune=0"
   $S cfg4a "$A" "$A,FOP_ROW_HOIST=0" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=4" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=5,FOP_BLOCK=192" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=8,FOP_BLOCK=128" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=16,FOP_BLOCK=64" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=4,FOP_ROW_PREFETCH=0" "$A" 2>&1 | cut -c1-220
   $S bert_layernorm "$A" "$A,FOP_ROW_HOIST=0,FOP_ROW_MINB=4" 2>&1 | cut -c1-220
+  ;;
+suite_fuzz)
+  # full GPU suite + fuzz campaigns on HEAD (compute-sanitizer is closed on this pool)
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  timeout 2400 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu_sf.log 2>&1; echo pytest=$?
+  tail -3 gpurun_out/pytest_gpu_sf.log
+  SEEDS="41 42 43 44 45" COUNT=300 bash tools/gpu_fuzz.sh
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
