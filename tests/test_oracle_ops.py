@@ -375,3 +375,19 @@ def test_int_rejections(expr, dt, msg):
 def test_int_move_keeps_bits():
     a = _irand(100, 34)
     assert np.array_equal(run_int([("load", 0)], [a]), a)
+
+
+def test_every_abi_opcode_has_a_named_pin_here():
+    """Every expression opcode include/fop.h declares (FOP_OP_*) is exercised by a pin in
+    this file (or, for ACC, tests/test_oracle.py) under its descriptor name, so a new opcode
+    cannot reach the ABI unpinned."""
+    import os
+    import re
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    ops = set(re.findall(r"FOP_OP_([A-Z0-9_]+)", open(os.path.join(root, "include", "fop.h")).read()))
+    ops -= {"_COUNT"}
+    # descriptor names are the lower-case opcodes; ACC (a REDUCE's finalize input) is pinned
+    # with the finalize expressions in tests/test_oracle.py
+    src = open(os.path.abspath(__file__)).read() + open(os.path.join(root, "tests", "test_oracle.py")).read()
+    missing = [op for op in sorted(ops) if f'"{op.lower()}"' not in src and f"'{op.lower()}'" not in src]
+    assert not missing, f"opcodes without a pin in tests/test_oracle_ops.py: {missing}"
