@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -434,6 +434,13 @@ suite_fuzz)
   timeout 2400 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu_sf.log 2>&1; echo pytest=$?
   tail -3 gpurun_out/pytest_gpu_sf.log
   SEEDS="41 42 43 44 45" COUNT=300 bash tools/gpu_fuzz.sh
+  ;;
+tma_misalign)
+  # the misaligned-TMA tests and the rest of the GPU suite after them
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  timeout 2400 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu_tm.log 2>&1; echo pytest=$?
+  tail -3 gpurun_out/pytest_gpu_tm.log
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
