@@ -212,10 +212,11 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
   std::vector<bool> reach = reachable(x);
   const std::string e0 = "2 * " + p, e1 = "2 * " + p + " + 1";
   auto opnd = [&](int i) { return var[i] ? pair_name(x, i, c) : "fop::pk1(" + node_name(x, var, i, c) + ")"; };
-  // a packed product feeding a packed add/sub must not be contracted (see fop::nofuse)
-  auto addend = [&](int i) {
-    return var[i] && x.nodes[i].op == FOP_OP_MUL ? "fop::nofuse(" + pair_name(x, i, c) + ", fop_zero)" : opnd(i);
-  };
+  // a packed product must never be contracted into a later packed add/sub (see fop::nofuse):
+  // every packed product is hidden at its source — not only where it feeds an add directly,
+  // since ptxas also sees through value-preserving steps in between (max(p, p), a negation:
+  // fuzz seed 51 case 289, one bf16 ulp off after (x0 - x1) * x1 -> max(p, p) + y)
+  auto addend = [&](int i) { return opnd(i); };
   for (size_t i = 0; i < x.nodes.size(); i++) {
     if (!reach[i] || !var[i] || (int)i == skip) continue;
     const XNode& n = x.nodes[i];
@@ -230,7 +231,7 @@ void emit_nodes_packed(Out& o, const XStmt& x, const std::vector<bool>& var, con
       case X_SELF: e = "fop::pk(" + c.self(e0) + ", " + c.self(e1) + ")"; break;
       case FOP_OP_ADD: e = "fop::add2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
       case FOP_OP_SUB: e = "fop::sub2(" + addend(n.a) + ", " + addend(n.b) + ")"; break;
-      case FOP_OP_MUL: e = "fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + ")"; break;
+      case FOP_OP_MUL: e = "fop::nofuse(fop::mul2(" + opnd(n.a) + ", " + opnd(n.b) + "), fop_zero)"; break;
       case FOP_OP_GELU_TANH:
         e = std::string(g_out_f16 ? "fop::op_gelu_tanh2(" : "fop::op_gelu_tanh2_wide(") + opnd(n.a) + ")";
         break;
@@ -1519,12 +1520,15 @@ struct Gen {
     o.ind++;
     std::string cell = "fop_tile + (((q * " + num(OW) + "u + e) % " + num(EV) + "u) * " + num(TR) + "u + (q * " +
                        num(OW) + "u + e) / " + num(EV) + "u) * " + num(esi) + "u";
-    if (OM) {   // the thread's OW output elements: one or two 16 B shared loads
+    if (OM) {   // the thread's OW output elements: 16 B shared loads (8 or 4 B when the thread's
+                // input bytes are fewer, e.g. 4 bf16 read out under 4 f32 stores — fuzz seed 51)
       const int nw = OW * esi / 4;
+      const int cw = nw % 4 == 0 ? 4 : nw % 2 == 0 ? 2 : 1;   // words per shared load
+      const std::string ty = cw == 4 ? "uint4" : cw == 2 ? "uint2" : "u32";
       o.l("u32 tw_[" + num(nw) + "];");
       o.l("#pragma unroll");
-      o.l("for (int c = 0; c < " + num(nw / 4) + "; ++c) reinterpret_cast<uint4*>(tw_)[c] = "
-          "reinterpret_cast<const uint4*>(fop_tile + q * " + num(OW * esi) + "u)[c];");
+      o.l("for (int c = 0; c < " + num(nw / cw) + "; ++c) reinterpret_cast<" + ty + "*>(tw_)[c] = "
+          "reinterpret_cast<const " + ty + "*>(fop_tile + q * " + num(OW * esi) + "u)[c];");
     }
     auto elem_bits = [&](const std::string& castty) {   // raw element e (u16 or u32 bits)
       if (!OM) return "*reinterpret_cast<const " + castty + "*>(" + cell + ")";

@@ -188,3 +188,29 @@ def test_fuzz_regression_descriptors_run(name, d):
     fc = importlib.util.module_from_spec(spec)
     spec.loader.exec_module(fc)
     fc.check(d, repeat=True)
+
+
+def test_packed_products_are_never_contracted_into_later_adds(tmp_path):
+    """fuzz seed 51 case 289: out = bf16(max(p, p) + y) with p = (x0 - x1) * x1 came out one
+    bf16 ulp off because ptxas saw through max(p, p) and fused the packed product into the add
+    (FFMA2).  Every packed product is now hidden at its source: the kernel's SASS has FMUL2 and
+    no FFMA2 (compiled here with nvcc -fmad=false, as NVRTC compiles it)."""
+    import json
+    import os
+    import shutil
+    import subprocess
+    nvcc = shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
+    cuobjdump = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not (os.path.exists(nvcc) and os.path.exists(cuobjdump)):
+        pytest.skip("needs nvcc + cuobjdump")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    d = json.load(open(os.path.join(root, "tests", "fuzz_regressions", "contract_seed51_case289.json")))
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    src = FusedOp(d, jit=0, autotune=0).source(0)
+    (tmp_path / "k.cu").write_text(src)
+    subprocess.run([nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-fmad=false", "-cubin",
+                    "-I", os.path.join(root, "paper_conf_cgo_bastoulzrlsjfjc22_b200", "csrc", "device"),
+                    "-o", str(tmp_path / "k.cubin"), str(tmp_path / "k.cu")], check=True)
+    sass = subprocess.run([cuobjdump, "-sass", str(tmp_path / "k.cubin")], check=True, capture_output=True,
+                          text=True).stdout
+    assert "FMUL2" in sass and "FFMA2" not in sass

@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -455,6 +455,11 @@ closing)
   tail -1 gpurun_out/bench_closing_ref.log | cut -c1-300
   bash tools/gpu_profile.sh r02d
   SEEDS="46 47 48 49 50 51" COUNT=300 bash tools/gpu_fuzz.sh
+  ;;
+rowtma)
+  # cfg4a-shaped ROW probe: generated register kernel vs a TMA-fed shared-memory row ring
+  set -x
+  cd tools/probes && nvcc -gencode arch=compute_100a,code=sm_100a -O3 -fmad=false -I ../../paper_conf_cgo_bastoulzrlsjfjc22_b200/csrc/device -o /tmp/row_tma_probe row_tma_probe.cu && /tmp/row_tma_probe
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
