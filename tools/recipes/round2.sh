@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -460,6 +460,20 @@ rowtma)
   # cfg4a-shaped ROW probe: generated register kernel vs a TMA-fed shared-memory row ring
   set -x
   cd tools/probes && nvcc -gencode arch=compute_100a,code=sm_100a -O3 -fmad=false -I ../../paper_conf_cgo_bastoulzrlsjfjc22_b200/csrc/device -o /tmp/row_tma_probe row_tma_probe.cu && /tmp/row_tma_probe
+  ;;
+final2)
+  # after the seed-51 fixes: full GPU suite, fuzz seeds 51-56, smoke, bench x2, ncu evidence
+  set -x
+  python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke_final2.log 2>&1; echo smoke=$?
+  tail -2 gpurun_out/smoke_final2.log
+  timeout 2400 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu_final2.log 2>&1; echo pytest=$?
+  tail -3 gpurun_out/pytest_gpu_final2.log
+  for i in 1 2; do
+  timeout 900 python bench.py > gpurun_out/bench_final2_$i.log 2>&1; echo bench=$?
+  tail -1 gpurun_out/bench_final2_$i.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),d['roofline']['kernel'],round(d['roofline']['frac'],3),d['clocks'],{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
+  done
+  bash tools/gpu_profile.sh r02e
+  SEEDS="51 52 53 54 55 56" COUNT=300 bash tools/gpu_fuzz.sh
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
