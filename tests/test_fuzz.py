@@ -214,3 +214,24 @@ def test_packed_products_are_never_contracted_into_later_adds(tmp_path):
     sass = subprocess.run([cuobjdump, "-sass", str(tmp_path / "k.cubin")], check=True, capture_output=True,
                           text=True).stdout
     assert "FMUL2" in sass and "FFMA2" not in sass
+
+
+def test_generated_kernels_have_no_zero_trip_copy_loops():
+    """Lint over random operators' generated sources: no `for (i = 0; i < 0; ...)` loop — the
+    shape of fuzz seed 51's bug, where a shared-memory read-out sized in 16 B chunks copied
+    nothing for a thread holding 8 B and the kernel stored uninitialised registers."""
+    import re
+    from paper_conf_cgo_bastoulzrlsjfjc22_b200 import FusedOp
+    pat = re.compile(r"for \((?:int|unsigned) (\w+) = 0; \1 < 0u?; ")
+    bad = []
+    for i, d in enumerate(_ops(300, 777)):
+        op = FusedOp(d, jit=0, autotune=0)
+        for k in range(len(op.info()["launches"])):
+            m = pat.search(op.source(k))
+            if m:
+                bad.append((i, k, op.source(k)[m.start():m.start() + 120]))
+    import json
+    d = json.load(open(__import__("os").path.join(__import__("os").path.dirname(__file__), "fuzz_regressions",
+                                                    "trsmem_seed51_case56.json")))
+    assert not pat.search(FusedOp(d, jit=0, autotune=0).source(0))
+    assert not bad, bad[:3]
