@@ -22,11 +22,16 @@ from harness import run_gpu, assert_bitexact, assert_ulp, assert_normwise, abs_t
 from oracle import oracle as O  # noqa: E402
 
 
-def check(d, repeat=False):
+def check(d, repeat=False, variants=False):
     x = W.make_inputs(d)
     got, op = run_gpu(d, x)
     ref = O.run(d, x, outputs=W.alloc_outputs(d))
     compare(d, x, got, ref)
+    if variants:   # every auto-tuning candidate forced in turn (opts.variant), not only the tuner's pick
+        nv = max(li["nvariants"] for li in op.info()["launches"])
+        for k in range(1, nv):
+            got, _ = run_gpu(d, x, variant=k)
+            compare(d, x, got, ref)
     if repeat:   # the same plan again (tuned geometry), a misaligned run (narrow variant), aligned again
         import torch
         from harness import device_tensors, to_host
@@ -65,6 +70,8 @@ def main():
     ap.add_argument("--count", type=int, default=500)
     ap.add_argument("--repeat", action="store_true", help="also re-run each plan (aligned, misaligned, aligned)")
     ap.add_argument("--trace", action="store_true", help="print each case index before running it (crash triage)")
+    ap.add_argument("--variants-every", type=int, default=0,
+                    help="every N-th operator also runs each auto-tuning candidate forced (0: never)")
     a = ap.parse_args()
     rng = np.random.default_rng(a.seed)
     fails, classes = [], {}
@@ -73,7 +80,7 @@ def main():
         if a.trace:
             print("case", i, d["name"], flush=True)
         try:
-            for c in check(d, a.repeat):
+            for c in check(d, a.repeat, a.variants_every > 0 and i % a.variants_every == 0):
                 classes[c] = classes.get(c, 0) + 1
         except Exception as e:  # noqa: BLE001
             fails.append({"case": i, "error": f"{type(e).__name__}: {str(e)[:300]}", "desc": d,
