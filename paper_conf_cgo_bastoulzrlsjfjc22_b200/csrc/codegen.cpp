@@ -379,7 +379,7 @@ struct Gen {
       o.l((written_here(t) ? std::string("char* __restrict__ T") : std::string("const char* __restrict__ T")) +
           num(t) + " = args.p[" + num(t) + "];");
     }
-    o.l("const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;");
+    o.l("const u64 fop_zero = (u64)args.zero;  (void)fop_zero;");
     if ((geometry_knob(L, "FOP_PDL_EMIT", 0) & 1) && geometry_knob(L, "FOP_PDL_POS", 1) == 0)
       o.l("fop::pdl_trigger();");
   }
@@ -1605,7 +1605,7 @@ struct Gen {
     o.l("unsigned char* sin = smem + wid * " + num((S + 2) * 8192) + "u;");
     o.l("unsigned char* sout = sin + " + num(S * 8192) + ";");
     o.l("u64* full = (u64*)(smem + " + num(NW * (S + 2) * 8192) + ") + wid * " + num(S) + "u;");
-    o.l("const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;");
+    o.l("const u64 fop_zero = (u64)args.zero;  (void)fop_zero;");
     if ((geometry_knob(L, "FOP_PDL_EMIT", 0) & 1) && geometry_knob(L, "FOP_PDL_POS", 1) == 0)
       o.l("fop::pdl_trigger();");
     for (int t = 0; t < d.ntensors; t++) {

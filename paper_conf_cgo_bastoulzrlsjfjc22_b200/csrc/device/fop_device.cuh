@@ -385,13 +385,11 @@ __device__ __forceinline__ u64 mul2(u64 a, u64 b) {
 }
 // ptxas (12.9, -O3) contracts mul.rn.f32x2 feeding add.rn.f32x2 into FFMA2
 // even under -fmad=false, which would change the rounding.  OR-ing the
-// product with a zero ptxas cannot prove (%dynamic_smem_size: kernels launch
-// with none) hides the pattern at the cost of one integer op per pair.
-__device__ __forceinline__ u64 opaque_zero() {
-  u32 z;
-  asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(z));
-  return (u64)z;
-}
+// product with a zero ptxas cannot prove hides the pattern at the cost of one
+// integer op per pair.  The zero is FopArgs::zero, a kernel parameter the
+// runtime always sets to 0 (round 2 used %dynamic_smem_size, which is NOT zero
+// in the kernels launched with dynamic shared memory — the TMA transposes —
+// and corrupted their products once every product was hidden).
 __device__ __forceinline__ u64 nofuse(u64 v, u64 zero) { return v | zero; }
 __device__ __forceinline__ u64 fma2(u64 a, u64 b, u64 c) {
   u64 r;
@@ -781,4 +779,5 @@ struct FopArgs {
   char* peer[8];     // exchange buffers of the peer group as seen from this GPU (fop_peer_group)
   unsigned rank;     // this GPU's index in the peer group
   unsigned world;
+  unsigned zero;     // always 0: the opaque zero of fop::nofuse (the runtime zero-fills FopArgs)
 };

@@ -328,6 +328,7 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
     char* ws;
     char* peer[8];
     unsigned rank, world;
+    unsigned zero;   // always 0 (fop::nofuse's opaque zero)
   } args;
   std::memset(&args, 0, sizeof args);
   if (peers && p.peer_bytes) {

@@ -630,3 +630,22 @@ def test_tma_transpose_misaligned_pointers_take_the_narrow_variant(mk, offset):
         op.run(dev)
         torch.cuda.synchronize()
         assert_bitexact(to_host(dev["out"], d["tensors"]["out"]["dtype"]), ref, f"offset {off}")
+
+
+@pytest.mark.parametrize("variant", [0, -1])
+@pytest.mark.parametrize("expr", [
+    [("load", 0), ("const", 0.3), ("mul", 0, 1), ("const", 0.125), ("add", 2, 3)],          # x*s + t
+    [("load", 0), ("load", 0), ("mul", 0, 1), ("load", 0), ("sub", 2, 3)],                  # x*x - x
+    [("load", 0), ("const", -1.7), ("mul", 0, 1), ("neg", 2), ("load", 0), ("add", 3, 4)]])  # -(x*s) + x
+def test_tma_transpose_products_feeding_adds_bitexact(variant, expr):
+    """Products feeding adds inside the TMA transpose (launched with dynamic shared memory):
+    every packed product is hidden from ptxas's contraction by OR-ing an opaque zero, which
+    must be a true zero there too (FopArgs::zero; %dynamic_smem_size was not).  Bit-exact vs
+    the oracle, the default TMA geometry (variant 0) and the tuner's pick."""
+    d = W.cfg3(2, 128, 16, 16)
+    d["stmts"][0]["expr"] = expr
+    x = W.make_inputs(d)
+    got, op = run_gpu(d, x, **({"variant": 0} if variant == 0 else {}))
+    if variant == 0:
+        assert "TRANSPOSE via TMA" in op.source()
+    assert_bitexact(got["out"], O.run(d, x)["out"], "out")

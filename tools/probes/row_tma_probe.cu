@@ -21,7 +21,7 @@ __global__ void __launch_bounds__(256, 3) row_reg(const FopArgs args) {
   char* __restrict__ T2 = args.p[2];
   char* __restrict__ T3 = args.p[3];
   char* __restrict__ T4 = args.p[4];
-  const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;
+  const u64 fop_zero = (u64)args.zero;  (void)fop_zero;
   const idx_t lane = threadIdx.x % 32u;
   float H1[3][8];
   fop::vload<fop::F16, 8, 16, fop::LD_CACHED>(H1[0], (T1 + (u64)((unsigned)(0 + ((lane + 0u) * 8u))) * 2));
@@ -192,7 +192,7 @@ __global__ void __launch_bounds__(256, MINB) row_tma(const FopArgs args) {
   char* __restrict__ T2 = args.p[2];
   char* __restrict__ T3 = args.p[3];
   char* __restrict__ T4 = args.p[4];
-  const u64 fop_zero = fop::opaque_zero();  (void)fop_zero;
+  const u64 fop_zero = (u64)args.zero;  (void)fop_zero;
   extern __shared__ __align__(128) unsigned char sm_[];
   const idx_t lane = threadIdx.x % 32u, warp = threadIdx.x / 32u;
   unsigned char* ring = sm_ + warp * (S * 1536u);
