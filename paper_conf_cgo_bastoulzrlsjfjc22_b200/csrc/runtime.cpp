@@ -501,10 +501,50 @@ fop_status run_plan(Plan& p, void* const* ptrs, int nptrs, void* ws, void* strea
         best_ms = ms;
       }
     }
+    // Candidates the cold timing cannot tell apart (within 1 % of the best) are
+    // ranked by back-to-back timing — how they sustain bandwidth once running —
+    // instead of by the order they were timed in (cfg2: the 32-byte geometry and
+    // a 16-byte one tie at 100.4 us cold, 6547 vs 6249 GB/s back to back).
+    // Only for operators well past L2 (back to back, a smaller one would run L2-hot).
+    int64_t all_bytes = 0;
+    for (int t = 0; t < d.ntensors; t++)
+      if (d.t[t].role != FOP_TEMP) all_bytes += span_bytes(d.t[t]);
+    std::vector<float> hlog(tlog.size(), 0.f);
+    if (scratch && all_bytes >= (int64_t(384) << 20) &&
+        !(std::getenv("FOP_TUNE_TIEBREAK") && *std::getenv("FOP_TUNE_TIEBREAK") == '0')) {
+      std::vector<size_t> tied;
+      for (size_t k = 0; k < tlog.size(); k++)
+        if (tlog[k] <= 1.01f * best_ms) tied.push_back(k);
+      if (tied.size() > 1) {
+        const int hreps = std::max(3, std::min(40, (int)(0.25f / std::max(best_ms, 1e-4f)) + 1));
+        float hbest = 0.f;
+        for (size_t k : tied) {
+          Launch* G = k == 0 ? &p.launches[i] : &p.variants[i][k - 1];
+          CUfunction f = k == 0 ? l.fns[i] : l.vfns[i][k - 1];
+          run_flush();
+          launch_one(G, f);   // warm-up
+          float ms = 0.f;
+          check(c.ev_record(e0, st), "cuEventRecord");
+          for (int r = 0; r < hreps; r++) launch_one(G, f);
+          check(c.ev_record(e1, st), "cuEventRecord");
+          check(c.ev_sync(e1), "cuEventSynchronize");
+          check(c.ev_elapsed(&ms, e0, e1), "cuEventElapsedTime");
+          hlog[k] = ms / hreps;
+          if (k == tied[0] || hlog[k] < hbest) {
+            hbest = hlog[k];
+            best = (int)k;
+          }
+        }
+        best_ms = tlog[best];
+      }
+    }
     if (best != 0 && best_ms > 0.985f * def_ms) best = 0;
     if (const char* lg = std::getenv("FOP_TUNE_LOG"); lg && *lg == '1') {   // diagnostics: the candidates' times
       std::fprintf(stderr, "[fop tune] launch %zu (%s): %s", i, scratch ? "cold" : "hot", p.launches[i].name.c_str());
-      for (size_t k = 0; k < tlog.size(); k++) std::fprintf(stderr, " v%zu=%.1fus", k, 1e3f * tlog[k]);
+      for (size_t k = 0; k < tlog.size(); k++) {
+        std::fprintf(stderr, " v%zu=%.1fus", k, 1e3f * tlog[k]);
+        if (hlog[k] > 0.f) std::fprintf(stderr, "(hot %.1f)", 1e3f * hlog[k]);
+      }
       std::fprintf(stderr, " -> v%d\n", best);
     }
     if (scratch) {
