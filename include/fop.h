@@ -266,7 +266,10 @@ FOP_API fop_status  fop_plan_cubin(const fop_plan_t* plan, int32_t launch, const
 /* Run the fused operator.  dev_ptrs[i] = device base address of desc.t[i]
  * (NULL allowed for TEMP tensors), nptrs = desc.ntensors.  workspace: device
  * buffer of fop_plan_workspace_bytes() bytes, ZERO-FILLED before its first use
- * with this plan (kernels leave it zeroed again), NULL if 0 bytes.
+ * with this plan, NULL if 0 bytes.  It holds COL_REDUCE arrival counters (the
+ * kernels return each to zero) and partial / folded sums (every value a run
+ * reads was written earlier in that run), so it stays valid run after run; one
+ * workspace serves one run at a time (concurrent runs need one each).
  * stream: a CUstream / cudaStream_t (NULL = legacy default stream) of the
  * CURRENT CUDA context.  Asynchronous and stream-ordered.  A base pointer that
  * is not aligned for the planned vector width silently selects a narrower

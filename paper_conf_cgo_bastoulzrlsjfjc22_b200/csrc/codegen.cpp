@@ -345,7 +345,12 @@ struct Gen {
   }
   std::string spol() const {
     const char* e = std::getenv("FOP_STORE_POLICY");
-    return (e && std::strcmp(e, "stream") == 0) ? "fop::ST_STREAM" : "fop::ST_DEFAULT";
+    if (e && std::strcmp(e, "stream") == 0) return "fop::ST_STREAM";
+    // ROW stores evict-first (st.global.cs, FOP_ROW_ST_STREAM=1): the row kernel
+    // leaves DRAM idle (cfg4a: 2.6 TB/s under ncu), so its outputs' write-back
+    // could happen inside its own window instead of the next operator's
+    if (L.kclass == FOP_CLASS_ROW_REDUCE && geometry_knob(L, "FOP_ROW_ST_STREAM", 0)) return "fop::ST_STREAM";
+    return "fop::ST_DEFAULT";
   }
   std::string ptr(int t, const std::string& off) const {
     return "(T" + num(t) + " + (u64)(" + off + ") * " + num(es(t)) + ")";

@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -485,6 +485,17 @@ tiebreak)
   tail -1 gpurun_out/bench_tb_$i.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),d['roofline']['kernel'],round(d['roofline']['frac'],3),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
   done
   timeout 900 python -m pytest tests/test_full_size_gpu.py tests/test_repeat_runs.py -q -m gpu > gpurun_out/pytest_tb.log 2>&1; echo pytest=$?; tail -1 gpurun_out/pytest_tb.log
+  ;;
+rowcs)
+  # ROW stores evict-first (st.global.cs): does cfg4a's y write-back move out of cfg4b's window?
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  b() { timeout 900 python bench.py --no-cpu "$@" 2>/dev/null | tail -1 | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),round(d['roofline']['frac'],3),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"; }
+  for i in 1 2; do
+  echo default; b
+  echo row_cs; FOP_ROW_ST_STREAM=1 b
+  done
+  timeout 300 python tools/sweep.py cfg4a opt:autotune=0 opt:autotune=0,FOP_ROW_ST_STREAM=1 2>&1 | cut -c1-200
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
