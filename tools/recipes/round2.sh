@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs multirank
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -496,6 +496,19 @@ rowcs)
   echo row_cs; FOP_ROW_ST_STREAM=1 b
   done
   timeout 300 python tools/sweep.py cfg4a opt:autotune=0 opt:autotune=0,FOP_ROW_ST_STREAM=1 2>&1 | cut -c1-200
+  ;;
+multirank)
+  # functional check of the N > 1 bench path on one GPU (weak + strong; exchange self-test + in-bench parity), final code
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  for mode in weak strong; do
+  for n in 2 4; do
+  FOP_BENCH_ONE_GPU=1 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node $n --master-addr 127.0.0.1 --master-port 2958$n bench.py --gpus $n --steps 5 --warmup 3 --scaling $mode --no-cpu --no-steady > gpurun_out/bench_onegpu${n}_$mode.log 2>&1; echo $mode$n=$?
+  tail -1 gpurun_out/bench_onegpu${n}_$mode.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),d['n_gpus'],d['scaling'],d['config']['global_batch_scale'],d['config']['exchange_check'],d['config'].get('exchange_note'),d['config']['parallelism'])"
+  done
+  done
+  timeout 900 python bench.py --steps 5 --warmup 3 --scaling strong --no-cpu --no-steady > gpurun_out/bench_strong1_final.log 2>&1; echo strong1=$?
+  tail -1 gpurun_out/bench_strong1_final.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),d['scaling'],d['config']['global_batch_scale'],d['ms_per_step'])"
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
