@@ -66,7 +66,7 @@ struct Cuda {
   CUresult (*tmap_encode)(void*, int, unsigned, void*, const uint64_t*, const uint64_t*, const unsigned*,
                           const unsigned*, int, int, int, int);
 };
-enum { CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES = 8 };
+enum { CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES = 8, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT = 9 };
 // cuLaunchKernelEx configuration (layout of cuda.h's CUlaunchConfig /
 // CUlaunchAttribute; the attribute value is a 64-byte union)
 struct LaunchAttr {
@@ -179,6 +179,11 @@ CUfunction load_fn(const Launch& L, std::vector<void*>& mods) {
   check(cuda().mod_func(&f, m, L.name.c_str()), "cuModuleGetFunction");
   if (L.tma && L.smem > 48 * 1024)
     check(cuda().func_attr(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)L.smem), "cuFuncSetAttribute");
+  // FOP_CARVEOUT=<percent>: one shared-memory carveout preference for every kernel
+  // (measurement knob: kernels with different carveouts back to back make the SM
+  // reconfigure its L1/shared split between them)
+  if (const char* cv = std::getenv("FOP_CARVEOUT"); cv && *cv)
+    check(cuda().func_attr(f, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, std::atoi(cv)), "cuFuncSetAttribute");
   mods.push_back(m);
   return f;
 }
