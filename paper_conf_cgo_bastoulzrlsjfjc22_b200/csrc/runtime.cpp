@@ -184,6 +184,8 @@ CUfunction load_fn(const Launch& L, std::vector<void*>& mods) {
   // reconfigure its L1/shared split between them)
   if (const char* cv = std::getenv("FOP_CARVEOUT"); cv && *cv)
     check(cuda().func_attr(f, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, std::atoi(cv)), "cuFuncSetAttribute");
+  else if (const char* ct = std::getenv("FOP_CARVEOUT_TMA"); L.tma && ct && *ct)   // the TMA kernels only
+    check(cuda().func_attr(f, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, std::atoi(ct)), "cuFuncSetAttribute");
   mods.push_back(m);
   return f;
 }
