@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs multirank carveout carveout_tma
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs multirank carveout carveout_tma final3
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -530,6 +530,17 @@ carveout_tma)
   echo default; b
   echo tma100; FOP_CARVEOUT_TMA=100 b
   done
+  ;;
+final3)
+  # closing validation of HEAD: smoke, whole GPU suite, bench line, launch list
+  set -x
+  python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke_final3.log 2>&1; echo smoke=$?
+  tail -2 gpurun_out/smoke_final3.log
+  timeout 2400 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu_final3.log 2>&1; echo pytest=$?
+  tail -3 gpurun_out/pytest_gpu_final3.log
+  timeout 900 python bench.py > gpurun_out/bench_final3.log 2>&1; echo bench=$?
+  tail -1 gpurun_out/bench_final3.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),d['roofline']['kernel'],round(d['roofline']['frac'],3),d['clocks'],round(d['e2e']['value'],1),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
+  timeout 900 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_final3_ref.log 2>&1; echo ref=$?
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
