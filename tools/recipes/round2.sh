@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs multirank carveout carveout_tma final3
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs multirank carveout carveout_tma final3 order2
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -541,6 +541,17 @@ final3)
   timeout 900 python bench.py > gpurun_out/bench_final3.log 2>&1; echo bench=$?
   tail -1 gpurun_out/bench_final3.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),d['roofline']['kernel'],round(d['roofline']['frac'],3),d['clocks'],round(d['e2e']['value'],1),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
   timeout 900 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_final3_ref.log 2>&1; echo ref=$?
+  ;;
+order2)
+  # op-order sweep with the TMA transpose default (each order twice)
+  set -x
+  python -m paper_conf_cgo_bastoulzrlsjfjc22_b200.build >/dev/null
+  for o in cfg2,cfg3,cfg4a,cfg4b cfg2,cfg3,cfg4b,cfg4a cfg3,cfg2,cfg4a,cfg4b cfg2,cfg4a,cfg3,cfg4b cfg2,cfg4b,cfg3,cfg4a cfg3,cfg4a,cfg2,cfg4b; do
+  for i in 1 2; do
+  echo $o
+  timeout 900 python bench.py --no-cpu --no-steady --op-order $o 2>/dev/null | tail -1 | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),{k:round(v['GB_s']) for k,v in d['config']['per_op'].items()})"
+  done
+  done
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
