@@ -259,6 +259,8 @@ FOP_API fop_status  fop_plan(const fop_desc* desc, const fop_plan_opts* opts, fo
 FOP_API fop_status  fop_plan_info_get(const fop_plan_t* plan, fop_plan_info* out);
 FOP_API size_t      fop_plan_workspace_bytes(const fop_plan_t* plan);
 /* Generated CUDA source / compiled cubin of launch i (inspection, tests).
+ * fop_plan_source also takes i = -1 - k: the source of launch k's narrow
+ * variant (the kernel run for base pointers off the planned alignment).
  * Pointers stay owned by the plan. */
 FOP_API fop_status  fop_plan_source(const fop_plan_t* plan, int32_t launch, const char** src);
 FOP_API fop_status  fop_plan_cubin(const fop_plan_t* plan, int32_t launch, const void** data, size_t* size);

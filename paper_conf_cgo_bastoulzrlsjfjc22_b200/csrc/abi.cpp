@@ -208,8 +208,19 @@ size_t fop_plan_workspace_bytes(const fop_plan_t* plan) { return plan ? plan->p.
 
 fop_status fop_plan_source(const fop_plan_t* plan, int32_t i, const char** src) {
   return guarded([&] {
-    if (!plan || !src || i < 0 || i >= (int)plan->p.launches.size()) fop::fail(FOP_E_INVALID, "bad launch index");
-    *src = plan->p.launches[i].src.c_str();
+    const int n = plan ? (int)plan->p.launches.size() : 0;
+    if (!plan || !src || i < -n || i >= n) fop::fail(FOP_E_INVALID, "bad launch index");
+    if (i >= 0) {
+      *src = plan->p.launches[i].src.c_str();
+      return FOP_OK;
+    }
+    // -1 - k: the narrow (misaligned-pointer) variant of launch k, generated here if
+    // no run has needed it yet (its kernel is compiled at first use)
+    fop::Plan& p = const_cast<fop::Plan&>(plan->p);
+    std::lock_guard<std::mutex> g(p.mu);
+    fop::Launch& N = p.narrow[-1 - i];
+    if (N.src.empty()) fop::generate(p, N, -1 - i);
+    *src = N.src.c_str();
     return FOP_OK;
   });
 }

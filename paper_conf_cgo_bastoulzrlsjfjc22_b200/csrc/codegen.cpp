@@ -2721,8 +2721,10 @@ struct Gen {
       const size_t FB = ((size_t)FP * (size_t)EV0 * sizeof(float) + 255) & ~size_t(255);
       o.l("{");
       o.ind++;
-      o.l("float* F_ = (float*)(args.ws + " + num((int64_t)L.fold_off) + "ull);");
-      o.l("unsigned* fc_ = (unsigned*)(args.ws + " + num((int64_t)(L.fold_off + FB)) + "ull);");
+      // (fold_off is relative to the launch's own workspace region, which starts at
+      // ws_off: tuning candidates and the narrow variant each have a region of their own)
+      o.l("float* F_ = (float*)(args.ws + " + num((int64_t)(L.ws_off + L.fold_off)) + "ull);");
+      o.l("unsigned* fc_ = (unsigned*)(args.ws + " + num((int64_t)(L.ws_off + L.fold_off + FB)) + "ull);");
       o.l("if (rl == 0u && okc) {");
       o.l("  #pragma unroll");
       o.l("  for (int e = 0; e < " + num(W) + "; ++e) F_[iv + e] = red[cv * " + num(W) + "u + e];");

@@ -340,9 +340,10 @@ class FusedOp:
     def nlaunch(self):
         return len(self.info()["launches"])
 
-    def source(self, i=0):
+    def source(self, i=0, narrow=False):
+        """CUDA source of launch i (narrow=True: its misaligned-pointer variant)."""
         s = C.c_char_p()
-        _check(_lib.fop_plan_source(self._h, i, C.byref(s)))
+        _check(_lib.fop_plan_source(self._h, -1 - i if narrow else i, C.byref(s)))
         return s.value.decode()
 
     def cubin(self, i=0):
