@@ -2215,6 +2215,13 @@ struct Gen {
     const int64_t NCH = L.nchunks;
     const int64_t RPC = (ROWS + NCH - 1) / NCH;
     const int SW = L.gv * W;
+    // workspace address of byte `rel` of THIS launch's region (tuning candidates and the
+    // narrow variant each own a region starting at their ws_off): checked at generation
+    const auto wsa = [&](int64_t rel) {
+      if (rel < 0 || rel >= (int64_t)L.ws_bytes)
+        fail(FOP_E_INVALID, "internal: COL_REDUCE workspace offset outside the launch's region");
+      return num((int64_t)L.ws_off + rel) + "ull";
+    };
     bool isMax = x.redop == FOP_RED_MAX;
     const bool ired = x.out_dtype == FOP_I32;   // integer reduction (R30): exact, any order
     std::string init = isMax ? (ired ? "__int_as_float(0x80000000)" : "__uint_as_float(0xff800000u)")
@@ -2723,8 +2730,8 @@ struct Gen {
       o.ind++;
       // (fold_off is relative to the launch's own workspace region, which starts at
       // ws_off: tuning candidates and the narrow variant each have a region of their own)
-      o.l("float* F_ = (float*)(args.ws + " + num((int64_t)(L.ws_off + L.fold_off)) + "ull);");
-      o.l("unsigned* fc_ = (unsigned*)(args.ws + " + num((int64_t)(L.ws_off + L.fold_off + FB)) + "ull);");
+      o.l("float* F_ = (float*)(args.ws + " + wsa((int64_t)L.fold_off) + ");");
+      o.l("unsigned* fc_ = (unsigned*)(args.ws + " + wsa((int64_t)(L.fold_off + FB)) + ");");
       o.l("if (rl == 0u && okc) {");
       o.l("  #pragma unroll");
       o.l("  for (int e = 0; e < " + num(W) + "; ++e) F_[iv + e] = red[cv * " + num(W) + "u + e];");
@@ -2798,7 +2805,7 @@ struct Gen {
       // the critical path (profiles/r02/sweep_r02_colfin.log).
       const int FM = L.col_fin == 3 ? 1 : L.col_fin;   // 3: mode 1 with a pure finalizer (no rows of its own)
       const std::string OWN = FM == 1 ? "c == " + num(NCH - 1) + "u" : "false";
-      o.l("u64* partw = (u64*)(args.ws + " + num((int64_t)L.ws_off) + "ull);");
+      o.l("u64* partw = (u64*)(args.ws + " + wsa(0) + ");");
       o.l(std::string("if (rl == 0u") + (FM == 1 ? " && chunk != " + num(NCH - 1) + "u" : "") + ") {");
       o.l("  #pragma unroll");
       o.l("  for (int e = 0; e < " + num(W) + "; ++e) fop::st_relaxed_gpu_u64(&partw[(chunk * " + num(slabs) +
@@ -2807,7 +2814,7 @@ struct Gen {
       o.l("}");
       if (FM == 2) {
         size_t words = ((size_t)NCH * (size_t)slabs * (size_t)SW * 8 + 255) & ~size_t(255);
-        o.l("unsigned* cnt = (unsigned*)(args.ws + " + num((int64_t)(L.ws_off + words)) + "ull);");
+        o.l("unsigned* cnt = (unsigned*)(args.ws + " + wsa((int64_t)words) + ");");
         o.l("__syncthreads();");
         o.l("if (tid == 0u) last_flag = (atomicAdd(&cnt[slab], 1u) == " + num(NCH - 1) + "u);");
         o.l("__syncthreads();");
@@ -2885,8 +2892,8 @@ struct Gen {
     } else {
       size_t part = (size_t)NCH * (size_t)slabs * (size_t)SW * sizeof(float);
       part = (part + 255) & ~size_t(255);
-      o.l("float* part = (float*)(args.ws + " + num((int64_t)L.ws_off) + "ull);");
-      o.l("unsigned* cnt = (unsigned*)(args.ws + " + num((int64_t)(L.ws_off + part)) + "ull);");
+      o.l("float* part = (float*)(args.ws + " + wsa(0) + ");");
+      o.l("unsigned* cnt = (unsigned*)(args.ws + " + wsa((int64_t)part) + ");");
       o.l("if (rl == 0u) {");
       o.l("  #pragma unroll");
       o.l("  for (int e = 0; e < " + num(W) + "; ++e) part[(chunk * " + num(slabs) + "u + slab) * " + num(SW) +
