@@ -2,7 +2,7 @@
 # Round-2 sweep recipes: the exact command lists that produced the profiles/r02/ logs.
 # usage (on a B200, from the repo root): bash tools/recipes/round2.sh <name>
 #   e.g. gpurun --timeout 1800 -- 'bash tools/recipes/round2.sh tma'
-# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs multirank carveout carveout_tma final3 order2 final4
+# names: a b c d e f g h i j k l m n o p q r s t tma u v w x y z za zb zc zd ze zf col_fold acqrel final rowpf tune2 rowhoist suite_fuzz tma_misalign closing rowtma final2 tiebreak rowcs multirank carveout carveout_tma final3 order2 final4 final5
 case "$1" in
 a)
   bash tools/gpu_sweep_vec32.sh > gpurun_out/sweep_vec32.log 2>&1; echo sweep=$?
@@ -563,6 +563,15 @@ final4)
   timeout 900 python bench.py > gpurun_out/bench_final4.log 2>&1; echo bench=$?
   tail -1 gpurun_out/bench_final4.log | python -c "import json,sys;d=json.loads(sys.stdin.read());print(round(d['value']),round(d['ms_per_step']*1e3,1),d['roofline']['kernel'],round(d['roofline']['frac'],3),d['clocks'],round(d['e2e']['value'],1),{k:(v['kernel'],round(v['GB_s']),v['steady'] and round(v['steady']['GB_s'])) for k,v in d['config']['per_op'].items()})"
   SEEDS="62 63 64 65" COUNT=300 VARIANTS_EVERY=4 bash tools/gpu_fuzz.sh
+  ;;
+final5)
+  # the COL workspace-address helper (refactor): COL/odd/int/repeat/fuzz-regression GPU tests, fuzz 66-69, smoke
+  set -x
+  python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke_final5.log 2>&1; echo smoke=$?
+  tail -1 gpurun_out/smoke_final5.log
+  timeout 2400 python -m pytest tests/test_odd_gpu.py tests/test_int_gpu.py tests/test_repeat_runs.py tests/test_fuzz.py tests/test_full_size_gpu.py tests/test_peer.py tests/test_parity_gpu.py -q -m gpu > gpurun_out/pytest_gpu_final5.log 2>&1; echo pytest=$?
+  tail -3 gpurun_out/pytest_gpu_final5.log
+  SEEDS="66 67 68 69" COUNT=300 VARIANTS_EVERY=4 bash tools/gpu_fuzz.sh
   ;;
 *)
   echo "usage: $0 <name>  (see the names list at the top)"; exit 2
