@@ -434,3 +434,15 @@ def test_column_reduction_over_odd_rows_folds_groups_of_rows(R, C, dtype, fold):
         assert f"q = rr * {P}u" in src and f"c_ < {C}u" in src
         assert ("tr_ < " in src) == (R % P != 0)
         assert op.info()["workspace_bytes"] >= P * C * 4
+
+
+def test_narrow_variant_source_is_inspectable():
+    """fop_plan_source(plan, -1 - k, ...) returns launch k's narrow variant (the kernel run for
+    base pointers off the planned alignment): scalar accesses, its own kernel name, and for a
+    TMA-planned transpose no tensor-map path (fuzz seed 41)."""
+    op = FusedOp(W.cfg3(2, 64, 8, 8), jit=0, autotune=0)
+    assert "TRANSPOSE via TMA" in op.source(0)
+    nsrc = op.source(0, narrow=True)
+    assert "_narrow" in nsrc and "TMA" not in nsrc and "tma_load" not in nsrc
+    with pytest.raises(Exception):
+        op.source(-5)
